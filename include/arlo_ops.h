@@ -1,0 +1,69 @@
+/*
+ * arlo_ops.h — per-kernel entry points of libarlo.so, one per hot-path step of
+ * SURVEY.md §8(a).  They launch exactly the kernels the runtime graphs launch
+ * (same code, same launch configuration chooser) on plain DEVICE buffers, so
+ * tests can check each step against the oracle in isolation and bench can
+ * time one kernel.  All pointers are DEVICE pointers; `stream` is a
+ * cudaStream_t (NULL = legacy default stream); calls are asynchronous.
+ * dtype is ARLO_BF16 or ARLO_FP32 (arlo.h); in ARLO_BF16 activations and
+ * matrices are bf16 and vectors (bias, gamma, beta) fp32; in ARLO_FP32 all
+ * are fp32.  Errors: ARLO_EINVAL for bad shapes/null pointers, ARLO_ECUDA for
+ * launch failures.
+ */
+#ifndef ARLO_OPS_H_
+#define ARLO_OPS_H_
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+enum { ARLO_EPI_BIAS = 0, ARLO_EPI_BIAS_GELU = 1, ARLO_EPI_BIAS_RESIDUAL = 2 };
+
+/*
+ * Step a2/a4/a6/a7: out[M,N] = epi(A[M,K] * W[N,K]^T + bias[N]) with
+ * epi = identity | GELU_erf | (+ residual[M,N]).  Row-major, K-major operands
+ * (PyTorch Linear layout).  Requires N % 64 == 0, K % 64 == 0, 1 <= M.
+ * ARLO_BF16 runs the tcgen05/TMEM/TMA kernel; ARLO_FP32 the FFMA kernel.
+ * force_bn: 0 = automatic tile width, else 64/128/256 (tests).
+ */
+int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, const void* A, const void* W,
+                 const float* bias, const void* residual, void* out, int32_t epi,
+                 int32_t force_bn, void* stream);
+
+/* Step a5/a8: out[M,H] = LN(in[M,H]; gamma, beta, eps) per row (biased variance). */
+int arlo_op_layernorm(int32_t dtype, int32_t M, int32_t H, const void* in, const float* gamma,
+                      const float* beta, float eps, void* out, void* stream);
+
+/*
+ * Step a1: out[b*L + t] = LN(word[id] + pos[t] + type[0]) with id = ids[b,t]
+ * for t < lengths[b] and id = 0 otherwise; ids outside [0, vocab) are replaced
+ * by 0 and set *err_flag (device int32, may be NULL) to 1.
+ */
+int arlo_op_embed(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t vocab,
+                  const int32_t* ids, const int32_t* lengths, const void* word, const void* pos,
+                  const void* type, const float* gamma, const float* beta, float eps, void* out,
+                  int32_t* err_flag, void* stream);
+
+/*
+ * Step a3: padding-masked multi-head attention over a static [B, L] batch.
+ * qkv [B*L, 3H] (Q | K | V, head j at columns j*64), o [B*L, H].  Query row t
+ * of sequence b attends keys 0..lengths[b]-1 with scale 1/8; key tiles past
+ * lengths[b] are skipped; rows of a query tile lying wholly at t >=
+ * lengths[b] are written as 0 (never read by a real token).
+ */
+int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t heads, const void* qkv,
+                      const int32_t* lengths, void* o, void* stream);
+
+/*
+ * Step a9: logits[b] = W_c tanh(W_p x[b*L] + b_p) + b_c for b < B, fp32 out [B, C].
+ */
+int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, const void* x,
+                 const void* w_p, const float* b_p, const void* w_c, const float* b_c,
+                 float* logits, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ARLO_OPS_H_ */

@@ -1,0 +1,214 @@
+// embed_ln.cu — steps a1 (embedding gather + LayerNorm) and a5/a8 (LayerNorm).
+//
+// BERT embedding and post-LN LayerNorm (Devlin et al. [17], PAPER.md:L422;
+// SURVEY.md §8(a) rows a1, a5, a8; reading S3: biased variance, eps inside the
+// square root; reading S4/S7: token type 0, pad positions t >= len use id 0).
+//
+// HBM-bound: one warp per row, 128-bit loads/stores, row held in registers,
+// two-pass mean/variance from registers (no second read), warp-shuffle
+// reductions, fp32 statistics, RNE conversion to bf16.  Algorithmic bytes per
+// row: LN 2*H*sizeof(T) (+8H for gamma/beta, L2-resident); embedding
+// 3*H*sizeof(T) read (word, pos, type) + H*sizeof(T) written.
+#include "common.cuh"
+#include "kernels.h"
+
+namespace arlo {
+
+namespace {
+
+constexpr int kRowsPerBlock = 8;  // 8 warps, 256 threads
+
+template <typename T> struct Vec;
+template <> struct Vec<bf16> {
+  static constexpr int N = 8;  // 16 B
+  static __device__ __forceinline__ void load(const bf16* p, float* f) {
+    uint4 u = __ldg(reinterpret_cast<const uint4*>(p));
+    float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
+    f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
+  }
+  static __device__ __forceinline__ void store(bf16* p, const float* f) {
+    uint4 u;
+    u.x = pack_bf16x2(f[0], f[1]); u.y = pack_bf16x2(f[2], f[3]);
+    u.z = pack_bf16x2(f[4], f[5]); u.w = pack_bf16x2(f[6], f[7]);
+    *reinterpret_cast<uint4*>(p) = u;
+  }
+};
+template <> struct Vec<float> {
+  static constexpr int N = 4;
+  static __device__ __forceinline__ void load(const float* p, float* f) {
+    float4 v = __ldg(reinterpret_cast<const float4*>(p));
+    f[0] = v.x; f[1] = v.y; f[2] = v.z; f[3] = v.w;
+  }
+  static __device__ __forceinline__ void store(float* p, const float* f) {
+    *reinterpret_cast<float4*>(p) = make_float4(f[0], f[1], f[2], f[3]);
+  }
+};
+
+// Normalise the row held in v[MAXV][VN] (only vectors lane + 32 i < nvec valid) and store it.
+template <typename T, int MAXV>
+__device__ __forceinline__ void ln_finish(float (&v)[MAXV][Vec<T>::N], int nvec, int H, int lane,
+                                          const float* __restrict__ g, const float* __restrict__ b,
+                                          float eps, T* __restrict__ out_row) {
+  constexpr int VN = Vec<T>::N;
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i) {
+    if (lane + 32 * i < nvec) {
+#pragma unroll
+      for (int j = 0; j < VN; ++j) s += v[i][j];
+    }
+  }
+  const float mean = warp_sum(s) / (float)H;
+  float q = 0.f;
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i) {
+    if (lane + 32 * i < nvec) {
+#pragma unroll
+      for (int j = 0; j < VN; ++j) {
+        const float d = v[i][j] - mean;
+        q += d * d;
+      }
+    }
+  }
+  const float var = warp_sum(q) / (float)H;
+  const float rstd = 1.0f / sqrtf(var + eps);
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i) {
+    const int vi = lane + 32 * i;
+    if (vi < nvec) {
+      const int c0 = vi * VN;
+      float gg[VN], bb[VN], o[VN];
+#pragma unroll
+      for (int j = 0; j < VN; j += 4) {
+        float4 g4 = __ldg(reinterpret_cast<const float4*>(g + c0 + j));
+        float4 b4 = __ldg(reinterpret_cast<const float4*>(b + c0 + j));
+        gg[j] = g4.x; gg[j + 1] = g4.y; gg[j + 2] = g4.z; gg[j + 3] = g4.w;
+        bb[j] = b4.x; bb[j + 1] = b4.y; bb[j + 2] = b4.z; bb[j + 3] = b4.w;
+      }
+#pragma unroll
+      for (int j = 0; j < VN; ++j) o[j] = (v[i][j] - mean) * rstd * gg[j] + bb[j];
+      Vec<T>::store(out_row + c0, o);
+    }
+  }
+}
+
+template <typename T, int MAXV>
+__global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* __restrict__ in,
+                                                        const float* __restrict__ g,
+                                                        const float* __restrict__ b, float eps,
+                                                        T* __restrict__ out) {
+  constexpr int VN = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
+  if (row >= M) return;
+  const int nvec = H / VN;
+  const T* src = in + (size_t)row * H;
+  float v[MAXV][VN];
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i)
+    if (lane + 32 * i < nvec) Vec<T>::load(src + (lane + 32 * i) * VN, v[i]);
+  ln_finish<T, MAXV>(v, nvec, H, lane, g, b, eps, out + (size_t)row * H);
+}
+
+template <typename T, int MAXV>
+__global__ void __launch_bounds__(256) embed_ln_kernel(int B, int L, int H, int vocab,
+                                                       const int32_t* __restrict__ ids,
+                                                       const int32_t* __restrict__ lengths,
+                                                       const T* __restrict__ word,
+                                                       const T* __restrict__ pos,
+                                                       const T* __restrict__ type,
+                                                       const float* __restrict__ g,
+                                                       const float* __restrict__ b, float eps,
+                                                       T* __restrict__ out, int32_t* err_flag) {
+  constexpr int VN = Vec<T>::N;
+  const int lane = threadIdx.x & 31;
+  const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
+  if (row >= B * L) return;
+  const int bi = row / L, t = row - bi * L;
+  int id = 0;
+  if (t < __ldg(lengths + bi)) {
+    id = __ldg(ids + row);
+    if (id < 0 || id >= vocab) {
+      if (lane == 0 && err_flag) *err_flag = 1;
+      id = 0;
+    }
+  }
+  const int nvec = H / VN;
+  const T* wr = word + (size_t)id * H;
+  const T* pr = pos + (size_t)t * H;
+  float v[MAXV][VN];
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i) {
+    const int vi = lane + 32 * i;
+    if (vi < nvec) {
+      float a[VN], p[VN], c[VN];
+      Vec<T>::load(wr + vi * VN, a);
+      Vec<T>::load(pr + vi * VN, p);
+      Vec<T>::load(type + vi * VN, c);
+#pragma unroll
+      for (int j = 0; j < VN; ++j) v[i][j] = a[j] + p[j] + c[j];
+    }
+  }
+  ln_finish<T, MAXV>(v, nvec, H, lane, g, b, eps, out + (size_t)row * H);
+}
+
+}  // namespace
+
+#define ARLO_MAXV_SWITCH(maxv, ...)            \
+  switch (maxv) {                              \
+    case 1: { constexpr int MV = 1; __VA_ARGS__; } break; \
+    case 2: { constexpr int MV = 2; __VA_ARGS__; } break; \
+    case 3: { constexpr int MV = 3; __VA_ARGS__; } break; \
+    case 4: { constexpr int MV = 4; __VA_ARGS__; } break; \
+    case 6: { constexpr int MV = 6; __VA_ARGS__; } break; \
+    case 8: { constexpr int MV = 8; __VA_ARGS__; } break; \
+    default: return cudaErrorInvalidValue;     \
+  }
+
+static int round_maxv(int nvec) {
+  int m = (nvec + 31) / 32;
+  if (m <= 4) return m;
+  if (m <= 6) return 6;
+  if (m <= 8) return 8;
+  return -1;
+}
+
+cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float* g, const float* b,
+                             float eps, void* out, cudaStream_t s) {
+  if (M <= 0) return cudaSuccess;
+  const int vn = dt == DT_BF16 ? 8 : 4;
+  if (H % vn) return cudaErrorInvalidValue;
+  const int maxv = round_maxv(H / vn);
+  dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
+  if (dt == DT_BF16) {
+    ARLO_MAXV_SWITCH(maxv, layernorm_kernel<bf16, MV><<<grid, block, 0, s>>>(
+        M, H, (const bf16*)in, g, b, eps, (bf16*)out));
+  } else {
+    ARLO_MAXV_SWITCH(maxv, layernorm_kernel<float, MV><<<grid, block, 0, s>>>(
+        M, H, (const float*)in, g, b, eps, (float*)out));
+  }
+  return cudaGetLastError();
+}
+
+cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int32_t* ids,
+                            const int32_t* lengths, const void* word, const void* pos,
+                            const void* type, const float* g, const float* b, float eps, void* out,
+                            int32_t* err_flag, cudaStream_t s) {
+  if (B * L <= 0) return cudaSuccess;
+  const int vn = dt == DT_BF16 ? 8 : 4;
+  if (H % vn) return cudaErrorInvalidValue;
+  const int maxv = round_maxv(H / vn);
+  dim3 grid((B * L + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
+  if (dt == DT_BF16) {
+    ARLO_MAXV_SWITCH(maxv, embed_ln_kernel<bf16, MV><<<grid, block, 0, s>>>(
+        B, L, H, vocab, ids, lengths, (const bf16*)word, (const bf16*)pos, (const bf16*)type, g, b,
+        eps, (bf16*)out, err_flag));
+  } else {
+    ARLO_MAXV_SWITCH(maxv, embed_ln_kernel<float, MV><<<grid, block, 0, s>>>(
+        B, L, H, vocab, ids, lengths, (const float*)word, (const float*)pos, (const float*)type, g,
+        b, eps, (float*)out, err_flag));
+  }
+  return cudaGetLastError();
+}
+
+}  // namespace arlo

@@ -1,0 +1,321 @@
+// gemm_tc.cu — tcgen05/TMEM/TMA GEMM with fused epilogues (steps a2, a4, a6, a7).
+//
+//   out[M,N] = epi(A[M,K] W[N,K]^T + bias[N]),  epi in {identity, GELU_erf, +residual}
+//
+// The projections of every BERT layer (QKV, attention output, FFN1, FFN2;
+// Devlin et al. [17]) on the padded static shape M = b*L of a
+// per-length runtime (§3.3: "GPUs are most efficient at matrix
+// multiplication when the sequence length is a multiple of the tile size").
+//
+// Blackwell design (not a port of anything in the paper, whose runtimes are
+// TensorRT engines for sm_86):
+//  * persistent CTAs (grid = min(tiles, #SMs)), static round-robin tile order;
+//  * warp 0 = TMA producer: 128x64 A tile + BNx64 W tile per stage, 128-byte
+//    swizzle, STAGES-deep smem ring guarded by full/empty mbarriers;
+//  * warp 1 = MMA issuer: one thread issues tcgen05.mma.cta_group::1.kind::f16
+//    (M=128, N=BN, K=16) into a TMEM fp32 accumulator; tcgen05.commit frees
+//    smem stages and signals the epilogue;
+//  * warps 2-5 = epilogue: tcgen05.ld 32 lanes x 32 columns, bias / GELU /
+//    residual in fp32, RNE to bf16, 16-byte stores.  Two TMEM accumulator
+//    buffers let the epilogue of tile i overlap the main loop of tile i+1.
+// Row results never depend on M, the tile width or the grid: the K loop of
+// every output element is the same sequence of K=16 MMAs (cross-L bitwise
+// invariance, SURVEY.md §7 "Cross-L argmax agreement").
+#include <cuda.h>
+
+#include "common.cuh"
+#include "kernels.h"
+#include "ptx.cuh"
+
+namespace arlo {
+namespace {
+
+constexpr int BM = 128, BK = 64;
+constexpr int kThreads = 192;  // 6 warps
+constexpr int kAccStages = 2;
+
+template <int BN>
+struct TcCfg {
+  static constexpr int A_BYTES = BM * BK * 2;
+  static constexpr int B_BYTES = BN * BK * 2;
+  static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
+  static constexpr int TMEM_COLS = (kAccStages * BN <= 32) ? 32
+                                   : (kAccStages * BN <= 64) ? 64
+                                   : (kAccStages * BN <= 128) ? 128
+                                   : (kAccStages * BN <= 256) ? 256 : 512;
+  static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages) + 16;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + BAR_BYTES;
+};
+
+template <int BN, int EPI>
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+               int M, int N, int K, const float* __restrict__ bias, const bf16* __restrict__ resid,
+               bf16* __restrict__ out) {
+  using C = TcCfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint64_t* tempty = tfull + kAccStages;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kAccStages);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int num_m = (M + BM - 1) / BM;
+  const int num_n = N / BN;
+  const int tiles = num_m * num_n;
+  const int kblocks = K / BK;
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < kAccStages; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 4);  // one arrive per epilogue warp
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait(&empty[stage], phase ^ 1);
+          ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+          ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
+          ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ------------------------------------------------------------- MMA issuer
+    if (lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+        ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait(&full[stage], phase);
+          ptx::tc_fence_after();
+          const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+          const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            ptx::mma_bf16_ss(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
+                             ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
+          }
+          ptx::mma_commit(&empty[stage]);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+        ptx::mma_commit(&tfull[acc]);
+        if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    // --------------------------------------------------------------- epilogue
+    const int q = warp & 3;  // TMEM lane quarter this warp may access
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+      const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+      ptx::mbar_wait(&tfull[acc], acc_phase);
+      ptx::tc_fence_after();
+      const int row = m0 + q * 32 + lane;
+      const uint32_t t_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
+#pragma unroll 1
+      for (int c = 0; c < BN; c += 32) {
+        uint32_t r[32];
+        ptx::tmem_ld_32x32b_x32(t_row + c, r);
+        ptx::tmem_wait_ld();
+        if (row < M) {
+          const int col = n0 + c;
+          float v[32];
+#pragma unroll
+          for (int j = 0; j < 32; j += 4) {
+            const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + col + j));
+            v[j] = __uint_as_float(r[j]) + b4.x;
+            v[j + 1] = __uint_as_float(r[j + 1]) + b4.y;
+            v[j + 2] = __uint_as_float(r[j + 2]) + b4.z;
+            v[j + 3] = __uint_as_float(r[j + 3]) + b4.w;
+          }
+          if (EPI == EPI_BIAS_GELU) {
+#pragma unroll
+            for (int j = 0; j < 32; ++j) v[j] = gelu_erf(v[j]);
+          }
+          if (EPI == EPI_BIAS_RESID) {
+            const uint4* rp = reinterpret_cast<const uint4*>(resid + (size_t)row * N + col);
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              const uint4 u = __ldg(rp + j);
+              float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z),
+                     f3 = unpack_bf16x2(u.w);
+              v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
+              v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
+            }
+          }
+          uint4* op = reinterpret_cast<uint4*>(out + (size_t)row * N + col);
+#pragma unroll
+          for (int j = 0; j < 4; ++j) {
+            uint4 u;
+            u.x = pack_bf16x2(v[8 * j + 0], v[8 * j + 1]);
+            u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);
+            u.z = pack_bf16x2(v[8 * j + 4], v[8 * j + 5]);
+            u.w = pack_bf16x2(v[8 * j + 6], v[8 * j + 7]);
+            op[j] = u;
+          }
+        }
+      }
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+      if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+    }
+  }
+
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem_base, C::TMEM_COLS);
+  }
+}
+
+typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
+                                  const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
+                                  const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
+                                  CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode_fn() {
+  static EncodeTiledFn fn = nullptr;
+  static bool tried = false;
+  if (!tried) {
+    tried = true;
+    void* p = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<EncodeTiledFn>(p);
+  }
+  return fn;
+}
+
+template <int BN, int EPI>
+cudaError_t launch_bn_epi(const TcGemmPlan& p, cudaStream_t s) {
+  using C = TcCfg<BN>;
+  auto kern = gemm_tc_kernel<BN, EPI>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  kern<<<p.grid, kThreads, C::SMEM, s>>>(p.tmA, p.tmB, p.M, p.N, p.K, p.bias, (const bf16*)p.resid,
+                                         (bf16*)p.out);
+  return cudaGetLastError();
+}
+
+template <int BN>
+cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
+  switch (p.epi) {
+    case EPI_BIAS: return launch_bn_epi<BN, EPI_BIAS>(p, s);
+    case EPI_BIAS_GELU: return launch_bn_epi<BN, EPI_BIAS_GELU>(p, s);
+    case EPI_BIAS_RESID: return launch_bn_epi<BN, EPI_BIAS_RESID>(p, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace
+
+int num_sms() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
+  }
+  return n;
+}
+
+bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
+                         uint32_t box_inner, uint32_t box_outer) {
+  EncodeTiledFn fn = get_encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {inner * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+// Tile-width choice: a function of (M, N, K) that minimises an estimate of
+// wave-quantised time.  Per-tile time ~ max(MMA cycles, operand bytes at a
+// per-SM TMA rate) + fixed prologue/epilogue cost.
+int tc_choose_bn(int M, int N, int K) {
+  const int sms = num_sms();
+  const int num_m = (M + BM - 1) / BM;
+  double best = 1e30;
+  int best_bn = 0;
+  const int cands[3] = {256, 128, 64};
+  for (int bn : cands) {
+    if (N % bn) continue;
+    const long tiles = (long)num_m * (N / bn);
+    const long waves = (tiles + sms - 1) / sms;
+    const double mma_cyc = (double)BM * bn * K * 2 / 8192.0;          // 8192 flop/clk/SM
+    const double load_cyc = (double)(BM + bn) * K * 2 / 64.0;         // ~64 B/clk/SM TMA share
+    const double t = waves * ((mma_cyc > load_cyc ? mma_cyc : load_cyc) + 1500.0);
+    if (t < best * 0.999) { best = t; best_bn = bn; }
+  }
+  return best_bn;
+}
+
+bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
+                  const float* bias, const void* resid, void* out, int epi, int force_bn) {
+  if (M <= 0 || N % 64 || K % 64 || K <= 0) return false;
+  const int bn = force_bn ? force_bn : tc_choose_bn(M, N, K);
+  if (bn != 64 && bn != 128 && bn != 256) return false;
+  if (N % bn) return false;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->epi = epi;
+  p->bias = bias; p->resid = resid; p->out = out;
+  const int tiles = ((M + BM - 1) / BM) * (N / bn);
+  p->grid = tiles < num_sms() ? tiles : num_sms();
+  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn)) return false;
+  return true;
+}
+
+cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
+  switch (p.BN) {
+    case 64: return launch_bn<64>(p, s);
+    case 128: return launch_bn<128>(p, s);
+    case 256: return launch_bn<256>(p, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+}  // namespace arlo

@@ -1,0 +1,59 @@
+// kernels.h — host-side launchers of the hot-path kernels.
+// Every launcher is asynchronous on `stream`, takes raw device pointers and
+// returns cudaSuccess or the launch error.  No torch types anywhere.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <cuda.h>  // CUtensorMap (header only; the driver entry point is resolved at run time)
+
+namespace arlo {
+
+enum DType { DT_BF16 = 0, DT_FP32 = 1 };
+enum Epi { EPI_BIAS = 0, EPI_BIAS_GELU = 1, EPI_BIAS_RESID = 2 };
+
+int num_sms();
+
+// ---- a1: embedding + LN;  a5/a8: LN ------------------------------------------------------
+cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int32_t* ids,
+                            const int32_t* lengths, const void* word, const void* pos,
+                            const void* type, const float* g, const float* b, float eps, void* out,
+                            int32_t* err_flag, cudaStream_t s);
+cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float* g,
+                             const float* b, float eps, void* out, cudaStream_t s);
+
+// ---- a2/a4/a6/a7: GEMM + fused epilogue ----------------------------------------------------
+// tcgen05 plan: tensor maps are encoded once (at runtime create) and the
+// launch is then a plain kernel launch that CUDA graphs can capture.
+struct TcGemmPlan {
+  CUtensorMap tmA;  // activations [M, K] bf16, box {64, 128}, 128B swizzle
+  CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN}, 128B swizzle
+  int M, N, K, BN, epi, grid;
+  const float* bias;
+  const void* resid;
+  void* out;
+};
+bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
+                  const float* bias, const void* resid, void* out, int epi, int force_bn);
+cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s);
+int tc_choose_bn(int M, int N, int K);
+
+cudaError_t launch_gemm_simt(DType dt, int M, int N, int K, const void* A, const void* W,
+                             const float* bias, const void* resid, void* out, int epi,
+                             cudaStream_t s);
+
+// ---- a3: masked attention -----------------------------------------------------------------
+cudaError_t launch_attention(DType dt, int B, int L, int heads, const void* qkv,
+                             const int32_t* lengths, void* o, cudaStream_t s);
+
+// ---- a9: CLS pooler + classifier ----------------------------------------------------------
+cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p,
+                        const float* b_p, const void* w_c, const float* b_c, float* logits,
+                        cudaStream_t s);
+
+// Resolve cuTensorMapEncodeTiled through the runtime (no link-time libcuda dependency).
+bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
+                         uint32_t box_inner, uint32_t box_outer);
+
+}  // namespace arlo

@@ -1,0 +1,504 @@
+// runtime.cu — per-length runtime (K9: CUDA-graph runtime builder) and the C ABI.
+//
+// A runtime is the B200 counterpart of one statically compiled engine of
+// Arlo's polymorphing: the model "compiled into multiple runtimes, each with a
+// different max_length" (PAPER.md:L123 step 2), one static (batch, length)
+// shape each (L77 §2.1).  Here "compile" = allocate a graph-stable activation
+// arena for (max_batch, L), encode the TMA descriptors of every GEMM once, and
+// capture one CUDA graph per batch bucket b in {1, 2, 4, ..., max_batch}.  A
+// request batch is served by copying ids/lengths into the arena and replaying
+// the graph of the smallest bucket b >= n (one launch instead of 2 + 7*layers).
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <mutex>
+#include <new>
+#include <string>
+#include <vector>
+
+#include "../../include/arlo.h"
+#include "../../include/arlo_ops.h"
+#include "errors.h"
+#include "kernels.h"
+
+namespace arlo {
+
+namespace {
+thread_local std::string g_err;
+}
+
+int set_error(int code, const char* fmt, ...) {
+  char buf[512];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof buf, fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return code;
+}
+void clear_error() { g_err.clear(); }
+
+static int cuda_fail(cudaError_t e, const char* what) {
+  return set_error(ARLO_ECUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
+}
+
+#define ARLO_CUDA(call, what)                    \
+  do {                                           \
+    cudaError_t e_ = (call);                     \
+    if (e_ != cudaSuccess) return cuda_fail(e_, what); \
+  } while (0)
+
+struct DeviceGuard {
+  int prev = -1;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) != cudaSuccess) prev = -1;
+    if (prev != dev) cudaSetDevice(dev);
+  }
+  ~DeviceGuard() {
+    int cur = -1;
+    if (prev >= 0 && cudaGetDevice(&cur) == cudaSuccess && cur != prev) cudaSetDevice(prev);
+  }
+};
+
+static int check_device(int device) {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess || n <= 0) return set_error(ARLO_ENODEV, "no CUDA device");
+  if (device < 0 || device >= n) return set_error(ARLO_ENODEV, "device %d out of range (%d devices)", device, n);
+  cudaDeviceProp p;
+  if (cudaGetDeviceProperties(&p, device) != cudaSuccess) return set_error(ARLO_ENODEV, "cudaGetDeviceProperties failed");
+  if (p.major != 10 || p.minor != 0)
+    return set_error(ARLO_ENODEV, "device %d is sm_%d%d; libarlo is built for sm_100a (B200) only", device, p.major,
+                     p.minor);
+  return ARLO_OK;
+}
+
+}  // namespace arlo
+
+using namespace arlo;
+
+// ------------------------------------------------------------------------ weights
+struct arlo_weights {
+  int device;
+  arlo_model_config cfg;
+  std::vector<const void*> t;  // canonical order
+  const void* word() const { return t[0]; }
+  const void* pos() const { return t[1]; }
+  const void* type() const { return t[2]; }
+  const float* emb_g() const { return (const float*)t[3]; }
+  const float* emb_b() const { return (const float*)t[4]; }
+  const void* lt(int layer, int k) const { return t[5 + 12 * layer + k]; }
+  const void* hd(int k) const { return t[5 + 12 * cfg.layers + k]; }
+};
+
+enum { LW_QKV = 0, LB_QKV, LW_O, LB_O, LN1_G, LN1_B, LW_1, LB_1, LW_2, LB_2, LN2_G, LN2_B };
+
+extern "C" const char* arlo_last_error(void) { return g_err.c_str(); }
+extern "C" const char* arlo_version(void) { return "arlo-b200 0.1 (sm_100a)"; }
+
+extern "C" int32_t arlo_weights_count(const arlo_model_config* cfg) {
+  return cfg ? 5 + 12 * cfg->layers + 4 : ARLO_EINVAL;
+}
+
+static int validate_cfg(const arlo_model_config* c) {
+  if (!c) return set_error(ARLO_EINVAL, "null config");
+  if (c->layers < 1 || c->hidden < 64 || c->heads < 1 || c->hidden != 64 * c->heads)
+    return set_error(ARLO_EINVAL, "config: need hidden == 64 * heads (head dim 64), layers >= 1");
+  if (c->hidden % 64 || c->ffn % 64 || c->ffn < 64)
+    return set_error(ARLO_EINVAL, "config: hidden and ffn must be multiples of 64");
+  if (c->hidden > 2048) return set_error(ARLO_EINVAL, "config: hidden > 2048 unsupported");
+  if (c->vocab < 1 || c->max_pos < 16 || c->type_vocab < 1 || c->num_labels < 1 || c->num_labels > 64)
+    return set_error(ARLO_EINVAL, "config: bad vocab/max_pos/type_vocab/num_labels");
+  if (c->dtype != ARLO_BF16 && c->dtype != ARLO_FP32) return set_error(ARLO_EINVAL, "config: bad dtype");
+  if (!(c->ln_eps > 0)) return set_error(ARLO_EINVAL, "config: ln_eps must be > 0");
+  return ARLO_OK;
+}
+
+extern "C" int arlo_weights_create(int32_t device, const arlo_model_config* cfg, const void* const* tensors,
+                                   int32_t n_tensors, arlo_weights** out) {
+  clear_error();
+  if (!out || !tensors) return set_error(ARLO_EINVAL, "arlo_weights_create: null argument");
+  int rc = validate_cfg(cfg);
+  if (rc) return rc;
+  if (n_tensors != arlo_weights_count(cfg))
+    return set_error(ARLO_EINVAL, "arlo_weights_create: expected %d tensors, got %d", arlo_weights_count(cfg), n_tensors);
+  if ((rc = check_device(device))) return rc;
+  for (int i = 0; i < n_tensors; ++i) {
+    if (!tensors[i] || (reinterpret_cast<uintptr_t>(tensors[i]) & 15))
+      return set_error(ARLO_EINVAL, "arlo_weights_create: tensor %d is null or not 16-byte aligned", i);
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, tensors[i]) != cudaSuccess || (a.type != cudaMemoryTypeDevice && a.type != cudaMemoryTypeManaged)) {
+      cudaGetLastError();
+      return set_error(ARLO_EINVAL, "arlo_weights_create: tensor %d is not device memory", i);
+    }
+  }
+  arlo_weights* w = new (std::nothrow) arlo_weights;
+  if (!w) return set_error(ARLO_ENOMEM, "out of host memory");
+  w->device = device;
+  w->cfg = *cfg;
+  w->t.assign(tensors, tensors + n_tensors);
+  *out = w;
+  return ARLO_OK;
+}
+
+extern "C" void arlo_weights_destroy(arlo_weights* w) { delete w; }
+
+// ------------------------------------------------------------------------ runtime
+struct LayerPlans {
+  TcGemmPlan qkv, o, f1, f2;
+};
+
+struct Bucket {
+  int b = 0;
+  std::vector<LayerPlans> plans;  // bf16 only
+  cudaGraphExec_t exec = nullptr;
+  size_t nodes = 0;
+};
+
+struct arlo_runtime {
+  int L = 0, max_batch = 0, device = 0;
+  const arlo_weights* w = nullptr;
+  DType dt = DT_BF16;
+  cudaStream_t own_stream = nullptr, stream = nullptr;
+  // arena (one allocation)
+  void* arena = nullptr;
+  int32_t* err = nullptr;      // [1]
+  int32_t* lengths = nullptr;  // [max_batch]  (err, lengths, ids are contiguous: one staging copy)
+  int32_t* ids = nullptr;      // [max_batch * L]
+  float* logits = nullptr;     // [max_batch * C]
+  void *X = nullptr, *QKV = nullptr, *O = nullptr, *Y = nullptr, *F = nullptr;
+  // pinned host staging
+  void* h_stage = nullptr;
+  size_t h_stage_bytes = 0;
+  std::vector<Bucket> buckets;
+};
+
+static int bucket_index(const arlo_runtime* rt, int n) {
+  for (size_t i = 0; i < rt->buckets.size(); ++i)
+    if (rt->buckets[i].b >= n) return (int)i;
+  return -1;
+}
+
+// Enqueue one forward at bucket size b (the body every graph captures).
+static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
+  const arlo_weights* w = rt->w;
+  const arlo_model_config& c = w->cfg;
+  const int b = bk.b, L = rt->L, H = c.hidden, F = c.ffn, M = b * L;
+  const DType dt = rt->dt;
+  ARLO_CUDA(launch_embed_ln(dt, b, L, H, c.vocab, rt->ids, rt->lengths, w->word(), w->pos(), w->type(), w->emb_g(),
+                            w->emb_b(), c.ln_eps, rt->X, rt->err, s),
+            "embed_ln launch");
+  for (int l = 0; l < c.layers; ++l) {
+    if (dt == DT_BF16) {
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].qkv, s), "qkv gemm launch");
+    } else {
+      ARLO_CUDA(launch_gemm_simt(dt, M, 3 * H, H, rt->X, w->lt(l, LW_QKV), (const float*)w->lt(l, LB_QKV), nullptr,
+                                 rt->QKV, EPI_BIAS, s),
+                "qkv gemm launch");
+    }
+    ARLO_CUDA(launch_attention(dt, b, L, c.heads, rt->QKV, rt->lengths, rt->O, s), "attention launch");
+    if (dt == DT_BF16) {
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].o, s), "out-proj gemm launch");
+    } else {
+      ARLO_CUDA(launch_gemm_simt(dt, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y,
+                                 EPI_BIAS_RESID, s),
+                "out-proj gemm launch");
+    }
+    ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
+                               c.ln_eps, rt->X, s),
+              "ln1 launch");
+    if (dt == DT_BF16) {
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].f1, s), "ffn1 gemm launch");
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].f2, s), "ffn2 gemm launch");
+    } else {
+      ARLO_CUDA(launch_gemm_simt(dt, M, F, H, rt->X, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, rt->F,
+                                 EPI_BIAS_GELU, s),
+                "ffn1 gemm launch");
+      ARLO_CUDA(launch_gemm_simt(dt, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
+                                 EPI_BIAS_RESID, s),
+                "ffn2 gemm launch");
+    }
+    ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
+                               c.ln_eps, rt->X, s),
+              "ln2 launch");
+  }
+  ARLO_CUDA(launch_head(dt, b, L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
+                        (const float*)w->hd(3), rt->logits, s),
+            "head launch");
+  return ARLO_OK;
+}
+
+static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
+  const arlo_weights* w = rt->w;
+  const arlo_model_config& c = w->cfg;
+  const int M = bk.b * rt->L, H = c.hidden, F = c.ffn;
+  bk.plans.resize(c.layers);
+  for (int l = 0; l < c.layers; ++l) {
+    LayerPlans& p = bk.plans[l];
+    bool ok = tc_plan_gemm(&p.qkv, M, 3 * H, H, rt->X, w->lt(l, LW_QKV), (const float*)w->lt(l, LB_QKV), nullptr,
+                           rt->QKV, EPI_BIAS, 0) &&
+              tc_plan_gemm(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y,
+                           EPI_BIAS_RESID, 0) &&
+              tc_plan_gemm(&p.f1, M, F, H, rt->X, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, rt->F,
+                           EPI_BIAS_GELU, 0) &&
+              tc_plan_gemm(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
+                           EPI_BIAS_RESID, 0);
+    if (!ok) return set_error(ARLO_ECUDA, "tensor-map encoding failed (cuTensorMapEncodeTiled unavailable?)");
+  }
+  return ARLO_OK;
+}
+
+static void destroy_runtime(arlo_runtime* rt) {
+  if (!rt) return;
+  for (auto& bk : rt->buckets)
+    if (bk.exec) cudaGraphExecDestroy(bk.exec);
+  if (rt->arena) cudaFree(rt->arena);
+  if (rt->h_stage) cudaFreeHost(rt->h_stage);
+  if (rt->own_stream) cudaStreamDestroy(rt->own_stream);
+  delete rt;
+}
+
+extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out) {
+  clear_error();
+  if (!w || !out) return set_error(ARLO_EINVAL, "arlo_runtime_create: null argument");
+  const arlo_model_config& c = w->cfg;
+  if (L < 16 || L % 16 || L > c.max_pos)
+    return set_error(ARLO_EINVAL, "arlo_runtime_create: need 16 <= L <= max_pos (%d) and L %% 16 == 0, got %d", c.max_pos, L);
+  if (max_batch < 1 || max_batch > 64) return set_error(ARLO_EINVAL, "arlo_runtime_create: need 1 <= max_batch <= 64");
+  DeviceGuard g(w->device);
+  arlo_runtime* rt = new (std::nothrow) arlo_runtime;
+  if (!rt) return set_error(ARLO_ENOMEM, "out of host memory");
+  rt->L = L;
+  rt->max_batch = max_batch;
+  rt->w = w;
+  rt->device = w->device;
+  rt->dt = c.dtype == ARLO_BF16 ? DT_BF16 : DT_FP32;
+  auto fail = [&](int code) { destroy_runtime(rt); return code; };
+  cudaError_t e = cudaStreamCreateWithFlags(&rt->own_stream, cudaStreamNonBlocking);
+  if (e != cudaSuccess) return fail(cuda_fail(e, "cudaStreamCreate"));
+  rt->stream = rt->own_stream;
+
+  const size_t es = rt->dt == DT_BF16 ? 2 : 4;
+  const size_t Mmax = (size_t)max_batch * L, H = c.hidden, F = c.ffn;
+  auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+  const size_t off_err = 0;
+  const size_t off_len = 16;  // err (int32) then lengths then ids, contiguous
+  const size_t off_ids = off_len + 4 * (size_t)max_batch;
+  size_t off = al(off_ids + 4 * Mmax);
+  const size_t off_logits = off; off = al(off + 4 * (size_t)max_batch * c.num_labels);
+  const size_t off_X = off; off = al(off + es * Mmax * H);
+  const size_t off_QKV = off; off = al(off + es * Mmax * 3 * H);
+  const size_t off_O = off; off = al(off + es * Mmax * H);
+  const size_t off_Y = off; off = al(off + es * Mmax * H);
+  const size_t off_F = off; off = al(off + es * Mmax * F);
+  e = cudaMalloc(&rt->arena, off);
+  if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "arena of %zu bytes: %s", off, cudaGetErrorString(e)));
+  e = cudaMemset(rt->arena, 0, off);
+  if (e != cudaSuccess) return fail(cuda_fail(e, "arena memset"));
+  char* a = (char*)rt->arena;
+  rt->err = (int32_t*)(a + off_err);
+  rt->lengths = (int32_t*)(a + off_len);
+  rt->ids = (int32_t*)(a + off_ids);
+  rt->logits = (float*)(a + off_logits);
+  rt->X = a + off_X; rt->QKV = a + off_QKV; rt->O = a + off_O; rt->Y = a + off_Y; rt->F = a + off_F;
+  rt->h_stage_bytes = off_ids + 4 * Mmax + 4 * (size_t)max_batch * c.num_labels + 64;
+  e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
+  if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "pinned staging: %s", cudaGetErrorString(e)));
+
+  // batch buckets 1, 2, 4, ..., max_batch
+  std::vector<int> bs;
+  for (int b = 1; b < max_batch; b *= 2) bs.push_back(b);
+  bs.push_back(max_batch);
+  rt->buckets.resize(bs.size());
+  for (size_t i = 0; i < bs.size(); ++i) {
+    Bucket& bk = rt->buckets[i];
+    bk.b = bs[i];
+    if (rt->dt == DT_BF16) {
+      int rc = plan_bucket(rt, bk);
+      if (rc) return fail(rc);
+    }
+    cudaGraph_t graph = nullptr;
+    e = cudaStreamBeginCapture(rt->own_stream, cudaStreamCaptureModeThreadLocal);
+    if (e != cudaSuccess) return fail(cuda_fail(e, "cudaStreamBeginCapture"));
+    int rc = enqueue_forward(rt, bk, rt->own_stream);
+    cudaError_t e2 = cudaStreamEndCapture(rt->own_stream, &graph);
+    if (rc) { if (graph) cudaGraphDestroy(graph); return fail(rc); }
+    if (e2 != cudaSuccess) return fail(cuda_fail(e2, "cudaStreamEndCapture"));
+    cudaGraphGetNodes(graph, nullptr, &bk.nodes);
+    e = cudaGraphInstantiate(&bk.exec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) return fail(cuda_fail(e, "cudaGraphInstantiate"));
+    e = cudaGraphUpload(bk.exec, rt->own_stream);
+    if (e != cudaSuccess) return fail(cuda_fail(e, "cudaGraphUpload"));
+  }
+  e = cudaStreamSynchronize(rt->own_stream);
+  if (e != cudaSuccess) return fail(cuda_fail(e, "runtime create sync"));
+  *out = rt;
+  return ARLO_OK;
+}
+
+extern "C" void arlo_runtime_destroy(arlo_runtime* rt) {
+  if (!rt) return;
+  DeviceGuard g(rt->device);
+  cudaStreamSynchronize(rt->stream);
+  destroy_runtime(rt);
+}
+
+extern "C" int arlo_runtime_set_stream(arlo_runtime* rt, void* stream) {
+  if (!rt) return set_error(ARLO_EINVAL, "null runtime");
+  rt->stream = stream ? (cudaStream_t)stream : rt->own_stream;
+  return ARLO_OK;
+}
+
+extern "C" int32_t arlo_runtime_length(const arlo_runtime* rt) { return rt ? rt->L : ARLO_EINVAL; }
+extern "C" int32_t arlo_runtime_max_batch(const arlo_runtime* rt) { return rt ? rt->max_batch : ARLO_EINVAL; }
+
+extern "C" int32_t arlo_runtime_kernel_count(const arlo_runtime* rt, int32_t n) {
+  if (!rt) return ARLO_EINVAL;
+  int bi = bucket_index(rt, n < 1 ? 1 : n);
+  return bi < 0 ? ARLO_EINVAL : (int32_t)rt->buckets[bi].nodes;
+}
+
+static bool is_device_ptr(const void* p) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  return a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged;
+}
+
+extern "C" int arlo_infer(arlo_runtime* rt, const int32_t* token_ids, const int32_t* lengths, float* logits) {
+  clear_error();
+  if (!rt || !token_ids || !lengths || !logits) return set_error(ARLO_EINVAL, "arlo_infer: null argument");
+  DeviceGuard g(rt->device);
+  const int L = rt->L, mb = rt->max_batch, C = rt->w->cfg.num_labels, V = rt->w->cfg.vocab;
+  cudaStream_t s = rt->stream;
+  const bool ids_dev = is_device_ptr(token_ids), len_dev = is_device_ptr(lengths), out_dev = is_device_ptr(logits);
+  // staging layout mirrors the arena: [err(16 B) | lengths[mb] | ids[mb*L] | logits[mb*C]]
+  char* hs = (char*)rt->h_stage;
+  int32_t* h_err = (int32_t*)hs;
+  int32_t* h_len = (int32_t*)(hs + 16);
+  int32_t* h_ids = h_len + mb;
+  float* h_logits = (float*)(h_ids + (size_t)mb * L);
+  if (len_dev) {
+    ARLO_CUDA(cudaMemcpyAsync(h_len, lengths, 4 * (size_t)mb, cudaMemcpyDeviceToHost, s), "lengths D2H");
+    ARLO_CUDA(cudaStreamSynchronize(s), "lengths sync");
+  } else {
+    memcpy(h_len, lengths, 4 * (size_t)mb);
+  }
+  int n = 0;
+  while (n < mb && h_len[n] > 0) ++n;
+  for (int i = 0; i < n; ++i)
+    if (h_len[i] > L) return set_error(ARLO_ETOOLONG, "arlo_infer: request %d has length %d > L = %d", i, h_len[i], L);
+  if (n == 0) return ARLO_OK;
+  const int bi = bucket_index(rt, n);
+  Bucket& bk = rt->buckets[bi];
+  for (int i = n; i < bk.b; ++i) h_len[i] = 0;
+  *h_err = 0;
+  if (!ids_dev) {
+    for (int i = 0; i < n; ++i) {
+      const int32_t* row = token_ids + (size_t)i * L;
+      for (int t = 0; t < h_len[i]; ++t)
+        if (row[t] < 0 || row[t] >= V)
+          return set_error(ARLO_EINVAL, "arlo_infer: token id %d at [%d,%d] outside [0, %d)", row[t], i, t, V);
+    }
+    memcpy(h_ids, token_ids, 4 * (size_t)n * L);
+    ARLO_CUDA(cudaMemcpyAsync(rt->err, h_err, 16 + 4 * (size_t)mb + 4 * (size_t)n * L, cudaMemcpyHostToDevice, s),
+              "inputs H2D");
+  } else {
+    ARLO_CUDA(cudaMemcpyAsync(rt->err, h_err, 16 + 4 * (size_t)mb, cudaMemcpyHostToDevice, s), "lengths H2D");
+    ARLO_CUDA(cudaMemcpyAsync(rt->ids, token_ids, 4 * (size_t)n * L, cudaMemcpyDeviceToDevice, s), "ids D2D");
+  }
+  ARLO_CUDA(cudaGraphLaunch(bk.exec, s), "cudaGraphLaunch");
+  if (out_dev) {
+    ARLO_CUDA(cudaMemcpyAsync(logits, rt->logits, 4 * (size_t)n * C, cudaMemcpyDeviceToDevice, s), "logits D2D");
+  } else {
+    ARLO_CUDA(cudaMemcpyAsync(h_logits, rt->logits, 4 * (size_t)n * C, cudaMemcpyDeviceToHost, s), "logits D2H");
+  }
+  ARLO_CUDA(cudaMemcpyAsync(h_err, rt->err, 4, cudaMemcpyDeviceToHost, s), "err D2H");
+  ARLO_CUDA(cudaStreamSynchronize(s), "arlo_infer sync");
+  if (*h_err) return set_error(ARLO_EINVAL, "arlo_infer: a token id at t < length is outside [0, %d)", V);
+  if (!out_dev) memcpy(logits, h_logits, 4 * (size_t)n * C);
+  return ARLO_OK;
+}
+
+extern "C" int arlo_enqueue(arlo_runtime* rt, int32_t n, const int32_t* token_ids, const int32_t* lengths,
+                            float* logits) {
+  if (!rt || !token_ids || !lengths || !logits) return set_error(ARLO_EINVAL, "arlo_enqueue: null argument");
+  if (n < 1 || n > rt->max_batch) return set_error(ARLO_EINVAL, "arlo_enqueue: need 1 <= n <= max_batch");
+  DeviceGuard g(rt->device);
+  cudaStream_t s = rt->stream;
+  const int bi = bucket_index(rt, n);
+  Bucket& bk = rt->buckets[bi];
+  const int L = rt->L, C = rt->w->cfg.num_labels;
+  ARLO_CUDA(cudaMemcpyAsync(rt->lengths, lengths, 4 * (size_t)n, cudaMemcpyDeviceToDevice, s), "lengths D2D");
+  if (bk.b > n) ARLO_CUDA(cudaMemsetAsync(rt->lengths + n, 0, 4 * (size_t)(bk.b - n), s), "lengths pad");
+  ARLO_CUDA(cudaMemcpyAsync(rt->ids, token_ids, 4 * (size_t)n * L, cudaMemcpyDeviceToDevice, s), "ids D2D");
+  ARLO_CUDA(cudaGraphLaunch(bk.exec, s), "cudaGraphLaunch");
+  ARLO_CUDA(cudaMemcpyAsync(logits, rt->logits, 4 * (size_t)n * C, cudaMemcpyDeviceToDevice, s), "logits D2D");
+  return ARLO_OK;
+}
+
+// ------------------------------------------------------------------------ ops ABI
+static DType to_dt(int32_t d) { return d == ARLO_FP32 ? DT_FP32 : DT_BF16; }
+
+extern "C" int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, const void* A, const void* W,
+                            const float* bias, const void* residual, void* out, int32_t epi, int32_t force_bn,
+                            void* stream) {
+  clear_error();
+  if (M < 1 || N % 64 || K % 64 || N < 64 || K < 64 || !A || !W || !bias || !out || epi < 0 || epi > 2 ||
+      (epi == ARLO_EPI_BIAS_RESIDUAL && !residual))
+    return set_error(ARLO_EINVAL, "arlo_op_gemm: bad arguments");
+  cudaStream_t s = (cudaStream_t)stream;
+  if (dtype == ARLO_BF16) {
+    TcGemmPlan p;
+    if (!tc_plan_gemm(&p, M, N, K, A, W, bias, residual, out, epi, force_bn))
+      return set_error(ARLO_EINVAL, "arlo_op_gemm: plan failed (tile width %d / tensor map)", force_bn);
+    ARLO_CUDA(tc_launch_gemm(p, s), "tcgen05 gemm");
+  } else {
+    ARLO_CUDA(launch_gemm_simt(DT_FP32, M, N, K, A, W, bias, residual, out, epi, s), "simt gemm");
+  }
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_layernorm(int32_t dtype, int32_t M, int32_t H, const void* in, const float* gamma,
+                                 const float* beta, float eps, void* out, void* stream) {
+  clear_error();
+  if (M < 0 || H < 8 || H % 8 || !in || !gamma || !beta || !out) return set_error(ARLO_EINVAL, "arlo_op_layernorm: bad arguments");
+  ARLO_CUDA(launch_layernorm(to_dt(dtype), M, H, in, gamma, beta, eps, out, (cudaStream_t)stream), "layernorm");
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_embed(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t vocab, const int32_t* ids,
+                             const int32_t* lengths, const void* word, const void* pos, const void* type,
+                             const float* gamma, const float* beta, float eps, void* out, int32_t* err_flag,
+                             void* stream) {
+  clear_error();
+  if (B < 0 || L < 1 || H < 8 || H % 8 || vocab < 1 || !ids || !lengths || !word || !pos || !type || !out)
+    return set_error(ARLO_EINVAL, "arlo_op_embed: bad arguments");
+  ARLO_CUDA(launch_embed_ln(to_dt(dtype), B, L, H, vocab, ids, lengths, word, pos, type, gamma, beta, eps, out,
+                            err_flag, (cudaStream_t)stream),
+            "embed");
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t heads, const void* qkv,
+                                 const int32_t* lengths, void* o, void* stream) {
+  clear_error();
+  if (B < 0 || L < 1 || heads < 1 || !qkv || !lengths || !o) return set_error(ARLO_EINVAL, "arlo_op_attention: bad arguments");
+  ARLO_CUDA(launch_attention(to_dt(dtype), B, L, heads, qkv, lengths, o, (cudaStream_t)stream), "attention");
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, const void* x,
+                            const void* w_p, const float* b_p, const void* w_c, const float* b_c, float* logits,
+                            void* stream) {
+  clear_error();
+  if (B < 0 || L < 1 || H < 8 || H % 8 || C < 1 || !x || !w_p || !b_p || !w_c || !b_c || !logits)
+    return set_error(ARLO_EINVAL, "arlo_op_head: bad arguments");
+  ARLO_CUDA(launch_head(to_dt(dtype), B, L, H, C, x, w_p, b_p, w_c, b_c, logits, (cudaStream_t)stream), "head");
+  return ARLO_OK;
+}

@@ -28,3 +28,12 @@ def pytest_collection_modifyitems(config, items):
     for item in items:
         if "gpu" in item.keywords:
             item.add_marker(skip)
+
+
+@pytest.fixture(scope="session")
+def arlo_lib():
+    """Build libarlo.so if missing or stale (nvcc cross-compiles without a GPU), then load it."""
+    from paper_conf_icpp_tanlyl024_b200 import build
+    build.build()
+    from paper_conf_icpp_tanlyl024_b200 import arlo
+    return arlo

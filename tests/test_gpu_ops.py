@@ -1,0 +1,197 @@
+"""Per-kernel parity of the CUDA path (through the C ABI, arlo_op_*) against the
+oracle's per-step functions, element by element (needs a B200)."""
+import numpy as np
+import pytest
+import torch
+
+from oracle import encoder as orc
+from paper_conf_icpp_tanlyl024_b200 import workload as wl
+
+pytestmark = pytest.mark.gpu
+
+
+def bf16_dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float32)).to("cuda", torch.bfloat16)
+
+
+def f32_dev(a):
+    return torch.from_numpy(np.ascontiguousarray(a, np.float32)).to("cuda")
+
+
+def host64(t):
+    return t.float().cpu().numpy().astype(np.float64)
+
+
+def rnd(shape, seed, std=1.0):
+    return wl.round_to_bf16(np.random.default_rng(seed).standard_normal(shape).astype(np.float32) * std)
+
+
+# --------------------------------------------------------------------------- GEMM
+GEMM_SHAPES = [
+    (64, 2304, 768), (200, 768, 768), (384, 3072, 768), (333, 768, 3072),  # ragged M tails
+    (1024, 1024, 1024), (128, 128, 128), (32, 384, 128), (4096, 2304, 768),
+]
+
+
+@pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
+@pytest.mark.parametrize("epi", [0, 1, 2])
+def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi):
+    A = rnd((M, K), 1)
+    W = rnd((N, K), 2, 0.02)
+    b = rnd((N,), 3, 0.02)
+    R = rnd((M, N), 4)
+    ref = orc.linear(A, W, b)
+    if epi == 1:
+        ref = orc.gelu(ref)
+    if epi == 2:
+        ref = ref + R
+    out = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_gemm(arlo_lib.BF16, bf16_dev(A), bf16_dev(W), f32_dev(b), out, epi=epi,
+                     residual=bf16_dev(R) if epi == 2 else None)
+    torch.cuda.synchronize()
+    got = host64(out)
+    # bf16 output rounding (2^-9 relative) on fp32-accumulated exact products
+    np.testing.assert_allclose(got, ref, rtol=8e-3, atol=8e-3)
+
+
+@pytest.mark.parametrize("bn", [64, 128, 256])
+def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
+    """Row results do not depend on the tile width (cross-L invariance contract)."""
+    M, N, K = 300, 768, 768
+    A, W, b = bf16_dev(rnd((M, K), 5)), bf16_dev(rnd((N, K), 6, 0.02)), f32_dev(rnd((N,), 7, 0.02))
+    outs = []
+    for force in (bn, 0):
+        o = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
+        arlo_lib.op_gemm(arlo_lib.BF16, A, W, b, o, epi=0, force_bn=force)
+        outs.append(o)
+    torch.cuda.synchronize()
+    assert torch.equal(outs[0], outs[1])
+    # and a row does not depend on M (prefix of rows)
+    o2 = torch.empty((77, N), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_gemm(arlo_lib.BF16, A[:77].contiguous(), W, b, o2, epi=0, force_bn=bn)
+    torch.cuda.synchronize()
+    assert torch.equal(o2, outs[0][:77])
+
+
+@pytest.mark.parametrize("M,N,K", [(100, 384, 128), (64, 128, 512), (257, 192, 64)])
+@pytest.mark.parametrize("epi", [0, 1, 2])
+def test_gemm_fp32_check_mode(arlo_lib, M, N, K, epi):
+    rng = np.random.default_rng(M + N + K)
+    A = rng.standard_normal((M, K)).astype(np.float32)
+    W = (rng.standard_normal((N, K)) * 0.05).astype(np.float32)
+    b = (rng.standard_normal(N) * 0.05).astype(np.float32)
+    R = rng.standard_normal((M, N)).astype(np.float32)
+    ref = orc.linear(A, W, b)
+    if epi == 1:
+        ref = orc.gelu(ref)
+    if epi == 2:
+        ref = ref + R
+    out = torch.empty((M, N), device="cuda", dtype=torch.float32)
+    arlo_lib.op_gemm(arlo_lib.FP32, f32_dev(A), f32_dev(W), f32_dev(b), out, epi=epi,
+                     residual=f32_dev(R) if epi == 2 else None)
+    torch.cuda.synchronize()
+    np.testing.assert_allclose(host64(out), ref, rtol=0, atol=2e-5)
+
+
+# ---------------------------------------------------------------------- LayerNorm
+@pytest.mark.parametrize("H", [128, 768, 1024])
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_layernorm(arlo_lib, H, dtype):
+    M = 257
+    x = rnd((M, H), H) * 3 + 1
+    g = rnd((H,), 1, 0.1) + 1
+    b = rnd((H,), 2, 0.02)
+    ref = orc.layer_norm(x, g, b, 1e-12)
+    dev = bf16_dev if dtype == 0 else f32_dev
+    out = torch.empty((M, H), device="cuda", dtype=torch.bfloat16 if dtype == 0 else torch.float32)
+    arlo_lib.op_layernorm(dtype, dev(x), f32_dev(g), f32_dev(b), 1e-12, out)
+    torch.cuda.synchronize()
+    tol = 2e-2 if dtype == 0 else 1e-5
+    np.testing.assert_allclose(host64(out), ref, rtol=0, atol=tol)
+
+
+# ---------------------------------------------------------------------- embedding
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_embedding_ln(arlo_lib, dtype):
+    cfg = wl.BERT_BASE
+    w = wl.make_weights(wl.ModelConfig("emb", 1, 768, 12, 3072, 2000), seed=1)
+    L = 96
+    lengths = np.array([96, 1, 50, 0], np.int32)
+    ids = wl.sample_token_ids(wl.ModelConfig("emb", 1, 768, 12, 3072, 2000), lengths, L, seed=3)
+    ids_garbage = ids.copy()
+    ids_garbage[2, 50:] = 123456  # beyond len: ignored, no error
+    dev = bf16_dev if dtype == 0 else f32_dev
+    out = torch.empty((4 * L, 768), device="cuda", dtype=torch.bfloat16 if dtype == 0 else torch.float32)
+    err = torch.zeros(1, dtype=torch.int32, device="cuda")
+    arlo_lib.op_embed(dtype, torch.from_numpy(ids_garbage).cuda(), torch.from_numpy(lengths).cuda(),
+                      dev(w["word_emb"]), dev(w["pos_emb"]), dev(w["type_emb"]), f32_dev(w["emb_ln_g"]),
+                      f32_dev(w["emb_ln_b"]), 1e-12, out, err)
+    torch.cuda.synchronize()
+    assert err.item() == 0
+    got = host64(out).reshape(4, L, 768)
+    tol = 2e-2 if dtype == 0 else 1e-5
+    for i in range(4):
+        tok = ids[i].copy()
+        tok[lengths[i]:] = 0
+        ref = orc.embed(cfg, w, tok)
+        np.testing.assert_allclose(got[i], ref, rtol=0, atol=tol)
+    # out-of-range id at a real position sets the flag
+    bad = ids.copy()
+    bad[0, 3] = 5000
+    err.zero_()
+    arlo_lib.op_embed(dtype, torch.from_numpy(bad).cuda(), torch.from_numpy(lengths).cuda(),
+                      dev(w["word_emb"]), dev(w["pos_emb"]), dev(w["type_emb"]), f32_dev(w["emb_ln_g"]),
+                      f32_dev(w["emb_ln_b"]), 1e-12, out, err)
+    torch.cuda.synchronize()
+    assert err.item() == 1
+
+
+# ---------------------------------------------------------------------- attention
+@pytest.mark.parametrize("L,heads,lengths", [
+    (128, 12, [128, 1, 65, 64, 0, 100]),
+    (512, 2, [512, 300, 7]),
+    (32, 2, [32, 5, 1, 17]),
+    (64, 16, [63, 64]),
+])
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_attention_masked(arlo_lib, L, heads, lengths, dtype):
+    B = len(lengths)
+    H = 64 * heads
+    qkv = rnd((B * L, 3 * H), L + heads, 1.0)
+    lens = np.array(lengths, np.int32)
+    dev = bf16_dev if dtype == 0 else f32_dev
+    out = torch.full((B * L, H), float("nan"), device="cuda",
+                     dtype=torch.bfloat16 if dtype == 0 else torch.float32)
+    arlo_lib.op_attention(dtype, B, L, heads, dev(qkv), torch.from_numpy(lens).cuda(), out)
+    torch.cuda.synchronize()
+    got = host64(out).reshape(B, L, H)
+    assert np.all(np.isfinite(got)), "pad rows must be finite"
+    tol = 2e-2 if dtype == 0 else 2e-5
+    for i, n in enumerate(lengths):
+        x = qkv[i * L:(i + 1) * L].astype(np.float64)
+        q, k, v = x[:, :H], x[:, H:2 * H], x[:, 2 * H:]
+        if n > 0:
+            ref = orc.attention(q[:n], k[:n], v[:n], heads)
+            np.testing.assert_allclose(got[i, :n], ref, rtol=0, atol=tol)
+            # rows of a partially padded query tile attend the real keys
+            end = min(L, ((n + 63) // 64) * 64)
+            if end > n:
+                refm = orc.attention_masked(q[:end], k[:end], v[:end], heads, n)
+                np.testing.assert_allclose(got[i, n:end], refm[n:end], rtol=0, atol=tol)
+        start = ((n + 63) // 64) * 64
+        assert np.all(got[i, start:] == 0)
+
+
+# --------------------------------------------------------------------------- head
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_head(arlo_lib, dtype):
+    cfg = wl.BERT_BASE
+    w = wl.make_weights(wl.ModelConfig("hd", 1, 768, 12, 3072, 100), seed=4)
+    B, L = 5, 64
+    x = rnd((B * L, 768), 9)
+    dev = bf16_dev if dtype == 0 else f32_dev
+    logits = torch.empty((B, 2), device="cuda", dtype=torch.float32)
+    arlo_lib.op_head(dtype, B, L, dev(x), dev(w["w_p"]), f32_dev(w["b_p"]), dev(w["w_c"]), f32_dev(w["b_c"]), logits)
+    torch.cuda.synchronize()
+    ref = np.stack([orc.head(w, x[i * L].astype(np.float64)) for i in range(B)])
+    np.testing.assert_allclose(logits.cpu().numpy(), ref, rtol=0, atol=1e-5)
