@@ -98,8 +98,8 @@ def test_gemm_fp32_check_mode(arlo_lib, M, N, K, epi):
 @pytest.mark.parametrize("dtype", [0, 1])
 def test_layernorm(arlo_lib, H, dtype):
     M = 257
-    x = rnd((M, H), H) * 3 + 1
-    g = rnd((H,), 1, 0.1) + 1
+    x = wl.round_to_bf16(rnd((M, H), H) * 3 + 1)
+    g = wl.round_to_bf16(rnd((H,), 1, 0.1) + 1)
     b = rnd((H,), 2, 0.02)
     ref = orc.layer_norm(x, g, b, 1e-12)
     dev = bf16_dev if dtype == 0 else f32_dev
