@@ -1,0 +1,428 @@
+#!/usr/bin/env python
+"""Benchmark of the polymorphed BERT-base runtimes on B200 (BASELINE.json configs[1]).
+
+One STEP = serving R synthetic requests (skewed Twitter-like lengths,
+paper_conf_icpp_tanlyl024_b200/workload.py) through the per-length runtimes
+L in {64, 128, 256, 512} (batch buckets up to 32, bf16): every request goes to
+its ideal runtime (smallest max_length >= len, §3.2 / Alg. 1
+with idle instances) and each runtime runs ceil(n_L / 32) static-shape
+forwards (embedding -> 12 x {QKV, masked attention, out-proj, LN, FFN1, FFN2,
+LN} -> pooler/classifier).  value = requests / second over the timed steps.
+
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl arlo|reference]
+Under torchrun each rank serves its own R requests per step on its own GPU
+(independent replicas, no data-path collective; weak scaling); timing is
+the max over ranks.  `--impl reference` times the fp64 CPU oracle on the
+same workload definition (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+from paper_conf_icpp_tanlyl024_b200 import metrics  # noqa: E402
+from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
+
+RUNTIME_LS = (64, 128, 256, 512)
+MAX_BATCH = 32
+METRIC = "BERT-base req/s & mean/p99 latency per length bucket; tensor-pipe util"
+
+
+def parse():
+    p = argparse.ArgumentParser()
+    p.add_argument("--gpus", type=int, default=1)
+    p.add_argument("--steps", type=int, default=20)
+    p.add_argument("--warmup", type=int, default=5)
+    p.add_argument("--impl", default="arlo", choices=["arlo", "reference"])
+    p.add_argument("--requests", type=int, default=512, help="requests per step per GPU")
+    p.add_argument("--no-cpu-baseline", action="store_true")
+    p.add_argument("--no-extras", action="store_true", help="skip per-L table / ST-512 / e2e (profiling runs)")
+    return p.parse_args()
+
+
+# ------------------------------------------------------------------------- workload plan
+def make_step_requests(step: int, rank: int, R: int, cfg):
+    lengths = wl.sample_lengths(R, seed=wl.SEED_LENGTHS + 7919 * step + 104729 * rank)
+    return lengths
+
+
+def plan_forwards(lengths, runtime_ls=RUNTIME_LS, max_batch=MAX_BATCH):
+    """Group requests by ideal runtime; chunks of <= max_batch. Returns [(L, [request idx])]."""
+    idx = wl.ideal_runtime(lengths, runtime_ls)
+    out = []
+    for r, L in enumerate(runtime_ls):
+        members = np.nonzero(idx == r)[0]
+        for s in range(0, len(members), max_batch):
+            out.append((L, members[s:s + max_batch]))
+    return out
+
+
+# ------------------------------------------------------------------------- clocks
+class ClockSampler:
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index: int):
+        self.gpu, self.rows, self.proc = gpu_index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 8:
+                self.rows.append(parts)
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if r[4 + i].lower().startswith("active")})
+        loaded = [s for s in sm if s > 500] or sm
+        return {"sm_mhz": float(np.median(loaded)) if loaded else None,
+                "sm_max_mhz": max(mx) if mx else None, "reasons": reasons, "samples": len(self.rows)}
+
+
+# ------------------------------------------------------------------------- reference arm
+def run_reference(args, rank):
+    """The oracle, as it stands, timed on this host's cores on bounded samples of the workload."""
+    from oracle import encoder as orc
+    import threadpoolctl
+    cfg = wl.BERT_BASE
+    w = wl.make_weights(cfg)
+    per_step = 4
+    times, n_req = [], 0
+    for step in range(args.warmup + args.steps):
+        lengths = make_step_requests(step, rank, args.requests, cfg)[:per_step]
+        ids = wl.sample_token_ids(cfg, lengths, int(lengths.max()), seed=wl.SEED_TOKENS + step)
+        t0 = time.perf_counter()
+        for i, n in enumerate(lengths):
+            orc.forward_request(cfg, w, ids[i, :n])
+        dt = time.perf_counter() - t0
+        if step >= args.warmup:
+            times.append(dt)
+            n_req += len(lengths)
+    total = sum(times)
+    threads = max((d.get("num_threads", 1) for d in threadpoolctl.threadpool_info()), default=1)
+    value = n_req / total
+    sample = f"{per_step} requests/step of the skewed length distribution (real prefixes, fp64 numpy)"
+    return {"metric": METRIC, "value": value, "unit": "req/s", "impl": "reference", "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / len(times),
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
+            "data": "synthetic", "config": {"workload": "bert-base polymorphed L{64,128,256,512} b<=32",
+                                            "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "req/s", "cores": threads, "kind": "oracle", "sample": sample},
+            "e2e": {"value": value, "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+
+
+def cpu_baseline(seconds=15.0):
+    from oracle import encoder as orc
+    import threadpoolctl
+    cfg = wl.BERT_BASE
+    w = wl.make_weights(cfg)
+    lengths = wl.sample_lengths(256, seed=wl.SEED_LENGTHS + 999)
+    ids = wl.sample_token_ids(cfg, lengths, 512, seed=wl.SEED_TOKENS + 999)
+    t0 = time.perf_counter()
+    n = 0
+    while n < len(lengths) and (time.perf_counter() - t0 < seconds or n < 4):
+        orc.forward_request(cfg, w, ids[n, :lengths[n]])
+        n += 1
+    dt = time.perf_counter() - t0
+    threads = max((d.get("num_threads", 1) for d in threadpoolctl.threadpool_info()), default=1)
+    return {"value": n / dt, "unit": "req/s", "cores": threads, "kind": "oracle",
+            "sample": f"{n} requests of the skewed distribution (mean len {lengths[:n].mean():.1f}), "
+                      f"real prefixes, numpy fp64, {dt:.1f} s, {os.cpu_count()} host cores"}
+
+
+# ------------------------------------------------------------------------- main arm
+def main():
+    args = parse()
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+
+    if args.impl == "reference":
+        if rank == 0:
+            print(json.dumps(run_reference(args, rank)), flush=True)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_icpp_tanlyl024_b200 import arlo
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    cfg = wl.BERT_BASE
+    w = wl.make_weights(cfg)
+    W = arlo.Weights(cfg, arlo.upload_weights(cfg, w, arlo.BF16, dev), arlo.BF16, local_rank)
+    stream = torch.cuda.current_stream(dev)
+    runtimes = {}
+    for L in RUNTIME_LS:
+        rt = arlo.Runtime(W, L, MAX_BATCH)
+        rt.set_stream(stream)
+        runtimes[L] = rt
+
+    R = args.requests
+    n_steps = args.warmup + args.steps
+    # pre-stage every step's inputs in HBM (device-resident timing)
+    steps = []
+    for s in range(n_steps):
+        lengths = make_step_requests(s, rank, R, cfg)
+        fwd = []
+        for L, members in plan_forwards(lengths):
+            lens = lengths[members].astype(np.int32)
+            ids = wl.sample_token_ids(cfg, lens, L, seed=wl.SEED_TOKENS + 31 * s + L)
+            fwd.append((L, len(members), torch.from_numpy(ids).to(dev), torch.from_numpy(lens).to(dev),
+                        torch.empty((len(members), cfg.num_labels), device=dev), ids, lens))
+        steps.append((lengths, fwd))
+    flush = torch.empty(512 * 1024 * 1024 // 4, dtype=torch.float32, device=dev)  # 512 MB > 126 MB L2
+
+    def run_step(fwd, ev_pairs=None):
+        for j, (L, n, ids_d, lens_d, out_d, _, _) in enumerate(fwd):
+            if ev_pairs is not None:
+                ev_pairs[j][0].record(stream)
+            runtimes[L].enqueue(n, ids_d, lens_d, out_d)
+            if ev_pairs is not None:
+                ev_pairs[j][1].record(stream)
+
+    for s in range(args.warmup):
+        run_step(steps[s][1])
+        flush.zero_()
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+
+    sampler = ClockSampler(local_rank)
+    sampler.start()
+    time.sleep(0.3)
+    step_ms, per_fwd = [], []
+    launches = 0
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    for s in range(args.warmup, n_steps):
+        fwd = steps[s][1]
+        ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in fwd]
+        st, en = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        st.record(stream)
+        run_step(fwd, ev)
+        en.record(stream)
+        flush.zero_()  # between timed steps, outside [st, en]
+        launches += sum(runtimes[L].kernel_count(n) for (L, n, *_rest) in fwd)
+        per_fwd.append((fwd, ev))
+        step_ms.append((st, en))
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    clocks = sampler.stop()
+    step_times = [a.elapsed_time(b) for a, b in step_ms]
+    total_ms = float(sum(step_times))
+    # per-bucket latency: a request's latency = its forward's duration (all arrive at step start,
+    # forwards run back to back: completion time from step start is also reported)
+    lat = {L: [] for L in RUNTIME_LS}
+    done = {L: [] for L in RUNTIME_LS}
+    for (fwd, ev), (st, _) in zip(per_fwd, step_ms):
+        for (L, n, *_r), (a, b) in zip(fwd, ev):
+            lat[L] += [a.elapsed_time(b)] * n
+            done[L] += [st.elapsed_time(b)] * n
+    total_req = R * args.steps
+    t_max = total_ms
+    if world > 1:
+        t = torch.tensor([total_ms], device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        t_max = float(t.item())
+    value = world * total_req / (t_max / 1e3)
+
+    result = None
+    if rank == 0:
+        result = {"metric": METRIC, "value": value, "unit": "req/s", "n_gpus": world, "steps": args.steps,
+                  "warmup": args.warmup, "ms_per_step": t_max / args.steps, "higher_is_better": True,
+                  "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+                  "config": {"workload": "bert-base polymorphed runtimes L{64,128,256,512}, batch buckets <=32 "
+                                         "(BASELINE configs[1])",
+                             "requests_per_step_per_gpu": R, "lengths": "LogNormal(ln21,0.6)<=125 x512/125",
+                             "weights": "random N(0,0.02) seed 0", "l2": "flushed (512 MB write) between steps",
+                             "parallelism": f"replicas x{world}"},
+                  "latency_ms_per_bucket": {
+                      str(L): {"requests": len(lat[L]),
+                               "forward_mean": float(np.mean(lat[L])) if lat[L] else None,
+                               "forward_p99": float(np.percentile(lat[L], 99)) if lat[L] else None,
+                               "completion_mean": float(np.mean(done[L])) if done[L] else None,
+                               "completion_p99": float(np.percentile(done[L], 99)) if done[L] else None}
+                      for L in RUNTIME_LS},
+                  "gpu_launches": int(launches), "clocks": clocks}
+        pad_tokens = sum(L * n for (_, fwd) in steps[args.warmup:] for (L, n, *_r) in fwd)
+        real_tokens = sum(int(x.sum()) for (x, _) in steps[args.warmup:])
+        static_flops = sum(metrics.forward_flops(cfg, n, L) for (_, fwd) in steps[args.warmup:] for (L, n, *_r) in fwd)
+        result["padding_efficiency"] = real_tokens / pad_tokens
+        result["static_tflops"] = static_flops / (total_ms / 1e3) / 1e12
+        result["useful_tflops"] = sum(metrics.useful_flops(cfg, x) for (x, _) in steps[args.warmup:]) / (total_ms / 1e3) / 1e12
+
+    if rank == 0 and not args.no_extras:
+        result["roofline"] = roofline_dominant(arlo, torch, dev, stream, step_times)
+        result["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
+        result["uniform_512"] = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
+        result["e2e"] = e2e(runtimes, torch, stream, steps[args.warmup:], R, cfg, flush)
+        if not args.no_cpu_baseline:
+            result["cpu_baseline"] = cpu_baseline()
+    if rank == 0:
+        print(json.dumps(result), flush=True)
+    for rt in runtimes.values():
+        rt.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+def roofline_dominant(arlo, torch, dev, stream, step_times):
+    """Dominant kernel: the FFN1 tcgen05 GEMM (+bias+GELU) of the L=128, b=32 runtime
+    (M=4096, N=3072, K=768), the single largest GEMM share of a step.  Timed live
+    with a CUDA event pair around each launch on the launching stream."""
+    M, N, K = 4096, 3072, 768
+    A = torch.randn(M, K, device=dev).to(torch.bfloat16)
+    Wt = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
+    b = torch.zeros(N, device=dev)
+    out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
+    for _ in range(5):
+        arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(50)]
+    for a, e in ev:
+        a.record(stream)
+        arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
+        e.record(stream)
+    torch.cuda.synchronize()
+    t = float(np.mean([a.elapsed_time(e) for a, e in ev])) / 1e3
+    flops = metrics.gemm_flops(M, N, K)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    peak = peaks.get("bf16_tflops", 1590.0)
+    traffic = None
+    try:
+        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get("ffn1_gemm_dram_bytes")
+    except Exception:
+        pass
+    achieved = flops / t / 1e12
+    return {"kernel": "gemm_tc_kernel<256, GELU> (FFN1, M=4096 N=3072 K=768)", "bound": "tensor",
+            "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+            "traffic": traffic, "peak_source": "MEASURED_PEAKS.json bf16_tflops (burst)" if peaks else
+            "fallback 1590 TFLOP/s (B200_PROFILING.md)", "launch_us": t * 1e6,
+            "algorithmic_flops_per_launch": flops}
+
+
+def per_L_table(runtimes, torch, dev, stream, cfg):
+    """Offline-profiler table (A4): latency of one forward vs batch bucket for every runtime."""
+    table = {}
+    for L, rt in runtimes.items():
+        row = {}
+        for b in (1, 2, 4, 8, 16, 32):
+            lens = np.full(b, L, np.int32)
+            ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
+            ld = torch.from_numpy(lens).to(dev)
+            out = torch.empty((b, cfg.num_labels), device=dev)
+            for _ in range(3):
+                rt.enqueue(b, ids, ld, out)
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(10)]
+            for a, e in ev:
+                a.record(stream)
+                rt.enqueue(b, ids, ld, out)
+                e.record(stream)
+            torch.cuda.synchronize()
+            ts = [a.elapsed_time(e) for a, e in ev]
+            row[str(b)] = {"median": float(np.median(ts)), "tflops": metrics.forward_flops(cfg, b, L) / (np.median(ts) / 1e3) / 1e12}
+        table[str(L)] = row
+    return table
+
+
+def uniform_512(runtimes, torch, dev, stream, steps, flush, R, cfg):
+    """Baseline ST: the same requests, all zero-padded to L=512."""
+    rt = runtimes[512]
+    tot = 0.0
+    nsteps = min(3, len(steps))
+    for lengths, _ in steps[:nsteps]:
+        evs = []
+        for s0 in range(0, len(lengths), MAX_BATCH):
+            lens = lengths[s0:s0 + MAX_BATCH].astype(np.int32)
+            ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, 512, seed=3)).to(dev)
+            ld = torch.from_numpy(lens).to(dev)
+            out = torch.empty((len(lens), cfg.num_labels), device=dev)
+            evs.append((len(lens), ids, ld, out))
+        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for n, ids, ld, out in evs:
+            rt.enqueue(n, ids, ld, out)
+        e.record(stream)
+        flush.zero_()
+        torch.cuda.synchronize()
+        tot += a.elapsed_time(e)
+    return {"value": nsteps * R / (tot / 1e3), "unit": "req/s", "steps": nsteps,
+            "note": "same requests, uniform zero-padding to L=512 (ST baseline)"}
+
+
+def e2e(runtimes, torch, stream, steps, R, cfg, flush):
+    """Same metric through the public C ABI with HOST buffers: arlo_infer on pinned host ids/lengths/
+    logits per forward (H2D of the inputs and D2H of the logits inside the timed region)."""
+    h2d = d2h = 0
+    host = []
+    for lengths, fwd in steps:
+        hf = []
+        for (L, n, _i, _l, _o, ids_np, lens_np) in fwd:
+            ids_h = torch.zeros((MAX_BATCH, L), dtype=torch.int32).pin_memory()
+            ids_h[:n] = torch.from_numpy(ids_np)
+            len_h = torch.zeros(MAX_BATCH, dtype=torch.int32).pin_memory()
+            len_h[:n] = torch.from_numpy(lens_np)
+            out_h = torch.zeros((MAX_BATCH, cfg.num_labels), dtype=torch.float32).pin_memory()
+            hf.append((L, n, ids_h, len_h, out_h))
+        host.append(hf)
+    tot = 0.0
+    for hf in host:
+        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        for (L, n, ids_h, len_h, out_h) in hf:
+            runtimes[L].infer(ids_h, len_h, out_h)
+        e.record(stream)
+        torch.cuda.synchronize()
+        tot += a.elapsed_time(e)
+        flush.zero_()
+    for hf in host:
+        for (L, n, *_r) in hf:
+            h2d += 16 + 4 * MAX_BATCH + 4 * n * L
+            d2h += 4 * n * cfg.num_labels + 4
+    h2d /= len(host)
+    d2h /= len(host)
+    return {"value": len(host) * R / (tot / 1e3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),
+            "d2h_bytes_per_step": int(d2h), "api": "arlo_infer (synchronous, pinned host buffers)"}
+
+
+if __name__ == "__main__":
+    main()
