@@ -184,7 +184,8 @@ def main():
     cfg = wl.BERT_BASE
     w = wl.make_weights(cfg)
     W = arlo.Weights(cfg, arlo.upload_weights(cfg, w, arlo.BF16, dev), arlo.BF16, local_rank)
-    stream = torch.cuda.current_stream(dev)
+    stream = torch.cuda.Stream(dev)  # runtimes, events and the L2 flush all on this stream
+    torch.cuda.set_stream(stream)
     runtimes = {}
     for L in RUNTIME_LS:
         rt = arlo.Runtime(W, L, MAX_BATCH)

@@ -108,6 +108,7 @@ typedef struct arlo_runtime arlo_runtime;
  */
 int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out);
 void arlo_runtime_destroy(arlo_runtime* rt);
+/* Launch stream for every later call (a cudaStream_t; NULL = legacy default stream). */
 int arlo_runtime_set_stream(arlo_runtime* rt, void* cuda_stream);
 int32_t arlo_runtime_length(const arlo_runtime* rt);
 int32_t arlo_runtime_max_batch(const arlo_runtime* rt);

@@ -57,11 +57,12 @@ int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t heads, const 
                       const int32_t* lengths, void* o, void* stream);
 
 /*
- * Step a9: logits[b] = W_c tanh(W_p x[b*L] + b_p) + b_c for b < B, fp32 out [B, C].
+ * Step a9: pooled[b] = tanh(W_p x[b*L] + b_p) (fp32 [B, H], caller-provided
+ * scratch), logits[b] = W_c pooled[b] + b_c for b < B, fp32 out [B, C].  H <= 2048.
  */
 int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, const void* x,
                  const void* w_p, const float* b_p, const void* w_c, const float* b_c,
-                 float* logits, void* stream);
+                 float* pooled, float* logits, void* stream);
 
 #ifdef __cplusplus
 }

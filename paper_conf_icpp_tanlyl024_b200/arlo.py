@@ -74,7 +74,7 @@ _sig("arlo_op_gemm", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _
 _sig("arlo_op_layernorm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp)
 _sig("arlo_op_embed", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp, _vp)
 _sig("arlo_op_attention", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp)
-_sig("arlo_op_head", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp)
+_sig("arlo_op_head", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp)
 
 
 class ArloError(RuntimeError):
@@ -253,8 +253,10 @@ def op_attention(dtype, B, L, heads, qkv, lengths, out, stream=None):
 
 
 def op_head(dtype, B, L, x, w_p, b_p, w_c, b_c, logits, stream=None):
+    import torch
     H = w_p.shape[1]
     Cn = w_c.shape[0]
-    check(lib.arlo_op_head(dtype, B, L, H, Cn, _ptr(x), _ptr(w_p), _ptr(b_p), _ptr(w_c), _ptr(b_c), _ptr(logits),
-                           _stream_ptr(stream)))
+    pooled = torch.empty((B, H), dtype=torch.float32, device=logits.device)
+    check(lib.arlo_op_head(dtype, B, L, H, Cn, _ptr(x), _ptr(w_p), _ptr(b_p), _ptr(w_c), _ptr(b_c), _ptr(pooled),
+                           _ptr(logits), _stream_ptr(stream)))
     return logits

@@ -31,7 +31,8 @@ namespace arlo {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int kThreads = 192;  // 6 warps
+constexpr int kEpiWarps = 16;  // 4 warpgroups: each TMEM lane quarter is drained by 4 warps
+constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp 0 TMA, warp 1 MMA, warps 2.. epilogue
 constexpr int kAccStages = 2;
 
 template <int BN>
@@ -79,7 +80,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
     for (int a = 0; a < kAccStages; ++a) {
       ptx::mbar_init(&tfull[a], 1);
-      ptx::mbar_init(&tempty[a], 4);  // one arrive per epilogue warp
+      ptx::mbar_init(&tempty[a], kEpiWarps);  // one arrive per epilogue warp
     }
     ptx::fence_mbar_init();
   }
@@ -136,7 +137,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
   } else {
     // --------------------------------------------------------------- epilogue
-    const int q = warp & 3;  // TMEM lane quarter this warp may access
+    // warp w may only touch TMEM lanes 32*(w%4)..+31 (rows of the tile); the
+    // four warps sharing a quarter split the BN columns into 4 groups.
+    const int q = warp & 3;
+    constexpr int COLS = BN / 4;
+    const int cg = (warp - 2) >> 2;
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
@@ -144,17 +149,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
       const int row = m0 + q * 32 + lane;
-      const uint32_t t_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN;
-#pragma unroll 1
-      for (int c = 0; c < BN; c += 32) {
-        uint32_t r[32];
-        ptx::tmem_ld_32x32b_x32(t_row + c, r);
+      const uint32_t t_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + cg * COLS;
+#pragma unroll
+      for (int c = 0; c < COLS; c += 16) {
+        uint32_t r[16];
+        ptx::tmem_ld_32x32b_x16(t_row + c, r);
         ptx::tmem_wait_ld();
         if (row < M) {
-          const int col = n0 + c;
-          float v[32];
+          const int col = n0 + cg * COLS + c;
+          float v[16];
 #pragma unroll
-          for (int j = 0; j < 32; j += 4) {
+          for (int j = 0; j < 16; j += 4) {
             const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + col + j));
             v[j] = __uint_as_float(r[j]) + b4.x;
             v[j + 1] = __uint_as_float(r[j + 1]) + b4.y;
@@ -163,12 +168,12 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           }
           if (EPI == EPI_BIAS_GELU) {
 #pragma unroll
-            for (int j = 0; j < 32; ++j) v[j] = gelu_erf(v[j]);
+            for (int j = 0; j < 16; ++j) v[j] = gelu_erf(v[j]);
           }
           if (EPI == EPI_BIAS_RESID) {
             const uint4* rp = reinterpret_cast<const uint4*>(resid + (size_t)row * N + col);
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
+            for (int j = 0; j < 2; ++j) {
               const uint4 u = __ldg(rp + j);
               float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z),
                      f3 = unpack_bf16x2(u.w);
@@ -178,7 +183,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           }
           uint4* op = reinterpret_cast<uint4*>(out + (size_t)row * N + col);
 #pragma unroll
-          for (int j = 0; j < 4; ++j) {
+          for (int j = 0; j < 2; ++j) {
             uint4 u;
             u.x = pack_bf16x2(v[8 * j + 0], v[8 * j + 1]);
             u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);

@@ -49,8 +49,8 @@ cudaError_t launch_attention(DType dt, int B, int L, int heads, const void* qkv,
 
 // ---- a9: CLS pooler + classifier ----------------------------------------------------------
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p,
-                        const float* b_p, const void* w_c, const float* b_c, float* logits,
-                        cudaStream_t s);
+                        const float* b_p, const void* w_c, const float* b_c, float* pooled,
+                        float* logits, cudaStream_t s);
 
 // Resolve cuTensorMapEncodeTiled through the runtime (no link-time libcuda dependency).
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,

@@ -168,6 +168,7 @@ struct arlo_runtime {
   int32_t* lengths = nullptr;  // [max_batch]  (err, lengths, ids are contiguous: one staging copy)
   int32_t* ids = nullptr;      // [max_batch * L]
   float* logits = nullptr;     // [max_batch * C]
+  float* pooled = nullptr;     // [max_batch * H] fp32 pooler output
   void *X = nullptr, *QKV = nullptr, *O = nullptr, *Y = nullptr, *F = nullptr;
   // pinned host staging
   void* h_stage = nullptr;
@@ -225,7 +226,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
               "ln2 launch");
   }
   ARLO_CUDA(launch_head(dt, b, L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
-                        (const float*)w->hd(3), rt->logits, s),
+                        (const float*)w->hd(3), rt->pooled, rt->logits, s),
             "head launch");
   return ARLO_OK;
 }
@@ -288,6 +289,7 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
   const size_t off_ids = off_len + 4 * (size_t)max_batch;
   size_t off = al(off_ids + 4 * Mmax);
   const size_t off_logits = off; off = al(off + 4 * (size_t)max_batch * c.num_labels);
+  const size_t off_pooled = off; off = al(off + 4 * (size_t)max_batch * H);
   const size_t off_X = off; off = al(off + es * Mmax * H);
   const size_t off_QKV = off; off = al(off + es * Mmax * 3 * H);
   const size_t off_O = off; off = al(off + es * Mmax * H);
@@ -302,6 +304,7 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
   rt->lengths = (int32_t*)(a + off_len);
   rt->ids = (int32_t*)(a + off_ids);
   rt->logits = (float*)(a + off_logits);
+  rt->pooled = (float*)(a + off_pooled);
   rt->X = a + off_X; rt->QKV = a + off_QKV; rt->O = a + off_O; rt->Y = a + off_Y; rt->F = a + off_F;
   rt->h_stage_bytes = off_ids + 4 * Mmax + 4 * (size_t)max_batch * c.num_labels + 64;
   e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
@@ -348,7 +351,7 @@ extern "C" void arlo_runtime_destroy(arlo_runtime* rt) {
 
 extern "C" int arlo_runtime_set_stream(arlo_runtime* rt, void* stream) {
   if (!rt) return set_error(ARLO_EINVAL, "null runtime");
-  rt->stream = stream ? (cudaStream_t)stream : rt->own_stream;
+  rt->stream = (cudaStream_t)stream;  // NULL = the legacy default stream
   return ARLO_OK;
 }
 
@@ -494,11 +497,13 @@ extern "C" int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t he
 }
 
 extern "C" int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, const void* x,
-                            const void* w_p, const float* b_p, const void* w_c, const float* b_c, float* logits,
-                            void* stream) {
+                            const void* w_p, const float* b_p, const void* w_c, const float* b_c, float* pooled,
+                            float* logits, void* stream) {
   clear_error();
-  if (B < 0 || L < 1 || H < 8 || H % 8 || C < 1 || !x || !w_p || !b_p || !w_c || !b_c || !logits)
+  if (B < 0 || L < 1 || H < 8 || H % 8 || H > 2048 || C < 1 || !x || !w_p || !b_p || !w_c || !b_c || !pooled ||
+      !logits)
     return set_error(ARLO_EINVAL, "arlo_op_head: bad arguments");
-  ARLO_CUDA(launch_head(to_dt(dtype), B, L, H, C, x, w_p, b_p, w_c, b_c, logits, (cudaStream_t)stream), "head");
+  ARLO_CUDA(launch_head(to_dt(dtype), B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, (cudaStream_t)stream),
+            "head");
   return ARLO_OK;
 }
