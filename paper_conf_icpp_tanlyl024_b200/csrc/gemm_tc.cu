@@ -142,46 +142,67 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     const int q = warp & 3;
     constexpr int COLS = BN / 4;
     const int cg = (warp - 2) >> 2;
+    // Software-pipelined over 16-column chunks: the TMEM load, bias and residual
+    // of chunk c+1 are in flight while chunk c is computed and stored; the
+    // accumulator buffer is released to the MMA warp right after its last load.
+    constexpr int NC = COLS / 16;
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
       const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+      const int row = m0 + q * 32 + lane;
+      const bool row_ok = row < M;
+      const int col0 = n0 + cg * COLS;
+      const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
+      const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
+      uint4* out4 = reinterpret_cast<uint4*>(out + (size_t)row * N + col0);
+      uint32_t r[2][16];
+      float4 bv[2][4];
+      uint4 rv[2][2];
+      // prefetch chunk 0's bias / residual before waiting for the accumulator
+#pragma unroll
+      for (int j = 0; j < 4; ++j) bv[0][j] = __ldg(bias4 + j);
+      if (EPI == EPI_BIAS_RESID && row_ok) { rv[0][0] = __ldg(res4); rv[0][1] = __ldg(res4 + 1); }
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      const int row = m0 + q * 32 + lane;
       const uint32_t t_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + cg * COLS;
+      ptx::tmem_ld_32x32b_x16(t_row, r[0]);
+      ptx::tmem_wait_ld();
 #pragma unroll
-      for (int c = 0; c < COLS; c += 16) {
-        uint32_t r[16];
-        ptx::tmem_ld_32x32b_x16(t_row + c, r);
-        ptx::tmem_wait_ld();
-        if (row < M) {
-          const int col = n0 + cg * COLS + c;
-          float v[16];
+      for (int c = 0; c < NC; ++c) {
+        const int cur = c & 1, nxt = cur ^ 1;
+        if (c + 1 < NC) {
+          ptx::tmem_ld_32x32b_x16(t_row + (c + 1) * 16, r[nxt]);
 #pragma unroll
-          for (int j = 0; j < 16; j += 4) {
-            const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + col + j));
-            v[j] = __uint_as_float(r[j]) + b4.x;
-            v[j + 1] = __uint_as_float(r[j + 1]) + b4.y;
-            v[j + 2] = __uint_as_float(r[j + 2]) + b4.z;
-            v[j + 3] = __uint_as_float(r[j + 3]) + b4.w;
+          for (int j = 0; j < 4; ++j) bv[nxt][j] = __ldg(bias4 + (c + 1) * 4 + j);
+          if (EPI == EPI_BIAS_RESID && row_ok) {
+            rv[nxt][0] = __ldg(res4 + (c + 1) * 2);
+            rv[nxt][1] = __ldg(res4 + (c + 1) * 2 + 1);
           }
-          if (EPI == EPI_BIAS_GELU) {
+        }
+        float v[16];
 #pragma unroll
-            for (int j = 0; j < 16; ++j) v[j] = gelu_erf(v[j]);
-          }
-          if (EPI == EPI_BIAS_RESID) {
-            const uint4* rp = reinterpret_cast<const uint4*>(resid + (size_t)row * N + col);
+        for (int j = 0; j < 4; ++j) {
+          v[4 * j + 0] = __uint_as_float(r[cur][4 * j + 0]) + bv[cur][j].x;
+          v[4 * j + 1] = __uint_as_float(r[cur][4 * j + 1]) + bv[cur][j].y;
+          v[4 * j + 2] = __uint_as_float(r[cur][4 * j + 2]) + bv[cur][j].z;
+          v[4 * j + 3] = __uint_as_float(r[cur][4 * j + 3]) + bv[cur][j].w;
+        }
+        if (EPI == EPI_BIAS_GELU) {
 #pragma unroll
-            for (int j = 0; j < 2; ++j) {
-              const uint4 u = __ldg(rp + j);
-              float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z),
-                     f3 = unpack_bf16x2(u.w);
-              v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
-              v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
-            }
+          for (int j = 0; j < 16; ++j) v[j] = gelu_erf_fast(v[j]);
+        }
+        if (EPI == EPI_BIAS_RESID && row_ok) {
+#pragma unroll
+          for (int j = 0; j < 2; ++j) {
+            const uint4 u = rv[cur][j];
+            float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z),
+                   f3 = unpack_bf16x2(u.w);
+            v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
+            v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
           }
-          uint4* op = reinterpret_cast<uint4*>(out + (size_t)row * N + col);
+        }
+        if (row_ok) {
 #pragma unroll
           for (int j = 0; j < 2; ++j) {
             uint4 u;
@@ -189,13 +210,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);
             u.z = pack_bf16x2(v[8 * j + 4], v[8 * j + 5]);
             u.w = pack_bf16x2(v[8 * j + 6], v[8 * j + 7]);
-            op[j] = u;
+            out4[c * 2 + j] = u;
           }
         }
+        ptx::tmem_wait_ld();
+        if (c == (NC >= 2 ? NC - 2 : 0)) {
+          // every TMEM load of this tile has completed: hand the buffer back
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
+        }
       }
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
   }
