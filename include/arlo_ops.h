@@ -26,7 +26,8 @@ enum { ARLO_EPI_BIAS = 0, ARLO_EPI_BIAS_GELU = 1, ARLO_EPI_BIAS_RESIDUAL = 2 };
  * epi = identity | GELU_erf | (+ residual[M,N]).  Row-major, K-major operands
  * (PyTorch Linear layout).  Requires N % 64 == 0, K % 64 == 0, 1 <= M.
  * ARLO_BF16 runs the tcgen05/TMEM/TMA kernel; ARLO_FP32 the FFMA kernel.
- * force_bn: 0 = automatic tile width, else 64/128/256 (tests).
+ * force_bn: 0 = automatic tile choice; 64/128/256 = single-CTA kernel with that tile
+ * width; -128/-256 = CTA-pair (cta_group::2, 256-row tiles) kernel (tests).
  */
 int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, const void* A, const void* W,
                  const float* bias, const void* residual, void* out, int32_t epi,

@@ -35,26 +35,111 @@ constexpr int kEpiWarps = 16;  // 4 warpgroups: each TMEM lane quarter is draine
 constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp 0 TMA, warp 1 MMA, warps 2.. epilogue
 constexpr int kAccStages = 2;
 
-template <int BN>
+constexpr int tmem_cols_for(int n) {
+  return n <= 32 ? 32 : n <= 64 ? 64 : n <= 128 ? 128 : n <= 256 ? 256 : 512;
+}
+
+// PAIR = false: one CTA computes a 128 x BN tile; PAIR = true: a CTA pair
+// (cluster of 2, cta_group::2) computes a 256 x BN tile, each CTA holding 128
+// rows of A, BN/2 rows of W and its 128 x BN half of the accumulator.
+template <int BN, bool PAIR>
 struct TcCfg {
   static constexpr int A_BYTES = BM * BK * 2;
-  static constexpr int B_BYTES = BN * BK * 2;
+  static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
+  static constexpr int B_BYTES = B_ROWS * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (BN == 256) ? 4 : (BN == 128 ? 6 : 8);
-  static constexpr int TMEM_COLS = (kAccStages * BN <= 32) ? 32
-                                   : (kAccStages * BN <= 64) ? 64
-                                   : (kAccStages * BN <= 128) ? 128
-                                   : (kAccStages * BN <= 256) ? 256 : 512;
+  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;
+  static constexpr int TMEM_COLS = tmem_cols_for(kAccStages * BN);
   static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages) + 16;
   static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + BAR_BYTES;
+  static constexpr int TILE_M = PAIR ? 2 * BM : BM;
 };
+
+// Epilogue of one accumulator tile for one warp: TMEM lane quarter q (rows),
+// column group cg (BN/4 columns).  Software-pipelined over 16-column chunks:
+// the TMEM load, bias and residual of chunk c+1 are in flight while chunk c is
+// computed and stored; `release()` is called as soon as the last TMEM load of
+// the tile has completed so the MMA warp can reuse the accumulator buffer.
+template <int BN, int EPI, typename Release>
+__device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row, int n0, int M,
+                                              int N, const float* __restrict__ bias,
+                                              const bf16* __restrict__ resid, bf16* __restrict__ out,
+                                              Release release) {
+  constexpr int COLS = BN / 4;
+  constexpr int NC = COLS / 16;
+  const bool row_ok = row < M;
+  const int col0 = n0 + cg * COLS;
+  const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
+  const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
+  uint4* out4 = reinterpret_cast<uint4*>(out + (size_t)row * N + col0);
+  const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16) + cg * COLS;
+  uint32_t r[2][16];
+  float4 bv[2][4];
+  uint4 rv[2][2];
+#pragma unroll
+  for (int j = 0; j < 4; ++j) bv[0][j] = __ldg(bias4 + j);
+  if (EPI == EPI_BIAS_RESID && row_ok) { rv[0][0] = __ldg(res4); rv[0][1] = __ldg(res4 + 1); }
+  ptx::tmem_ld_32x32b_x16(t_row, r[0]);
+  ptx::tmem_wait_ld();
+#pragma unroll
+  for (int c = 0; c < NC; ++c) {
+    const int cur = c & 1, nxt = cur ^ 1;
+    if (c + 1 < NC) {
+      ptx::tmem_ld_32x32b_x16(t_row + (c + 1) * 16, r[nxt]);
+#pragma unroll
+      for (int j = 0; j < 4; ++j) bv[nxt][j] = __ldg(bias4 + (c + 1) * 4 + j);
+      if (EPI == EPI_BIAS_RESID && row_ok) {
+        rv[nxt][0] = __ldg(res4 + (c + 1) * 2);
+        rv[nxt][1] = __ldg(res4 + (c + 1) * 2 + 1);
+      }
+    }
+    float v[16];
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      v[4 * j + 0] = __uint_as_float(r[cur][4 * j + 0]) + bv[cur][j].x;
+      v[4 * j + 1] = __uint_as_float(r[cur][4 * j + 1]) + bv[cur][j].y;
+      v[4 * j + 2] = __uint_as_float(r[cur][4 * j + 2]) + bv[cur][j].z;
+      v[4 * j + 3] = __uint_as_float(r[cur][4 * j + 3]) + bv[cur][j].w;
+    }
+    if (EPI == EPI_BIAS_GELU) {
+#pragma unroll
+      for (int j = 0; j < 16; ++j) v[j] = gelu_erf_fast(v[j]);
+    }
+    if (EPI == EPI_BIAS_RESID && row_ok) {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        const uint4 u = rv[cur][j];
+        float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z), f3 = unpack_bf16x2(u.w);
+        v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
+        v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
+      }
+    }
+    if (row_ok) {
+#pragma unroll
+      for (int j = 0; j < 2; ++j) {
+        uint4 u;
+        u.x = pack_bf16x2(v[8 * j + 0], v[8 * j + 1]);
+        u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);
+        u.z = pack_bf16x2(v[8 * j + 4], v[8 * j + 5]);
+        u.w = pack_bf16x2(v[8 * j + 6], v[8 * j + 7]);
+        out4[c * 2 + j] = u;
+      }
+    }
+    ptx::tmem_wait_ld();
+    if (c == (NC >= 2 ? NC - 2 : 0)) {
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) release();
+    }
+  }
+}
 
 template <int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                int M, int N, int K, const float* __restrict__ bias, const bf16* __restrict__ resid,
                bf16* __restrict__ out) {
-  using C = TcCfg<BN>;
+  using C = TcCfg<BN, false>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -139,88 +224,16 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     // --------------------------------------------------------------- epilogue
     // warp w may only touch TMEM lanes 32*(w%4)..+31 (rows of the tile); the
     // four warps sharing a quarter split the BN columns into 4 groups.
-    const int q = warp & 3;
-    constexpr int COLS = BN / 4;
-    const int cg = (warp - 2) >> 2;
-    // Software-pipelined over 16-column chunks: the TMEM load, bias and residual
-    // of chunk c+1 are in flight while chunk c is computed and stored; the
-    // accumulator buffer is released to the MMA warp right after its last load.
-    constexpr int NC = COLS / 16;
+    const int q = warp & 3, cg = (warp - 2) >> 2;
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
       const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
-      const int row = m0 + q * 32 + lane;
-      const bool row_ok = row < M;
-      const int col0 = n0 + cg * COLS;
-      const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
-      const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
-      uint4* out4 = reinterpret_cast<uint4*>(out + (size_t)row * N + col0);
-      uint32_t r[2][16];
-      float4 bv[2][4];
-      uint4 rv[2][2];
-      // prefetch chunk 0's bias / residual before waiting for the accumulator
-#pragma unroll
-      for (int j = 0; j < 4; ++j) bv[0][j] = __ldg(bias4 + j);
-      if (EPI == EPI_BIAS_RESID && row_ok) { rv[0][0] = __ldg(res4); rv[0][1] = __ldg(res4 + 1); }
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
-      const uint32_t t_row = tmem_base + ((uint32_t)(q * 32) << 16) + acc * BN + cg * COLS;
-      ptx::tmem_ld_32x32b_x16(t_row, r[0]);
-      ptx::tmem_wait_ld();
-#pragma unroll
-      for (int c = 0; c < NC; ++c) {
-        const int cur = c & 1, nxt = cur ^ 1;
-        if (c + 1 < NC) {
-          ptx::tmem_ld_32x32b_x16(t_row + (c + 1) * 16, r[nxt]);
-#pragma unroll
-          for (int j = 0; j < 4; ++j) bv[nxt][j] = __ldg(bias4 + (c + 1) * 4 + j);
-          if (EPI == EPI_BIAS_RESID && row_ok) {
-            rv[nxt][0] = __ldg(res4 + (c + 1) * 2);
-            rv[nxt][1] = __ldg(res4 + (c + 1) * 2 + 1);
-          }
-        }
-        float v[16];
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-          v[4 * j + 0] = __uint_as_float(r[cur][4 * j + 0]) + bv[cur][j].x;
-          v[4 * j + 1] = __uint_as_float(r[cur][4 * j + 1]) + bv[cur][j].y;
-          v[4 * j + 2] = __uint_as_float(r[cur][4 * j + 2]) + bv[cur][j].z;
-          v[4 * j + 3] = __uint_as_float(r[cur][4 * j + 3]) + bv[cur][j].w;
-        }
-        if (EPI == EPI_BIAS_GELU) {
-#pragma unroll
-          for (int j = 0; j < 16; ++j) v[j] = gelu_erf_fast(v[j]);
-        }
-        if (EPI == EPI_BIAS_RESID && row_ok) {
-#pragma unroll
-          for (int j = 0; j < 2; ++j) {
-            const uint4 u = rv[cur][j];
-            float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z),
-                   f3 = unpack_bf16x2(u.w);
-            v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
-            v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
-          }
-        }
-        if (row_ok) {
-#pragma unroll
-          for (int j = 0; j < 2; ++j) {
-            uint4 u;
-            u.x = pack_bf16x2(v[8 * j + 0], v[8 * j + 1]);
-            u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);
-            u.z = pack_bf16x2(v[8 * j + 4], v[8 * j + 5]);
-            u.w = pack_bf16x2(v[8 * j + 6], v[8 * j + 7]);
-            out4[c * 2 + j] = u;
-          }
-        }
-        ptx::tmem_wait_ld();
-        if (c == (NC >= 2 ? NC - 2 : 0)) {
-          // every TMEM load of this tile has completed: hand the buffer back
-          ptx::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) ptx::mbar_arrive(&tempty[acc]);
-        }
-      }
+      uint64_t* te = &tempty[acc];
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32 + lane, n0, M, N, bias, resid, out,
+                             [te]() { ptx::mbar_arrive(te); });
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
   }
@@ -230,6 +243,124 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   if (warp == 1) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem_base, C::TMEM_COLS);
+  }
+}
+
+// CTA-pair kernel: cluster (2,1,1); the pair computes 256 x BN tiles with
+// tcgen05.mma.cta_group::2 issued by the leader (rank 0).  Each CTA's TMA
+// loads its 128 rows of A and its BN/2 rows of W and counts the bytes on the
+// leader's full barrier; the leader's commits arrive on both CTAs' empty and
+// tfull barriers (multicast); both CTAs' epilogue warps arrive on the
+// leader's tempty barrier.  Halves the L2->SM operand traffic per FLOP and
+// doubles the smem pipeline depth relative to the single-CTA kernel.
+template <int BN, int EPI>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                    int M, int N, int K, const float* __restrict__ bias, const bf16* __restrict__ resid,
+                    bf16* __restrict__ out) {
+  using C = TcCfg<BN, true>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint64_t* tempty = tfull + kAccStages;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kAccStages);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
+  const int num_m = (M + 2 * BM - 1) / (2 * BM);
+  const int num_n = N / BN;
+  const int tiles = num_m * num_n;
+  const int kblocks = K / BK;
+
+  if (warp == 0 && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < kAccStages; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], 2 * kEpiWarps);  // both CTAs' epilogue warps
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 1) ptx::tmem_alloc_pair(tmem_slot, C::TMEM_COLS);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int tile = pair; tile < tiles; tile += npairs) {
+        const int m0 = (tile % num_m) * 2 * BM + rank * BM;
+        const int n0 = (tile / num_m) * BN + rank * C::B_ROWS;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait(&empty[stage], phase ^ 1);
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+          const uint32_t fb = ptx::mapa_shared(&full[stage], 0);
+          ptx::tma_load_2d_pair(sA + stage * C::A_BYTES, &tmA, fb, kb * BK, m0);
+          ptx::tma_load_2d_pair(sB + stage * C::B_BYTES, &tmB, fb, kb * BK, n0);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && rank == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16_f32(2 * BM, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int tile = pair; tile < tiles; tile += npairs) {
+        ptx::mbar_wait_cluster(&tempty[acc], acc_phase ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait_cluster(&full[stage], phase);
+          ptx::tc_fence_after();
+          const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+          const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k) {
+            ptx::mma_bf16_ss_pair(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
+                                  ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
+          }
+          ptx::mma_commit_pair(&empty[stage]);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+        ptx::mma_commit_pair(&tfull[acc]);
+        if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    const int q = warp & 3, cg = (warp - 2) >> 2;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int tile = pair; tile < tiles; tile += npairs) {
+      const int m0 = (tile % num_m) * 2 * BM + rank * BM, n0 = (tile / num_m) * BN;
+      ptx::mbar_wait(&tfull[acc], acc_phase);
+      ptx::tc_fence_after();
+      const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32 + lane, n0, M, N, bias, resid, out,
+                             [te]() { ptx::mbar_arrive_cluster(te); });
+      if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+    }
+  }
+
+  ptx::tc_fence_before();
+  ptx::cluster_sync();
+  if (warp == 1) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc_pair(tmem_base, C::TMEM_COLS);
   }
 }
 
@@ -252,10 +383,10 @@ EncodeTiledFn get_encode_fn() {
   return fn;
 }
 
-template <int BN, int EPI>
-cudaError_t launch_bn_epi(const TcGemmPlan& p, cudaStream_t s) {
-  using C = TcCfg<BN>;
-  auto kern = gemm_tc_kernel<BN, EPI>;
+template <int BN, int EPI, bool PAIR>
+cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
+  using C = TcCfg<BN, PAIR>;
+  auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI> : gemm_tc_kernel<BN, EPI>;
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
@@ -267,12 +398,12 @@ cudaError_t launch_bn_epi(const TcGemmPlan& p, cudaStream_t s) {
   return cudaGetLastError();
 }
 
-template <int BN>
+template <int BN, bool PAIR>
 cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
   switch (p.epi) {
-    case EPI_BIAS: return launch_bn_epi<BN, EPI_BIAS>(p, s);
-    case EPI_BIAS_GELU: return launch_bn_epi<BN, EPI_BIAS_GELU>(p, s);
-    case EPI_BIAS_RESID: return launch_bn_epi<BN, EPI_BIAS_RESID>(p, s);
+    case EPI_BIAS: return launch_cfg<BN, EPI_BIAS, PAIR>(p, s);
+    case EPI_BIAS_GELU: return launch_cfg<BN, EPI_BIAS_GELU, PAIR>(p, s);
+    case EPI_BIAS_RESID: return launch_cfg<BN, EPI_BIAS_RESID, PAIR>(p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -303,23 +434,29 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
   return r == CUDA_SUCCESS;
 }
 
-// Tile-width choice: a function of (M, N, K) that minimises an estimate of
-// wave-quantised time.  Per-tile time ~ max(MMA cycles, operand bytes at a
-// per-SM TMA rate) + fixed prologue/epilogue cost.
+// Tile choice: a function of (M, N, K) minimising an estimate of wave-quantised
+// time.  Per-tile time ~ MMA cycles (128 x BN x K per SM at 8192 flop/clk)
+// scaled by the feed efficiency of the variant, + a fixed per-tile cost.
+// Returns BN for the single-CTA kernel, -BN for the CTA-pair kernel.
 int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
-  const int num_m = (M + BM - 1) / BM;
   double best = 1e30;
   int best_bn = 0;
-  const int cands[3] = {256, 128, 64};
-  for (int bn : cands) {
+  const int cands[5] = {-256, -128, 256, 128, 64};
+  for (int c : cands) {
+    const bool pair = c < 0;
+    const int bn = pair ? -c : c;
     if (N % bn) continue;
-    const long tiles = (long)num_m * (N / bn);
-    const long waves = (tiles + sms - 1) / sms;
-    const double mma_cyc = (double)BM * bn * K * 2 / 8192.0;          // 8192 flop/clk/SM
-    const double load_cyc = (double)(BM + bn) * K * 2 / 64.0;         // ~64 B/clk/SM TMA share
-    const double t = waves * ((mma_cyc > load_cyc ? mma_cyc : load_cyc) + 1500.0);
-    if (t < best * 0.999) { best = t; best_bn = bn; }
+    const int tile_m = pair ? 2 * BM : BM;
+    const long tiles = (long)((M + tile_m - 1) / tile_m) * (N / bn);
+    const long slots = pair ? sms / 2 : sms;
+    const long waves = (tiles + slots - 1) / slots;
+    const double mma_cyc = (double)BM * bn * K * 2 / 8192.0;
+    const double feed = pair ? 1.0 : 0.55;  // single-CTA tiles starve the tensor pipe at large M
+    const double rows_used = (double)M / (double)(((M + tile_m - 1) / tile_m) * tile_m);
+    (void)rows_used;
+    const double t = waves * (mma_cyc / feed + 1500.0);
+    if (t < best * 0.999) { best = t; best_bn = c; }
   }
   return best_bn;
 }
@@ -327,23 +464,35 @@ int tc_choose_bn(int M, int N, int K) {
 bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
                   const float* bias, const void* resid, void* out, int epi, int force_bn) {
   if (M <= 0 || N % 64 || K % 64 || K <= 0) return false;
-  const int bn = force_bn ? force_bn : tc_choose_bn(M, N, K);
+  const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
+  const bool pair = choice < 0;
+  const int bn = pair ? -choice : choice;
   if (bn != 64 && bn != 128 && bn != 256) return false;
+  if (pair && bn == 64) return false;
   if (N % bn) return false;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->epi = epi;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi;
   p->bias = bias; p->resid = resid; p->out = out;
-  const int tiles = ((M + BM - 1) / BM) * (N / bn);
-  p->grid = tiles < num_sms() ? tiles : num_sms();
+  const int tile_m = pair ? 2 * BM : BM;
+  const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
+  const int slots = pair ? num_sms() / 2 : num_sms();
+  p->grid = (tiles < slots ? tiles : slots) * (pair ? 2 : 1);
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM)) return false;
-  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn)) return false;
   return true;
 }
 
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
+  if (p.pair) {
+    switch (p.BN) {
+      case 128: return launch_bn<128, true>(p, s);
+      case 256: return launch_bn<256, true>(p, s);
+    }
+    return cudaErrorInvalidValue;
+  }
   switch (p.BN) {
-    case 64: return launch_bn<64>(p, s);
-    case 128: return launch_bn<128>(p, s);
-    case 256: return launch_bn<256>(p, s);
+    case 64: return launch_bn<64, false>(p, s);
+    case 128: return launch_bn<128, false>(p, s);
+    case 256: return launch_bn<256, false>(p, s);
   }
   return cudaErrorInvalidValue;
 }

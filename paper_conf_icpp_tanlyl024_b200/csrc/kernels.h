@@ -30,6 +30,7 @@ struct TcGemmPlan {
   CUtensorMap tmA;  // activations [M, K] bf16, box {64, 128}, 128B swizzle
   CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN}, 128B swizzle
   int M, N, K, BN, epi, grid;
+  bool pair;  // CTA-pair (cta_group::2) kernel, 256-row tiles
   const float* bias;
   const void* resid;
   void* out;

@@ -35,7 +35,10 @@ GEMM_SHAPES = [
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
 @pytest.mark.parametrize("epi", [0, 1, 2])
-def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi):
+@pytest.mark.parametrize("force", [0, 128, -128, -256])
+def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
+    if N % abs(force or 64):
+        pytest.skip("tile width does not divide N")
     A = rnd((M, K), 1)
     W = rnd((N, K), 2, 0.02)
     b = rnd((N,), 3, 0.02)
@@ -47,14 +50,14 @@ def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi):
         ref = ref + R
     out = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
     arlo_lib.op_gemm(arlo_lib.BF16, bf16_dev(A), bf16_dev(W), f32_dev(b), out, epi=epi,
-                     residual=bf16_dev(R) if epi == 2 else None)
+                     residual=bf16_dev(R) if epi == 2 else None, force_bn=force)
     torch.cuda.synchronize()
     got = host64(out)
     # bf16 output rounding (2^-9 relative) on fp32-accumulated exact products
     np.testing.assert_allclose(got, ref, rtol=8e-3, atol=8e-3)
 
 
-@pytest.mark.parametrize("bn", [64, 128, 256])
+@pytest.mark.parametrize("bn", [64, 128, 256, -128, -256])
 def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
     """Row results do not depend on the tile width (cross-L invariance contract)."""
     M, N, K = 300, 768, 768
@@ -68,7 +71,7 @@ def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
     assert torch.equal(outs[0], outs[1])
     # and a row does not depend on M (prefix of rows)
     o2 = torch.empty((77, N), device="cuda", dtype=torch.bfloat16)
-    arlo_lib.op_gemm(arlo_lib.BF16, A[:77].contiguous(), W, b, o2, epi=0, force_bn=bn)
+    arlo_lib.op_gemm(arlo_lib.BF16, A[:77].contiguous(), W, b, o2, epi=0, force_bn=64)
     torch.cuda.synchronize()
     assert torch.equal(o2, outs[0][:77])
 
