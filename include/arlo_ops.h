@@ -65,6 +65,13 @@ int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, cons
                  const void* w_p, const float* b_p, const void* w_c, const float* b_c,
                  float* pooled, float* logits, void* stream);
 
+/*
+ * Profiling hook (tools/gemm_trace.py): when `buf` is a DEVICE buffer of
+ * >= 64 * grid uint64 entries, later single-CTA GEMM launches write
+ * %globaltimer stamps of their pipeline events into it; NULL turns it off.
+ */
+int arlo_debug_gemm_trace(void* buf);
+
 #ifdef __cplusplus
 }
 #endif

@@ -31,9 +31,27 @@ namespace arlo {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int kEpiWarps = 16;  // 4 warpgroups: each TMEM lane quarter is drained by 4 warps
-constexpr int kThreads = 64 + 32 * kEpiWarps;  // warp 0 TMA, warp 1 MMA, warps 2.. epilogue
+constexpr int kEpiWarps = 8;                   // warps 0-7: two per TMEM lane quarter
+constexpr int kProducerWarp = kEpiWarps;       // warp 8: TMA producer
+constexpr int kMmaWarp = kEpiWarps + 1;        // warp 9: MMA issuer
+constexpr int kThreads = 32 * (kEpiWarps + 2);
 constexpr int kAccStages = 2;
+constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 staging tile (SWIZZLE_64B)
+constexpr int kStagingBytes = kEpiWarps * 2 * kStgBytes;  // double-buffered per epilogue warp
+constexpr int kSmemBudget = 229376;            // 224 KB of the 227 KB opt-in maximum
+
+// Optional event trace (tools/gemm_trace.py): when g_trace != nullptr every CTA
+// writes %globaltimer stamps to g_trace[blockIdx.x * 64 + slot].  One
+// predictable branch per event; never set in production.
+__device__ unsigned long long* g_trace = nullptr;
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ void trace(int slot) {
+  if (g_trace != nullptr && slot < 64) g_trace[blockIdx.x * 64 + slot] = gtimer();
+}
 
 constexpr int tmem_cols_for(int n) {
   return n <= 32 ? 32 : n <= 64 ? 64 : n <= 128 ? 128 : n <= 256 ? 256 : 512;
@@ -48,83 +66,90 @@ struct TcCfg {
   static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
   static constexpr int B_BYTES = B_ROWS * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (192 * 1024) / STAGE_BYTES;
+  static constexpr int STAGES_FIT = (kSmemBudget - kStagingBytes) / STAGE_BYTES;
+  static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int TMEM_COLS = tmem_cols_for(kAccStages * BN);
   static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages) + 16;
-  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + BAR_BYTES;
-  static constexpr int TILE_M = PAIR ? 2 * BM : BM;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + kStagingBytes + BAR_BYTES;
+  static_assert(SMEM <= 232448, "shared memory budget");
 };
 
-// Epilogue of one accumulator tile for one warp: TMEM lane quarter q (rows),
-// column group cg (BN/4 columns).  Software-pipelined over 16-column chunks:
-// the TMEM load, bias and residual of chunk c+1 are in flight while chunk c is
-// computed and stored; `release()` is called as soon as the last TMEM load of
-// the tile has completed so the MMA warp can reuse the accumulator buffer.
+// Epilogue of one accumulator tile for one warp: TMEM lane quarter q (32
+// rows), column half cg (BN/2 columns), processed in 32-column chunks.  For
+// each chunk: tcgen05.ld (the next chunk's load, bias and residual are issued
+// before this chunk is computed), bias / GELU / residual in fp32, RNE to bf16,
+// st.shared into a 64-byte-swizzled 32x32 staging tile, then one TMA bulk
+// tensor store of the tile (coalesced, asynchronous; rows >= M clipped by the
+// tensor map).  `release()` fires once the last TMEM load has completed.
 template <int BN, int EPI, typename Release>
-__device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row, int n0, int M,
+__device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int N, const float* __restrict__ bias,
-                                              const bf16* __restrict__ resid, bf16* __restrict__ out,
-                                              Release release) {
-  constexpr int COLS = BN / 4;
-  constexpr int NC = COLS / 16;
+                                              const bf16* __restrict__ resid, const CUtensorMap* tmC,
+                                              uint8_t* stg, int& sc, Release release) {
+  constexpr int COLS = BN / 2;
+  constexpr int NC = COLS / 32;
+  const int row = row0 + lane;
   const bool row_ok = row < M;
   const int col0 = n0 + cg * COLS;
   const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
   const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
-  uint4* out4 = reinterpret_cast<uint4*>(out + (size_t)row * N + col0);
   const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16) + cg * COLS;
-  uint32_t r[2][16];
-  float4 bv[2][4];
-  uint4 rv[2][2];
+  uint32_t r[2][32];
+  uint4 rv[2][4];
+  if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-  for (int j = 0; j < 4; ++j) bv[0][j] = __ldg(bias4 + j);
-  if (EPI == EPI_BIAS_RESID && row_ok) { rv[0][0] = __ldg(res4); rv[0][1] = __ldg(res4 + 1); }
-  ptx::tmem_ld_32x32b_x16(t_row, r[0]);
+    for (int j = 0; j < 4; ++j) rv[0][j] = __ldg(res4 + j);
+  }
+  ptx::tmem_ld_32x32b_x32(t_row, r[0]);
   ptx::tmem_wait_ld();
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
     const int cur = c & 1, nxt = cur ^ 1;
     if (c + 1 < NC) {
-      ptx::tmem_ld_32x32b_x16(t_row + (c + 1) * 16, r[nxt]);
-#pragma unroll
-      for (int j = 0; j < 4; ++j) bv[nxt][j] = __ldg(bias4 + (c + 1) * 4 + j);
+      ptx::tmem_ld_32x32b_x32(t_row + (c + 1) * 32, r[nxt]);
       if (EPI == EPI_BIAS_RESID && row_ok) {
-        rv[nxt][0] = __ldg(res4 + (c + 1) * 2);
-        rv[nxt][1] = __ldg(res4 + (c + 1) * 2 + 1);
+#pragma unroll
+        for (int j = 0; j < 4; ++j) rv[nxt][j] = __ldg(res4 + (c + 1) * 4 + j);
       }
     }
-    float v[16];
+    uint32_t pk[16];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float4 b4 = __ldg(bias4 + c * 8 + j);
+      float v0 = __uint_as_float(r[cur][4 * j + 0]) + b4.x;
+      float v1 = __uint_as_float(r[cur][4 * j + 1]) + b4.y;
+      float v2 = __uint_as_float(r[cur][4 * j + 2]) + b4.z;
+      float v3 = __uint_as_float(r[cur][4 * j + 3]) + b4.w;
+      if (EPI == EPI_BIAS_GELU) {
+        v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
+      }
+      if (EPI == EPI_BIAS_RESID) {
+        const uint4 u = rv[cur][j >> 1];
+        const float2 fa = unpack_bf16x2((j & 1) ? u.z : u.x), fb = unpack_bf16x2((j & 1) ? u.w : u.y);
+        v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
+      }
+      pk[2 * j] = pack_bf16x2(v0, v1);
+      pk[2 * j + 1] = pack_bf16x2(v2, v3);
+    }
+    // staging buffer (sc & 1) was last used two chunks ago: make sure its TMA store has read it
+    uint8_t* buf = stg + (sc & 1) * kStgBytes;
+    if (sc >= 2) {
+      if (lane == 0) ptx::bulk_wait_read<1>();
+      __syncwarp();
+    }
 #pragma unroll
     for (int j = 0; j < 4; ++j) {
-      v[4 * j + 0] = __uint_as_float(r[cur][4 * j + 0]) + bv[cur][j].x;
-      v[4 * j + 1] = __uint_as_float(r[cur][4 * j + 1]) + bv[cur][j].y;
-      v[4 * j + 2] = __uint_as_float(r[cur][4 * j + 2]) + bv[cur][j].z;
-      v[4 * j + 3] = __uint_as_float(r[cur][4 * j + 3]) + bv[cur][j].w;
+      const int sw = j ^ ((lane >> 1) & 3);  // SWIZZLE_64B: 16-byte chunk ^= address bits [7:8]
+      *reinterpret_cast<uint4*>(buf + lane * 64 + sw * 16) =
+          make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
     }
-    if (EPI == EPI_BIAS_GELU) {
-#pragma unroll
-      for (int j = 0; j < 16; ++j) v[j] = gelu_erf_fast(v[j]);
+    ptx::fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+      ptx::tma_store_2d(tmC, buf, col0 + c * 32, row0);
+      ptx::bulk_commit();
     }
-    if (EPI == EPI_BIAS_RESID && row_ok) {
-#pragma unroll
-      for (int j = 0; j < 2; ++j) {
-        const uint4 u = rv[cur][j];
-        float2 f0 = unpack_bf16x2(u.x), f1 = unpack_bf16x2(u.y), f2 = unpack_bf16x2(u.z), f3 = unpack_bf16x2(u.w);
-        v[8 * j + 0] += f0.x; v[8 * j + 1] += f0.y; v[8 * j + 2] += f1.x; v[8 * j + 3] += f1.y;
-        v[8 * j + 4] += f2.x; v[8 * j + 5] += f2.y; v[8 * j + 6] += f3.x; v[8 * j + 7] += f3.y;
-      }
-    }
-    if (row_ok) {
-#pragma unroll
-      for (int j = 0; j < 2; ++j) {
-        uint4 u;
-        u.x = pack_bf16x2(v[8 * j + 0], v[8 * j + 1]);
-        u.y = pack_bf16x2(v[8 * j + 2], v[8 * j + 3]);
-        u.z = pack_bf16x2(v[8 * j + 4], v[8 * j + 5]);
-        u.w = pack_bf16x2(v[8 * j + 6], v[8 * j + 7]);
-        out4[c * 2 + j] = u;
-      }
-    }
+    ++sc;
     ptx::tmem_wait_ld();
     if (c == (NC >= 2 ? NC - 2 : 0)) {
       ptx::tc_fence_before();
@@ -137,14 +162,15 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
 template <int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-               int M, int N, int K, const float* __restrict__ bias, const bf16* __restrict__ resid,
-               bf16* __restrict__ out) {
+               const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
+               const bf16* __restrict__ resid) {
   using C = TcCfg<BN, false>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
@@ -156,9 +182,10 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   const int tiles = num_m * num_n;
   const int kblocks = K / BK;
 
-  if (warp == 0 && lane == 0) {
+  if (warp == kProducerWarp && lane == 0) {
     ptx::tma_prefetch_desc(&tmA);
     ptx::tma_prefetch_desc(&tmB);
+    ptx::tma_prefetch_desc(&tmC);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -169,19 +196,22 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 1) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
+  if (warp == kMmaWarp) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (threadIdx.x == 0) trace(0);
 
-  if (warp == 0) {
+  if (warp == kProducerWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+      int it = 0;
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
         const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+        trace(2 + 6 * it);
         for (int kb = 0; kb < kblocks; ++kb) {
           ptx::mbar_wait(&empty[stage], phase ^ 1);
           ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
@@ -191,7 +221,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         }
       }
     }
-  } else if (warp == 1) {
+  } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------- MMA issuer
     if (lane == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
@@ -199,13 +229,16 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+      int it = 0;
+      for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
         ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
+        trace(3 + 6 * it);
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < kblocks; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
+          if (kb == 0) trace(4 + 6 * it);
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
@@ -217,30 +250,38 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
         ptx::mma_commit(&tfull[acc]);
+        trace(5 + 6 * it);
         if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
       }
     }
   } else {
     // --------------------------------------------------------------- epilogue
     // warp w may only touch TMEM lanes 32*(w%4)..+31 (rows of the tile); the
-    // four warps sharing a quarter split the BN columns into 4 groups.
-    const int q = warp & 3, cg = (warp - 2) >> 2;
+    // two warps sharing a quarter take one column half each.
+    const int q = warp & 3, cg = warp >> 2;
+    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x) {
+    int it = 0;
+    for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
       const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
+      if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32 + lane, n0, M, N, bias, resid, out,
-                             [te]() { ptx::mbar_arrive(te); });
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, N, bias, resid, &tmC, stg,
+                             sc, [te]() { ptx::mbar_arrive(te); });
+      if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
+    if (lane == 0) ptx::bulk_wait<0>();
   }
 
   ptx::tc_fence_before();
   __syncthreads();
-  if (warp == 1) {
+  if (threadIdx.x == 0) trace(1);
+  if (warp == kMmaWarp) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem_base, C::TMEM_COLS);
   }
@@ -252,18 +293,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 // leader's full barrier; the leader's commits arrive on both CTAs' empty and
 // tfull barriers (multicast); both CTAs' epilogue warps arrive on the
 // leader's tempty barrier.  Halves the L2->SM operand traffic per FLOP and
-// doubles the smem pipeline depth relative to the single-CTA kernel.
+// deepens the smem pipeline relative to the single-CTA kernel.
 template <int BN, int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                    int M, int N, int K, const float* __restrict__ bias, const bf16* __restrict__ resid,
-                    bf16* __restrict__ out) {
+                    const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
+                    const bf16* __restrict__ resid) {
   using C = TcCfg<BN, true>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
-  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
@@ -277,9 +319,10 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   const int tiles = num_m * num_n;
   const int kblocks = K / BK;
 
-  if (warp == 0 && lane == 0) {
+  if (warp == kProducerWarp && lane == 0) {
     ptx::tma_prefetch_desc(&tmA);
     ptx::tma_prefetch_desc(&tmB);
+    ptx::tma_prefetch_desc(&tmC);
     for (int s = 0; s < C::STAGES; ++s) {
       ptx::mbar_init(&full[s], 1);
       ptx::mbar_init(&empty[s], 1);
@@ -290,13 +333,13 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 1) ptx::tmem_alloc_pair(tmem_slot, C::TMEM_COLS);
+  if (warp == kMmaWarp) ptx::tmem_alloc_pair(tmem_slot, C::TMEM_COLS);
   ptx::tc_fence_before();
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
-  if (warp == 0) {
+  if (warp == kProducerWarp) {
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
@@ -313,7 +356,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
         }
       }
     }
-  } else if (warp == 1) {
+  } else if (warp == kMmaWarp) {
     if (lane == 0 && rank == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(2 * BM, BN);
       int stage = 0;
@@ -321,11 +364,11 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       int acc = 0;
       uint32_t acc_phase = 0;
       for (int tile = pair; tile < tiles; tile += npairs) {
-        ptx::mbar_wait_cluster(&tempty[acc], acc_phase ^ 1);
+        ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < kblocks; ++kb) {
-          ptx::mbar_wait_cluster(&full[stage], phase);
+          ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
@@ -342,7 +385,9 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       }
     }
   } else {
-    const int q = warp & 3, cg = (warp - 2) >> 2;
+    const int q = warp & 3, cg = warp >> 2;
+    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
     for (int tile = pair; tile < tiles; tile += npairs) {
@@ -350,15 +395,16 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32 + lane, n0, M, N, bias, resid, out,
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, N, bias, resid, &tmC, stg, sc,
                              [te]() { ptx::mbar_arrive_cluster(te); });
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
+    if (lane == 0) ptx::bulk_wait<0>();
   }
 
   ptx::tc_fence_before();
   ptx::cluster_sync();
-  if (warp == 1) {
+  if (warp == kMmaWarp) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc_pair(tmem_base, C::TMEM_COLS);
   }
@@ -393,8 +439,7 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  kern<<<p.grid, kThreads, C::SMEM, s>>>(p.tmA, p.tmB, p.M, p.N, p.K, p.bias, (const bf16*)p.resid,
-                                         (bf16*)p.out);
+  kern<<<p.grid, kThreads, C::SMEM, s>>>(p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias, (const bf16*)p.resid);
   return cudaGetLastError();
 }
 
@@ -410,6 +455,10 @@ cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
 
 }  // namespace
 
+int set_gemm_trace(unsigned long long* buf) {
+  return (int)cudaMemcpyToSymbol(g_trace, &buf, sizeof(buf));
+}
+
 int num_sms() {
   static int n = 0;
   if (n == 0) {
@@ -421,7 +470,7 @@ int num_sms() {
 }
 
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
-                         uint32_t box_inner, uint32_t box_outer) {
+                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes) {
   EncodeTiledFn fn = get_encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {inner, outer};
@@ -429,7 +478,11 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
-                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                  estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  swizzle_bytes == 128  ? CU_TENSOR_MAP_SWIZZLE_128B
+                  : swizzle_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                  : swizzle_bytes == 32 ? CU_TENSOR_MAP_SWIZZLE_32B
+                                        : CU_TENSOR_MAP_SWIZZLE_NONE,
                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
@@ -476,8 +529,9 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
   const int slots = pair ? num_sms() / 2 : num_sms();
   p->grid = (tiles < slots ? tiles : slots) * (pair ? 2 : 1);
-  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM)) return false;
-  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn, 128)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, 32, 32, 64)) return false;
   return true;
 }
 

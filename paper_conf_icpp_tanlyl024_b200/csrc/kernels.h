@@ -14,6 +14,7 @@ enum DType { DT_BF16 = 0, DT_FP32 = 1 };
 enum Epi { EPI_BIAS = 0, EPI_BIAS_GELU = 1, EPI_BIAS_RESID = 2 };
 
 int num_sms();
+int set_gemm_trace(unsigned long long* buf);  // profiling hook, nullptr = off
 
 // ---- a1: embedding + LN;  a5/a8: LN ------------------------------------------------------
 cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int32_t* ids,
@@ -28,7 +29,8 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
 // launch is then a plain kernel launch that CUDA graphs can capture.
 struct TcGemmPlan {
   CUtensorMap tmA;  // activations [M, K] bf16, box {64, 128}, 128B swizzle
-  CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN}, 128B swizzle
+  CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN (BN/2 for a pair)}, 128B swizzle
+  CUtensorMap tmC;  // output      [M, N] bf16, box {32, 32}, 64B swizzle (epilogue TMA stores)
   int M, N, K, BN, epi, grid;
   bool pair;  // CTA-pair (cta_group::2) kernel, 256-row tiles
   const float* bias;
@@ -55,6 +57,6 @@ cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, con
 
 // Resolve cuTensorMapEncodeTiled through the runtime (no link-time libcuda dependency).
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
-                         uint32_t box_inner, uint32_t box_outer);
+                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes);
 
 }  // namespace arlo

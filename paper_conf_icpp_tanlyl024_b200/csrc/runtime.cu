@@ -507,3 +507,8 @@ extern "C" int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int3
             "head");
   return ARLO_OK;
 }
+
+extern "C" int arlo_debug_gemm_trace(void* buf) {
+  cudaError_t e = (cudaError_t)set_gemm_trace((unsigned long long*)buf);
+  return e == cudaSuccess ? ARLO_OK : cuda_fail(e, "arlo_debug_gemm_trace");
+}

@@ -1,0 +1,47 @@
+"""Per-CTA pipeline timeline of one single-CTA tcgen05 GEMM launch (globaltimer stamps).
+
+    python tools/gemm_trace.py M N K [BN]
+Slots per CTA: 0 start (after setup), 1 end; per tile i: 2+6i producer starts tile,
+3+6i MMA got accumulator, 4+6i first stage landed, 5+6i last MMA issued,
+6+6i epilogue got tile, 7+6i epilogue done (warp 2).
+"""
+import os
+import sys
+
+import numpy as np
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_icpp_tanlyl024_b200 import arlo  # noqa: E402
+
+M, N, K = (int(x) for x in sys.argv[1:4])
+bn = int(sys.argv[4]) if len(sys.argv) > 4 else 256
+dev = torch.device("cuda")
+A = torch.randn(M, K, device=dev).to(torch.bfloat16)
+W = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
+b = torch.zeros(N, device=dev)
+out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
+for _ in range(3):
+    arlo.op_gemm(arlo.BF16, A, W, b, out, force_bn=bn)
+buf = torch.zeros(148 * 64, dtype=torch.int64, device=dev)
+arlo.check(arlo.lib.arlo_debug_gemm_trace(buf.data_ptr()))
+arlo.op_gemm(arlo.BF16, A, W, b, out, force_bn=bn)
+torch.cuda.synchronize()
+arlo.check(arlo.lib.arlo_debug_gemm_trace(None))
+t = buf.cpu().numpy().reshape(148, 64).astype(np.float64)
+grid = int((t[:, 0] > 0).sum())
+t = t[:grid]
+t0 = t[:, 0].min()
+rel = np.where(t > 0, (t - t0) / 1e3, np.nan)  # microseconds
+print(f"M={M} N={N} K={K} BN={bn} grid={grid}  kernel span {np.nanmax(rel[:, 1]):.2f} us (from first CTA start)")
+print("start spread: min %.2f max %.2f us" % (np.nanmin(rel[:, 0]), np.nanmax(rel[:, 0])))
+for i in range(4):
+    cols = rel[:, 2 + 6 * i: 8 + 6 * i]
+    if np.all(np.isnan(cols[:, 0])):
+        break
+    med = np.nanmedian(cols, axis=0)
+    print(f"tile {i}: producer {med[0]:7.2f} | mma acc {med[1]:7.2f} first-stage {med[2]:7.2f} last-mma {med[3]:7.2f}"
+          f" | epi start {med[4]:7.2f} done {med[5]:7.2f}   (median over CTAs, us)")
+print("end: median %.2f max %.2f us" % (np.nanmedian(rel[:, 1]), np.nanmax(rel[:, 1])))
+for c in (0, 1, grid - 1):
+    print(f"cta {c}:", " ".join(f"{x:6.2f}" for x in rel[c, :14] if not np.isnan(x)))
