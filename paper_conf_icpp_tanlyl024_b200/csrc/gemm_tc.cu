@@ -487,15 +487,18 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
   return r == CUDA_SUCCESS;
 }
 
-// Tile choice: a function of (M, N, K) minimising an estimate of wave-quantised
-// time.  Per-tile time ~ MMA cycles (128 x BN x K per SM at 8192 flop/clk)
-// scaled by the feed efficiency of the variant, + a fixed per-tile cost.
-// Returns BN for the single-CTA kernel, -BN for the CTA-pair kernel.
+// Tile choice: a function of (M, N, K) only (never of the data), minimising a
+// wave-quantised time estimate.  Per tile: MMA time of a 128 x BN x K slab at
+// 8192 flop/clk/SM divided by a feed efficiency measured on B200
+// (tools/gemm_sweep.py: CTA pairs and single CTAs at BN >= 192 sustain the
+// tensor pipe; BN = 128 tiles re-read A twice as often and run ~30% slower),
+// plus a fixed ~1 us tile prologue/epilogue cost.  Returns BN for the
+// single-CTA kernel, -BN for the CTA-pair kernel.
 int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
   double best = 1e30;
   int best_bn = 0;
-  const int cands[5] = {-256, -128, 256, 128, 64};
+  const int cands[7] = {-256, -192, 256, 192, -128, 128, 64};
   for (int c : cands) {
     const bool pair = c < 0;
     const int bn = pair ? -c : c;
@@ -504,11 +507,9 @@ int tc_choose_bn(int M, int N, int K) {
     const long tiles = (long)((M + tile_m - 1) / tile_m) * (N / bn);
     const long slots = pair ? sms / 2 : sms;
     const long waves = (tiles + slots - 1) / slots;
-    const double mma_cyc = (double)BM * bn * K * 2 / 8192.0;
-    const double feed = pair ? 1.0 : 0.55;  // single-CTA tiles starve the tensor pipe at large M
-    const double rows_used = (double)M / (double)(((M + tile_m - 1) / tile_m) * tile_m);
-    (void)rows_used;
-    const double t = waves * (mma_cyc / feed + 1500.0);
+    const double mma_us = (double)BM * bn * K * 2 / 8192.0 / 1.9e3;
+    double eff = bn >= 192 ? (pair ? 1.0 : 0.92) : (bn == 128 ? 0.68 : 0.5);
+    const double t = waves * (mma_us / eff + 1.0);
     if (t < best * 0.999) { best = t; best_bn = c; }
   }
   return best_bn;
@@ -520,7 +521,7 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
   const bool pair = choice < 0;
   const int bn = pair ? -choice : choice;
-  if (bn != 64 && bn != 128 && bn != 256) return false;
+  if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn == 64) return false;
   if (N % bn) return false;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi;
@@ -539,6 +540,7 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
   if (p.pair) {
     switch (p.BN) {
       case 128: return launch_bn<128, true>(p, s);
+      case 192: return launch_bn<192, true>(p, s);
       case 256: return launch_bn<256, true>(p, s);
     }
     return cudaErrorInvalidValue;
@@ -546,6 +548,7 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
   switch (p.BN) {
     case 64: return launch_bn<64, false>(p, s);
     case 128: return launch_bn<128, false>(p, s);
+    case 192: return launch_bn<192, false>(p, s);
     case 256: return launch_bn<256, false>(p, s);
   }
   return cudaErrorInvalidValue;

@@ -11,7 +11,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_icpp_tanlyl024_b200 import arlo  # noqa: E402
 
 SHAPES = [(4096, 2304, 768), (4096, 3072, 768), (4096, 768, 3072), (8192, 8192, 8192), (4096, 4096, 8192),
-          (16384, 3072, 768), (16384, 1024, 4096), (2048, 768, 768), (64, 2304, 768), (128, 768, 3072)]
+          (16384, 3072, 768), (16384, 1024, 4096), (16384, 768, 3072), (8192, 2304, 768), (2048, 768, 768),
+          (64, 2304, 768), (128, 768, 3072)]
 
 
 def time_op(fn, reps=20):
@@ -42,7 +43,7 @@ def time_op(fn, reps=20):
 
 
 def main():
-    forces = [int(x) for x in sys.argv[1:]] or [0, 256, 128, -256, -128]
+    forces = [int(x) for x in sys.argv[1:]] or [0, 256, 192, 128, -256, -192, -128]
     dev = torch.device("cuda")
     for (M, N, K) in SHAPES:
         A = torch.randn(M, K, device=dev).to(torch.bfloat16)
