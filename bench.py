@@ -305,22 +305,35 @@ def main():
 
 def roofline_dominant(arlo, torch, dev, stream, step_times):
     """Dominant kernel: the FFN1 tcgen05 GEMM (+bias+GELU) of the L=128, b=32 runtime
-    (M=4096, N=3072, K=768), the single largest GEMM share of a step.  Timed live
-    with a CUDA event pair around each launch on the launching stream."""
+    (M=4096, N=3072, K=768), the single largest GEMM share of a step, in the tile
+    configuration the runtime graphs use.  Timed live on the launching stream:
+    REPS launches captured in one CUDA graph (as in the runtime graphs, so no host
+    launch gaps), CUDA events around each replay, averaged per launch."""
     M, N, K = 4096, 3072, 768
+    REPS = 20
     A = torch.randn(M, K, device=dev).to(torch.bfloat16)
     Wt = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
     b = torch.zeros(N, device=dev)
     out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-    for _ in range(5):
+    for _ in range(3):
         arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
-    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(50)]
-    for a, e in ev:
-        a.record(stream)
-        arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
-        e.record(stream)
     torch.cuda.synchronize()
-    t = float(np.mean([a.elapsed_time(e) for a, e in ev])) / 1e3
+    g = torch.cuda.CUDAGraph()
+    with torch.cuda.graph(g, stream=stream):
+        for _ in range(REPS):
+            arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
+    g.replay()
+    torch.cuda.synchronize()
+    ts = []
+    for _ in range(10):
+        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        g.replay()
+        e.record(stream)
+        torch.cuda.synchronize()
+        ts.append(a.elapsed_time(e) / REPS)
+    t = float(np.mean(ts)) / 1e3
+    choice = arlo.gemm_tile_choice(M, N, K)
     flops = metrics.gemm_flops(M, N, K)
     peaks = {}
     try:
@@ -334,7 +347,8 @@ def roofline_dominant(arlo, torch, dev, stream, step_times):
     except Exception:
         pass
     achieved = flops / t / 1e12
-    return {"kernel": "gemm_tc_kernel<256, GELU> (FFN1, M=4096 N=3072 K=768)", "bound": "tensor",
+    kname = (f"gemm_tc_pair_kernel<{-choice}, GELU>" if choice < 0 else f"gemm_tc_kernel<{choice}, GELU>")
+    return {"kernel": kname + " (FFN1, M=4096 N=3072 K=768)", "bound": "tensor",
             "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
             "traffic": traffic, "peak_source": "MEASURED_PEAKS.json bf16_tflops (burst)" if peaks else
             "fallback 1590 TFLOP/s (B200_PROFILING.md)", "launch_us": t * 1e6,

@@ -65,6 +65,10 @@ int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, cons
                  const void* w_p, const float* b_p, const void* w_c, const float* b_c,
                  float* pooled, float* logits, void* stream);
 
+/* The tile configuration arlo_op_gemm / the runtime graphs use for (M, N, K):
+ * BN for the single-CTA kernel, -BN for the CTA-pair kernel, 0 if unsupported. */
+int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K);
+
 /*
  * Profiling hook (tools/gemm_trace.py): when `buf` is a DEVICE buffer of
  * >= 64 * grid uint64 entries, later single-CTA GEMM launches write
