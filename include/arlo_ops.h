@@ -52,7 +52,8 @@ int arlo_op_embed(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t vocab,
  * qkv [B*L, 3H] (Q | K | V, head j at columns j*64), o [B*L, H].  Query row t
  * of sequence b attends keys 0..lengths[b]-1 with scale 1/8; key tiles past
  * lengths[b] are skipped; rows of a query tile lying wholly at t >=
- * lengths[b] are written as 0 (never read by a real token).
+ * lengths[b] are written as 0 (never read by a real token).  Query tiles are
+ * 128 rows (bf16: tcgen05 kernel, requires L <= 512).
  */
 int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t heads, const void* qkv,
                       const int32_t* lengths, void* o, void* stream);

@@ -11,211 +11,246 @@
 // reading S5).  A real query row's result depends only on keys < len_b, so it
 // is bitwise identical for every runtime L >= len_b.
 //
-// bf16 path: flash-attention style, one CTA per (64-query tile, head,
-// sequence), 4 warps x 16 query rows, S = QK^T and O += PV on mma.sync
-// m16n8k16 (bf16 in, fp32 accumulate), online softmax in fp32 with exp2,
-// K/V 64-key tiles double-buffered in 128B-XOR-swizzled shared memory via
-// cp.async.  fp32 check mode: one warp per query row, exact fp32 FFMA.
+// bf16 path (attn_tc_kernel): flash attention on the 5th-gen tensor cores —
+// tcgen05.mma with S and O accumulators in TMEM, operands staged by TMA, one
+// CTA per (128-query tile, head, sequence), 128-key tiles, L <= 512.
+// fp32 check mode: one warp per query row, exact fp32 FFMA.
 #include "common.cuh"
 #include "kernels.h"
+#include "ptx.cuh"
 
 namespace arlo {
 namespace {
 
-constexpr int D = 64;       // head dim (all configs)
-constexpr int QT = 64;      // query rows per CTA
-constexpr int KT = 64;      // keys per tile
+constexpr int D = 64;        // head dim (all configs)
+constexpr int AQ = 128;      // queries per CTA (TMEM lanes)
+constexpr int AK = 128;      // keys per tile
+constexpr int kMaxKT = 4;    // L <= 512
+constexpr int kAttnThreads = 192;  // warps 0-3 softmax (one TMEM lane quarter each), 4 TMA, 5 MMA
+constexpr int kTileBytes = 128 * 128;   // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
+constexpr int kPBytes = 2 * kTileBytes;  // P tile: 128 queries x 128 keys = two 64-key K-blocks
+constexpr int kAttnSmem = 1024 + kTileBytes * (1 + 2 * kMaxKT) + 2 * kPBytes + 256;
+constexpr uint32_t kTmemCols = 512;      // S double buffer (2 x 128) + O (64)
+constexpr uint32_t kOCol = 256;
+// lazy rescale: keep a stale row max unless a tile's max exceeds it by > 2^8 in p
+constexpr float kRescaleLog2 = 8.0f;
 
-__device__ __forceinline__ uint32_t swz(int row, int chunk) {  // byte offset in a [64][128B] tile
-  return (uint32_t)(row * 128 + ((chunk ^ (row & 7)) << 4));
-}
+__device__ __forceinline__ bool valid_key(int key, int len) { return key < len; }
 
-__device__ __forceinline__ void cp_async16(uint32_t saddr, const void* g, bool valid) {
-  const int n = valid ? 16 : 0;  // zero-fill when out of range
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(saddr), "l"(g), "r"(n) : "memory");
-}
-__device__ __forceinline__ void cp_async_commit() { asm volatile("cp.async.commit_group;" ::: "memory"); }
-template <int N>
-__device__ __forceinline__ void cp_async_wait() { asm volatile("cp.async.wait_group %0;" ::"n"(N) : "memory"); }
-
-__device__ __forceinline__ void ldsm_x4(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
-  asm volatile("ldmatrix.sync.aligned.m8n8.x4.shared.b16 {%0,%1,%2,%3}, [%4];"
-               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3) : "r"(addr));
-}
-__device__ __forceinline__ void ldsm_x4_t(uint32_t addr, uint32_t& r0, uint32_t& r1, uint32_t& r2, uint32_t& r3) {
-  asm volatile("ldmatrix.sync.aligned.m8n8.x4.trans.shared.b16 {%0,%1,%2,%3}, [%4];"
-               : "=r"(r0), "=r"(r1), "=r"(r2), "=r"(r3) : "r"(addr));
-}
-__device__ __forceinline__ void mma16816(float (&d)[4], const uint32_t (&a)[4], uint32_t b0, uint32_t b1) {
-  asm volatile(
-      "mma.sync.aligned.m16n8k16.row.col.f32.bf16.bf16.f32 {%0,%1,%2,%3}, {%4,%5,%6,%7}, {%8,%9}, "
-      "{%0,%1,%2,%3};"
-      : "+f"(d[0]), "+f"(d[1]), "+f"(d[2]), "+f"(d[3])
-      : "r"(a[0]), "r"(a[1]), "r"(a[2]), "r"(a[3]), "r"(b0), "r"(b1));
-}
-
-// Load a [64 rows][64 dims] bf16 tile (row stride ld elements) into swizzled smem.
-__device__ __forceinline__ void load_tile(uint32_t sbase, const bf16* g, int ld, int row0, int rows_valid) {
-  for (int i = threadIdx.x; i < 64 * 8; i += 128) {
-    const int r = i >> 3, c = i & 7;
-    const bool ok = (row0 + r) < rows_valid;
-    const bf16* src = g + (size_t)(ok ? r : 0) * ld + c * 8;
-    cp_async16(sbase + swz(r, c), src, ok);
-  }
-}
-
-__global__ void __launch_bounds__(128) attn_bf16_kernel(int L, int heads, const bf16* __restrict__ qkv,
-                                                        const int32_t* __restrict__ lengths,
-                                                        bf16* __restrict__ o) {
-  __shared__ __align__(128) uint8_t sQ[QT * 128];
-  __shared__ __align__(128) uint8_t sK[2][KT * 128];
-  __shared__ __align__(128) uint8_t sV[2][KT * 128];
+// One CTA = (128-query tile, head, sequence).  S_j = Q K_j^T (M=128, N=128,
+// K=64) and O += P_j V_j (M=128, N=64, K=128, V as MN-major B) on tcgen05 with
+// S double-buffered in TMEM; 4 softmax warps (thread = query row) read S_j from
+// TMEM, keep a lazily-rescaled running max (O rescaled in TMEM only when a
+// tile raises the max by > 2^8), write P_j as bf16 into 128B-swizzled smem
+// (the A operand of the PV MMA) and accumulate the row sum in fp32.  Q, every
+// K_j and V_j (<= 4 tiles each, L <= 512) are loaded once by TMA.  Key tiles
+// starting at >= len are never loaded or multiplied; keys >= len inside the
+// last tile get p = 0 exactly.
+__global__ void __launch_bounds__(kAttnThreads, 1)
+attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const int32_t* __restrict__ lengths,
+               bf16* __restrict__ o) {
   const int qt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
-  const int H = heads * D, ld = 3 * H;
+  const int H = heads * D;
   const int len = __ldg(lengths + b);
-  const int q0 = qt * QT;
-  const size_t row_base = (size_t)b * L;
+  const int q0 = qt * AQ;
+  const int row_base = b * L;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-
   if (q0 >= len) {  // wholly padded query tile (or empty slot): zeros
-    for (int i = threadIdx.x; i < QT * 8; i += 128) {
+    const int rows = min(AQ, L - q0);
+    for (int i = threadIdx.x; i < rows * 8; i += kAttnThreads) {
       const int r = i >> 3, c = i & 7;
-      if (q0 + r < L)
-        *reinterpret_cast<uint4*>(o + (row_base + q0 + r) * H + h * D + c * 8) = make_uint4(0, 0, 0, 0);
+      *reinterpret_cast<uint4*>(o + (size_t)(row_base + q0 + r) * H + h * D + c * 8) = make_uint4(0, 0, 0, 0);
     }
     return;
   }
-  const bf16* gq = qkv + row_base * ld + h * D;
-  const bf16* gk = gq + H;
-  const bf16* gv = gq + 2 * H;
-  const uint32_t aQ = (uint32_t)__cvta_generic_to_shared(sQ);
-  const uint32_t aK[2] = {(uint32_t)__cvta_generic_to_shared(sK[0]), (uint32_t)__cvta_generic_to_shared(sK[1])};
-  const uint32_t aV[2] = {(uint32_t)__cvta_generic_to_shared(sV[0]), (uint32_t)__cvta_generic_to_shared(sV[1])};
+  const int n_kt = (len + AK - 1) / AK;
 
-  const int n_kt = (len + KT - 1) / KT;
-  load_tile(aQ, gq + (size_t)q0 * ld, ld, q0, L);
-  load_tile(aK[0], gk, ld, 0, L);
-  load_tile(aV[0], gv, ld, 0, L);
-  cp_async_commit();
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK = sQ + kTileBytes;
+  uint8_t* sV = sK + kMaxKT * kTileBytes;
+  uint8_t* sP = sV + kMaxKT * kTileBytes;
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + 2 * kPBytes);
+  uint64_t* bar_v = bar_k + kMaxKT;
+  uint64_t* s_full = bar_v + kMaxKT;
+  uint64_t* p_full = s_full + 2;
+  uint64_t* pv_done = p_full + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2);
 
-  // softmax in base 2: p = 2^(s * scale*log2e - m)
-  const float sl2 = 0.125f * 1.4426950408889634f;
-  float m_i[2] = {-INFINITY, -INFINITY}, l_i[2] = {0.f, 0.f};
-  float acc_o[8][4];
-#pragma unroll
-  for (int i = 0; i < 8; ++i) acc_o[i][0] = acc_o[i][1] = acc_o[i][2] = acc_o[i][3] = 0.f;
-  uint32_t qf[4][4];
-  const int g = lane >> 2, t4 = lane & 3;
-
-  for (int kt = 0; kt < n_kt; ++kt) {
-    const int cur = kt & 1;
-    if (kt + 1 < n_kt) {
-      load_tile(aK[cur ^ 1], gk + (size_t)(kt + 1) * KT * ld, ld, (kt + 1) * KT, L);
-      load_tile(aV[cur ^ 1], gv + (size_t)(kt + 1) * KT * ld, ld, (kt + 1) * KT, L);
-      cp_async_commit();
-      cp_async_wait<1>();
-    } else {
-      cp_async_wait<0>();
+  if (warp == 4 && lane == 0) {
+    ptx::tma_prefetch_desc(&tm);
+    for (int j = 0; j < kMaxKT; ++j) {
+      ptx::mbar_init(&bar_k[j], 1);
+      ptx::mbar_init(&bar_v[j], 1);
     }
-    __syncthreads();
-    if (kt == 0) {
-#pragma unroll
-      for (int ks = 0; ks < 4; ++ks) {
-        const int i = lane >> 3;
-        const int r = warp * 16 + (i & 1) * 8 + (lane & 7);
-        ldsm_x4(aQ + swz(r, ks * 2 + (i >> 1)), qf[ks][0], qf[ks][1], qf[ks][2], qf[ks][3]);
-      }
+    for (int i = 0; i < 2; ++i) {
+      ptx::mbar_init(&s_full[i], 1);
+      ptx::mbar_init(&p_full[i], 4);
+      ptx::mbar_init(&pv_done[i], 1);
     }
-    // S = Q K^T for this warp's 16 rows x 64 keys
-    float s[8][4];
-#pragma unroll
-    for (int i = 0; i < 8; ++i) s[i][0] = s[i][1] = s[i][2] = s[i][3] = 0.f;
-#pragma unroll
-    for (int ks = 0; ks < 4; ++ks) {
-#pragma unroll
-      for (int np = 0; np < 4; ++np) {  // pairs of 8-key n-tiles
-        const int i = lane >> 3;
-        const int r = (np * 2 + (i >> 1)) * 8 + (lane & 7);
-        uint32_t b0, b1, b2, b3;
-        ldsm_x4(aK[cur] + swz(r, ks * 2 + (i & 1)), b0, b1, b2, b3);
-        mma16816(s[2 * np], qf[ks], b0, b1);
-        mma16816(s[2 * np + 1], qf[ks], b2, b3);
-      }
-    }
-    // mask keys >= len (only the last tile can hold any), online softmax
-    const int kbase = kt * KT;
-    float mx[2] = {-INFINITY, -INFINITY};
-#pragma unroll
-    for (int nt = 0; nt < 8; ++nt) {
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int key = kbase + nt * 8 + t4 * 2 + (e & 1);
-        if (key >= len) s[nt][e] = -INFINITY;
-        mx[e >> 1] = fmaxf(mx[e >> 1], s[nt][e]);
-      }
-    }
-    float scale_o[2];
-#pragma unroll
-    for (int r = 0; r < 2; ++r) {
-      mx[r] = fmaxf(mx[r], __shfl_xor_sync(0xffffffffu, mx[r], 1));
-      mx[r] = fmaxf(mx[r], __shfl_xor_sync(0xffffffffu, mx[r], 2));
-      const float m_new = fmaxf(m_i[r], mx[r] * sl2);  // key 0 is always real: finite
-      scale_o[r] = exp2f(m_i[r] - m_new);
-      m_i[r] = m_new;
-    }
-    float rs[2] = {0.f, 0.f};
-    uint32_t pf[4][4];  // P as bf16 A fragments, 4 k-steps of 16 keys
-#pragma unroll
-    for (int nt = 0; nt < 8; ++nt) {
-      float p[4];
-#pragma unroll
-      for (int e = 0; e < 4; ++e) {
-        const int key = kbase + nt * 8 + t4 * 2 + (e & 1);
-        p[e] = key < len ? exp2f(s[nt][e] * sl2 - m_i[e >> 1]) : 0.f;
-        rs[e >> 1] += p[e];
-      }
-      const int ks = nt >> 1, hi = nt & 1;
-      pf[ks][hi * 2 + 0] = pack_bf16x2(p[0], p[1]);
-      pf[ks][hi * 2 + 1] = pack_bf16x2(p[2], p[3]);
-    }
-#pragma unroll
-    for (int r = 0; r < 2; ++r) {
-      rs[r] += __shfl_xor_sync(0xffffffffu, rs[r], 1);
-      rs[r] += __shfl_xor_sync(0xffffffffu, rs[r], 2);
-      l_i[r] = l_i[r] * scale_o[r] + rs[r];
-    }
-#pragma unroll
-    for (int dt = 0; dt < 8; ++dt) {
-      acc_o[dt][0] *= scale_o[0]; acc_o[dt][1] *= scale_o[0];
-      acc_o[dt][2] *= scale_o[1]; acc_o[dt][3] *= scale_o[1];
-    }
-    // O += P V
-#pragma unroll
-    for (int ks = 0; ks < 4; ++ks) {
-#pragma unroll
-      for (int dp = 0; dp < 4; ++dp) {
-        const int i = lane >> 3;
-        const int r = ks * 16 + (i & 1) * 8 + (lane & 7);
-        uint32_t b0, b1, b2, b3;
-        ldsm_x4_t(aV[cur] + swz(r, dp * 2 + (i >> 1)), b0, b1, b2, b3);
-        // A fragment order for m16n8k16: a0 (g, k 0-7), a1 (g+8, k 0-7), a2 (g, k 8-15), a3 (g+8, k 8-15)
-        const uint32_t a[4] = {pf[ks][0], pf[ks][1], pf[ks][2], pf[ks][3]};
-        mma16816(acc_o[2 * dp], a, b0, b1);
-        mma16816(acc_o[2 * dp + 1], a, b2, b3);
-      }
-    }
-    __syncthreads();  // buffer `cur` is refilled by the next iteration's prefetch
+    ptx::fence_mbar_init();
   }
-  // normalise and store
-  const float inv0 = 1.f / l_i[0], inv1 = 1.f / l_i[1];
-  const int r0 = q0 + warp * 16 + g, r1 = r0 + 8;
+  if (warp == 5) ptx::tmem_alloc(tmem_slot, kTmemCols);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 4) {
+    // ------------------------------------------------------------ TMA producer
+    if (lane == 0) {
+      ptx::mbar_arrive_expect_tx(&bar_k[0], 2 * kTileBytes);
+      ptx::tma_load_2d(sQ, &tm, &bar_k[0], h * D, row_base + q0);
+      ptx::tma_load_2d(sK, &tm, &bar_k[0], H + h * D, row_base);
+      for (int j = 1; j < n_kt; ++j) {
+        ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
+        ptx::tma_load_2d(sK + j * kTileBytes, &tm, &bar_k[j], H + h * D, row_base + j * AK);
+      }
+      for (int j = 0; j < n_kt; ++j) {
+        ptx::mbar_arrive_expect_tx(&bar_v[j], kTileBytes);
+        ptx::tma_load_2d(sV + j * kTileBytes, &tm, &bar_v[j], 2 * H + h * D, row_base + j * AK);
+      }
+    }
+  } else if (warp == 5) {
+    // ------------------------------------------------------------- MMA issuer
+    if (lane == 0) {
+      constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, AK);
+      constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
+      const uint32_t q_addr = ptx::smem_u32(sQ);
+      auto issue_s = [&](int j) {
+        ptx::mbar_wait(&bar_k[j], 0);
+        ptx::tc_fence_after();
+        const uint32_t k_addr = ptx::smem_u32(sK + j * kTileBytes);
 #pragma unroll
-  for (int dt = 0; dt < 8; ++dt) {
-    const int col = h * D + dt * 8 + t4 * 2;
-    if (r0 < L)
-      *reinterpret_cast<uint32_t*>(o + (row_base + r0) * H + col) = pack_bf16x2(acc_o[dt][0] * inv0, acc_o[dt][1] * inv0);
-    if (r1 < L)
-      *reinterpret_cast<uint32_t*>(o + (row_base + r1) * H + col) = pack_bf16x2(acc_o[dt][2] * inv1, acc_o[dt][3] * inv1);
+        for (int k = 0; k < D / 16; ++k)
+          ptx::mma_bf16_ss(tmem + (j & 1) * AK, ptx::desc_k_sw128(q_addr + k * 32),
+                           ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
+        ptx::mma_commit(&s_full[j & 1]);
+      };
+      issue_s(0);
+      if (n_kt > 1) issue_s(1);
+      for (int j = 0; j < n_kt; ++j) {
+        ptx::mbar_wait(&p_full[j & 1], (j >> 1) & 1);
+        ptx::mbar_wait(&bar_v[j], 0);
+        ptx::tc_fence_after();
+        const uint32_t p_addr = ptx::smem_u32(sP + (j & 1) * kPBytes);
+        const uint32_t v_addr = ptx::smem_u32(sV + j * kTileBytes);
+#pragma unroll
+        for (int ks = 0; ks < AK / 16; ++ks)
+          ptx::mma_bf16_ss(tmem + kOCol, ptx::desc_k_sw128(p_addr + (ks >> 2) * kTileBytes + (ks & 3) * 32),
+                           ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (j | ks) != 0);
+        ptx::mma_commit(&pv_done[j & 1]);
+        if (j + 2 < n_kt) issue_s(j + 2);
+      }
+    }
+  } else {
+    // ----------------------------------------------------------------- softmax
+    const int r = warp * 32 + lane;  // query row within the tile == TMEM lane
+    const uint32_t t_lane = tmem + ((uint32_t)(warp * 32) << 16);
+    const float c = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
+    float m = -INFINITY, l = 0.f;
+    for (int j = 0; j < n_kt; ++j) {
+      ptx::mbar_wait(&s_full[j & 1], (j >> 1) & 1);
+      ptx::tc_fence_after();
+      const uint32_t t_s = t_lane + (j & 1) * AK;
+      const bool full_tile = (j + 1) * AK <= len;
+      float tmax = -INFINITY;
+#pragma unroll
+      for (int ch = 0; ch < AK / 32; ++ch) {
+        uint32_t v[32];
+        ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
+        ptx::tmem_wait_ld();
+#pragma unroll
+        for (int e = 0; e < 32; ++e) {
+          const float sv = __uint_as_float(v[e]);
+          if (full_tile || valid_key(j * AK + ch * 32 + e, len)) tmax = fmaxf(tmax, sv);
+        }
+      }
+      if (j == 0) {
+        m = tmax;
+      } else if ((tmax - m) * c > kRescaleLog2) {
+        const float alpha = ex2_approx((m - tmax) * c);
+        l *= alpha;
+        m = tmax;
+        // O holds PV_0..PV_{j-1}: wait for PV_{j-1}, rescale it in TMEM
+        ptx::mbar_wait(&pv_done[(j - 1) & 1], ((j - 1) >> 1) & 1);
+        ptx::tc_fence_after();
+#pragma unroll
+        for (int half = 0; half < 2; ++half) {
+          uint32_t v[32];
+          ptx::tmem_ld_32x32b_x32(t_lane + kOCol + half * 32, v);
+          ptx::tmem_wait_ld();
+#pragma unroll
+          for (int e = 0; e < 32; ++e) v[e] = __float_as_uint(__uint_as_float(v[e]) * alpha);
+          ptx::tmem_st_32x32b_x32(t_lane + kOCol + half * 32, v);
+        }
+        ptx::tmem_wait_st();
+      }
+      // P buffer (j & 1) was read by PV_{j-2}
+      if (j >= 2) ptx::mbar_wait(&pv_done[j & 1], ((j - 2) >> 1) & 1);
+      const float mc = m * c;
+      uint8_t* pbuf = sP + (j & 1) * kPBytes;
+#pragma unroll
+      for (int ch = 0; ch < AK / 32; ++ch) {
+        uint32_t v[32];
+        ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
+        ptx::tmem_wait_ld();
+        uint32_t pk[16];
+#pragma unroll
+        for (int e = 0; e < 32; e += 2) {
+          float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c, -mc));
+          float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c, -mc));
+          if (!full_tile) {
+            if (!valid_key(j * AK + ch * 32 + e, len)) p0 = 0.f;
+            if (!valid_key(j * AK + ch * 32 + e + 1, len)) p1 = 0.f;
+          }
+          l += p0 + p1;
+          pk[e >> 1] = pack_bf16x2(p0, p1);
+        }
+        // keys ch*32 .. ch*32+31 -> K-block ch/2, 16-byte chunks (ch%2)*4 .. +3 of row r
+        uint8_t* rowp = pbuf + (ch >> 1) * kTileBytes + r * 128;
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          const int chunk = (ch & 1) * 4 + i;
+          *reinterpret_cast<uint4*>(rowp + ((chunk ^ (r & 7)) << 4)) =
+              make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+        }
+      }
+      ptx::fence_proxy_async_smem();
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) ptx::mbar_arrive(&p_full[j & 1]);
+    }
+    // O = (sum_j P_j V_j) / l
+    ptx::mbar_wait(&pv_done[(n_kt - 1) & 1], ((n_kt - 1) >> 1) & 1);
+    ptx::tc_fence_after();
+    const float inv = 1.f / l;
+    const int row = q0 + r;
+    uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + row) * H + h * D);
+#pragma unroll
+    for (int half = 0; half < 2; ++half) {
+      uint32_t v[32];
+      ptx::tmem_ld_32x32b_x32(t_lane + kOCol + half * 32, v);
+      ptx::tmem_wait_ld();
+      if (row < L) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) {
+          uint4 u;
+          u.x = pack_bf16x2(__uint_as_float(v[8 * i + 0]) * inv, __uint_as_float(v[8 * i + 1]) * inv);
+          u.y = pack_bf16x2(__uint_as_float(v[8 * i + 2]) * inv, __uint_as_float(v[8 * i + 3]) * inv);
+          u.z = pack_bf16x2(__uint_as_float(v[8 * i + 4]) * inv, __uint_as_float(v[8 * i + 5]) * inv);
+          u.w = pack_bf16x2(__uint_as_float(v[8 * i + 6]) * inv, __uint_as_float(v[8 * i + 7]) * inv);
+          orow[half * 4 + i] = u;
+        }
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, kTmemCols);
   }
 }
 
@@ -231,7 +266,7 @@ __global__ void __launch_bounds__(128) attn_f32_kernel(int B, int L, int heads, 
   const int b = row / L, t = row - b * L;
   const int len = __ldg(lengths + b);
   float* orow = o + (size_t)row * H + h * D;
-  if ((t / QT) * QT >= len) {  // same zero rule as the bf16 path
+  if ((t / AQ) * AQ >= len) {  // same zero rule as the bf16 path
     orow[2 * lane] = 0.f;
     orow[2 * lane + 1] = 0.f;
     return;
@@ -256,15 +291,27 @@ __global__ void __launch_bounds__(128) attn_f32_kernel(int B, int L, int heads, 
 
 }  // namespace
 
-cudaError_t launch_attention(DType dt, int B, int L, int heads, const void* qkv, const int32_t* lengths,
-                             void* o, cudaStream_t s) {
-  if (B <= 0 || L <= 0) return cudaSuccess;
-  if (dt == DT_BF16) {
-    dim3 grid((L + QT - 1) / QT, heads, B);
-    attn_bf16_kernel<<<grid, 128, 0, s>>>(L, heads, (const bf16*)qkv, lengths, (bf16*)o);
+bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) {
+  p->B = B; p->L = L; p->heads = heads; p->dt = dt; p->qkv = qkv;
+  if (dt != DT_BF16) return true;
+  if (L > AK * kMaxKT) return false;
+  return encode_tmap_bf16_2d(&p->tm, qkv, (uint64_t)3 * heads * D, (uint64_t)B * L, 64, 128, 128);
+}
+
+cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
+  if (p.B <= 0 || p.L <= 0) return cudaSuccess;
+  if (p.dt == DT_BF16) {
+    static bool attr = false;
+    if (!attr) {
+      cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kAttnSmem);
+      if (e != cudaSuccess) return e;
+      attr = true;
+    }
+    dim3 grid((p.L + AQ - 1) / AQ, p.heads, p.B);
+    attn_tc_kernel<<<grid, kAttnThreads, kAttnSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
   } else {
-    const long warps = (long)B * L * heads;
-    attn_f32_kernel<<<(unsigned)((warps + 3) / 4), 128, 0, s>>>(B, L, heads, (const float*)qkv, lengths,
+    const long warps = (long)p.B * p.L * p.heads;
+    attn_f32_kernel<<<(unsigned)((warps + 3) / 4), 128, 0, s>>>(p.B, p.L, p.heads, (const float*)p.qkv, lengths,
                                                                  (float*)o);
   }
   return cudaGetLastError();

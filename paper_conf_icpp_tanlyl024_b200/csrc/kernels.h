@@ -47,8 +47,16 @@ cudaError_t launch_gemm_simt(DType dt, int M, int N, int K, const void* A, const
                              cudaStream_t s);
 
 // ---- a3: masked attention -----------------------------------------------------------------
-cudaError_t launch_attention(DType dt, int B, int L, int heads, const void* qkv,
-                             const int32_t* lengths, void* o, cudaStream_t s);
+// bf16: tcgen05 flash attention, QKV read through a TMA map encoded once per
+// (buffer, B, L) at plan time; fp32 check mode: FFMA kernel.  L <= 512 (bf16).
+struct AttnPlan {
+  CUtensorMap tm;  // QKV [B*L, 3H] bf16, box {64, 128}, 128B swizzle
+  int B, L, heads;
+  DType dt;
+  const void* qkv;
+};
+bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv);
+cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s);
 
 // ---- a9: CLS pooler + classifier ----------------------------------------------------------
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p,

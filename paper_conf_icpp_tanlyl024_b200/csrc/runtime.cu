@@ -153,6 +153,7 @@ struct LayerPlans {
 struct Bucket {
   int b = 0;
   std::vector<LayerPlans> plans;  // bf16 only
+  AttnPlan attn;
   cudaGraphExec_t exec = nullptr;
   size_t nodes = 0;
 };
@@ -199,7 +200,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  rt->QKV, EPI_BIAS, s),
                 "qkv gemm launch");
     }
-    ARLO_CUDA(launch_attention(dt, b, L, c.heads, rt->QKV, rt->lengths, rt->O, s), "attention launch");
+    ARLO_CUDA(attn_launch(bk.attn, rt->lengths, rt->O, s), "attention launch");
     if (dt == DT_BF16) {
       ARLO_CUDA(tc_launch_gemm(bk.plans[l].o, s), "out-proj gemm launch");
     } else {
@@ -318,6 +319,8 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
   for (size_t i = 0; i < bs.size(); ++i) {
     Bucket& bk = rt->buckets[i];
     bk.b = bs[i];
+    if (!attn_plan(&bk.attn, rt->dt, bk.b, L, c.heads, rt->QKV))
+      return fail(set_error(ARLO_EINVAL, "attention plan failed (bf16 attention needs L <= 512)"));
     if (rt->dt == DT_BF16) {
       int rc = plan_bucket(rt, bk);
       if (rc) return fail(rc);
@@ -492,7 +495,10 @@ extern "C" int arlo_op_attention(int32_t dtype, int32_t B, int32_t L, int32_t he
                                  const int32_t* lengths, void* o, void* stream) {
   clear_error();
   if (B < 0 || L < 1 || heads < 1 || !qkv || !lengths || !o) return set_error(ARLO_EINVAL, "arlo_op_attention: bad arguments");
-  ARLO_CUDA(launch_attention(to_dt(dtype), B, L, heads, qkv, lengths, o, (cudaStream_t)stream), "attention");
+  AttnPlan p;
+  if (!attn_plan(&p, to_dt(dtype), B, L, heads, qkv))
+    return set_error(ARLO_EINVAL, "arlo_op_attention: plan failed (bf16 needs L <= 512)");
+  ARLO_CUDA(attn_launch(p, lengths, o, (cudaStream_t)stream), "attention");
   return ARLO_OK;
 }
 

@@ -177,11 +177,11 @@ def test_attention_masked(arlo_lib, L, heads, lengths, dtype):
             ref = orc.attention(q[:n], k[:n], v[:n], heads)
             np.testing.assert_allclose(got[i, :n], ref, rtol=0, atol=tol)
             # rows of a partially padded query tile attend the real keys
-            end = min(L, ((n + 63) // 64) * 64)
+            end = min(L, ((n + 127) // 128) * 128)
             if end > n:
                 refm = orc.attention_masked(q[:end], k[:end], v[:end], heads, n)
                 np.testing.assert_allclose(got[i, n:end], refm[n:end], rtol=0, atol=tol)
-        start = ((n + 63) // 64) * 64
+        start = ((n + 127) // 128) * 128
         assert np.all(got[i, start:] == 0)
 
 
@@ -198,3 +198,27 @@ def test_head(arlo_lib, dtype):
     torch.cuda.synchronize()
     ref = np.stack([orc.head(w, x[i * L].astype(np.float64)) for i in range(B)])
     np.testing.assert_allclose(logits.cpu().numpy(), ref, rtol=0, atol=1e-5)
+
+
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_attention_lazy_rescale_path(arlo_lib, dtype):
+    """Later key tiles with much larger scores force the running-max rescale of O
+    (bf16 kernel: tile max exceeding the stale max by > 2^8 in p)."""
+    B, L, heads = 2, 512, 4
+    H = 64 * heads
+    qkv = rnd((B * L, 3 * H), 77, 1.0)
+    x = qkv.reshape(B, L, 3 * H)
+    x[:, 300:330, H:2 * H] *= 8.0   # keys in tile 2 dominate
+    x[:, 400:410, H:2 * H] *= 12.0  # and tile 3 even more
+    qkv = wl.round_to_bf16(x.reshape(B * L, 3 * H))
+    lens = np.array([512, 420], np.int32)
+    dev = bf16_dev if dtype == 0 else f32_dev
+    out = torch.empty((B * L, H), device="cuda", dtype=torch.bfloat16 if dtype == 0 else torch.float32)
+    arlo_lib.op_attention(dtype, B, L, heads, dev(qkv), torch.from_numpy(lens).cuda(), out)
+    torch.cuda.synchronize()
+    got = host64(out).reshape(B, L, H)
+    tol = 2e-2 if dtype == 0 else 2e-5
+    for i, n in enumerate(lens):
+        xx = qkv[i * L:(i + 1) * L].astype(np.float64)
+        ref = orc.attention(xx[:n, :H], xx[:n, H:2 * H], xx[:n, 2 * H:], heads)
+        np.testing.assert_allclose(got[i, :n], ref, rtol=0, atol=tol)
