@@ -169,10 +169,15 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       }
       if (j == 0) {
         m = tmax;
-      } else if ((tmax - m) * c > kRescaleLog2) {
-        const float alpha = ex2_approx((m - tmax) * c);
-        l *= alpha;
-        m = tmax;
+      } else if (__any_sync(0xffffffffu, (tmax - m) * c > kRescaleLog2)) {
+        // warp-uniform branch (tcgen05.ld/st are warp-collective): rows whose max
+        // rose by > 2^8 rescale, the others multiply by 1
+        float alpha = 1.f;
+        if ((tmax - m) * c > kRescaleLog2) {
+          alpha = ex2_approx((m - tmax) * c);
+          l *= alpha;
+          m = tmax;
+        }
         // O holds PV_0..PV_{j-1}: wait for PV_{j-1}, rescale it in TMEM
         ptx::mbar_wait(&pv_done[(j - 1) & 1], ((j - 1) >> 1) & 1);
         ptx::tc_fence_after();
