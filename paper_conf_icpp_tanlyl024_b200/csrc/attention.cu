@@ -23,40 +23,47 @@ namespace arlo {
 namespace {
 
 constexpr int D = 64;        // head dim (all configs)
-constexpr int AQ = 128;      // queries per CTA (TMEM lanes)
+constexpr int AQ = 128;      // queries per q-tile (TMEM lanes)
+constexpr int NQ = 2;        // q-tiles per CTA: their softmax and MMAs interleave
 constexpr int AK = 128;      // keys per tile
 constexpr int kMaxKT = 4;    // L <= 512
-constexpr int kAttnThreads = 192;  // warps 0-3 softmax (one TMEM lane quarter each), 4 TMA, 5 MMA
-constexpr int kTileBytes = 128 * 128;   // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
-constexpr int kPBytes = 2 * kTileBytes;  // P tile: 128 queries x 128 keys = two 64-key K-blocks
-constexpr int kAttnSmem = 1024 + kTileBytes * (1 + 2 * kMaxKT) + 2 * kPBytes + 256;
-constexpr uint32_t kTmemCols = 512;      // S double buffer (2 x 128) + O (64)
-constexpr uint32_t kOCol = 256;
+constexpr int kSoftWarps = 4 * NQ;            // warps 0..7: q-tile w/4, TMEM lane quarter w%4
+constexpr int kProdWarp = kSoftWarps;         // warp 8: TMA
+constexpr int kMmaWarp = kSoftWarps + 1;      // warp 9: MMA
+constexpr int kAttnThreads = 32 * (kSoftWarps + 2);
+constexpr int kTileBytes = 128 * 128;         // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
+constexpr int kPBytes = 2 * kTileBytes;       // P: 128 queries x 128 keys = two 64-key K-blocks
+constexpr int kAttnSmem = 1024 + kTileBytes * (NQ + 2 * kMaxKT) + NQ * kPBytes + 256;
+constexpr uint32_t kTmemCols = 512;           // S (NQ x 128) + O (NQ x 64)
+constexpr uint32_t kOCol = NQ * AK;
 // lazy rescale: keep a stale row max unless a tile's max exceeds it by > 2^8 in p
 constexpr float kRescaleLog2 = 8.0f;
+static_assert(kAttnSmem <= 232448, "attention smem");
 
 __device__ __forceinline__ bool valid_key(int key, int len) { return key < len; }
 
-// One CTA = (128-query tile, head, sequence).  S_j = Q K_j^T (M=128, N=128,
-// K=64) and O += P_j V_j (M=128, N=64, K=128, V as MN-major B) on tcgen05 with
-// S double-buffered in TMEM; 4 softmax warps (thread = query row) read S_j from
-// TMEM, keep a lazily-rescaled running max (O rescaled in TMEM only when a
-// tile raises the max by > 2^8), write P_j as bf16 into 128B-swizzled smem
-// (the A operand of the PV MMA) and accumulate the row sum in fp32.  Q, every
-// K_j and V_j (<= 4 tiles each, L <= 512) are loaded once by TMA.  Key tiles
-// starting at >= len are never loaded or multiplied; keys >= len inside the
-// last tile get p = 0 exactly.
+// One CTA = (two 128-query tiles, head, sequence), 128-key tiles.  Per q-tile
+// qi: S_qi,j = Q_qi K_j^T (M=128, N=128, K=64) and O_qi += P_qi,j V_j (M=128,
+// N=64, K=128; V is an MN-major B operand) on tcgen05 with S_qi and O_qi in
+// TMEM.  Four softmax warps per q-tile (thread = query row) read S from TMEM,
+// keep a lazily-rescaled running max (O rescaled in TMEM only when a tile
+// raises a row max by > 2^8 in p), write P as bf16 into 128B-swizzled smem
+// (the A operand of the PV MMA) and accumulate the fp32 row sum.  The two
+// q-tiles' softmax and MMAs interleave (one's softmax runs while the other's
+// S/PV MMAs execute); Q, every K_j and V_j (<= 4 tiles, L <= 512) are loaded
+// once by TMA and shared by both q-tiles.  Key tiles starting at >= len are
+// never loaded or multiplied; keys >= len inside the last tile get p = 0.
 __global__ void __launch_bounds__(kAttnThreads, 1)
 attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const int32_t* __restrict__ lengths,
                bf16* __restrict__ o) {
-  const int qt = blockIdx.x, h = blockIdx.y, b = blockIdx.z;
+  const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
   const int len = __ldg(lengths + b);
-  const int q0 = qt * AQ;
+  const int q0 = blockIdx.x * (NQ * AQ);
   const int row_base = b * L;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  if (q0 >= len) {  // wholly padded query tile (or empty slot): zeros
-    const int rows = min(AQ, L - q0);
+  if (q0 >= len) {  // every q-tile wholly padded (or empty slot): zeros
+    const int rows = min(NQ * AQ, L - q0);
     for (int i = threadIdx.x; i < rows * 8; i += kAttnThreads) {
       const int r = i >> 3, c = i & 7;
       *reinterpret_cast<uint4*>(o + (size_t)(row_base + q0 + r) * H + h * D + c * 8) = make_uint4(0, 0, 0, 0);
@@ -64,44 +71,45 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     return;
   }
   const int n_kt = (len + AK - 1) / AK;
+  const int nq = (q0 + AQ < len) ? 2 : 1;  // live q-tiles (the second may be wholly padded)
 
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
-  uint8_t* sK = sQ + kTileBytes;
+  uint8_t* sK = sQ + NQ * kTileBytes;
   uint8_t* sV = sK + kMaxKT * kTileBytes;
   uint8_t* sP = sV + kMaxKT * kTileBytes;
-  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + 2 * kPBytes);
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * kPBytes);
   uint64_t* bar_v = bar_k + kMaxKT;
   uint64_t* s_full = bar_v + kMaxKT;
-  uint64_t* p_full = s_full + 2;
-  uint64_t* pv_done = p_full + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2);
+  uint64_t* p_full = s_full + NQ;
+  uint64_t* pv_done = p_full + NQ;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + NQ);
 
-  if (warp == 4 && lane == 0) {
+  if (warp == kProdWarp && lane == 0) {
     ptx::tma_prefetch_desc(&tm);
     for (int j = 0; j < kMaxKT; ++j) {
       ptx::mbar_init(&bar_k[j], 1);
       ptx::mbar_init(&bar_v[j], 1);
     }
-    for (int i = 0; i < 2; ++i) {
+    for (int i = 0; i < NQ; ++i) {
       ptx::mbar_init(&s_full[i], 1);
       ptx::mbar_init(&p_full[i], 4);
       ptx::mbar_init(&pv_done[i], 1);
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 5) ptx::tmem_alloc(tmem_slot, kTmemCols);
+  if (warp == kMmaWarp) ptx::tmem_alloc(tmem_slot, kTmemCols);
   ptx::tc_fence_before();
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
 
-  if (warp == 4) {
+  if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
-      ptx::mbar_arrive_expect_tx(&bar_k[0], 2 * kTileBytes);
-      ptx::tma_load_2d(sQ, &tm, &bar_k[0], h * D, row_base + q0);
+      ptx::mbar_arrive_expect_tx(&bar_k[0], (nq + 1) * kTileBytes);
+      for (int qi = 0; qi < nq; ++qi) ptx::tma_load_2d(sQ + qi * kTileBytes, &tm, &bar_k[0], h * D, row_base + q0 + qi * AQ);
       ptx::tma_load_2d(sK, &tm, &bar_k[0], H + h * D, row_base);
       for (int j = 1; j < n_kt; ++j) {
         ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
@@ -112,148 +120,158 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         ptx::tma_load_2d(sV + j * kTileBytes, &tm, &bar_v[j], 2 * H + h * D, row_base + j * AK);
       }
     }
-  } else if (warp == 5) {
+  } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------- MMA issuer
     if (lane == 0) {
       constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, AK);
       constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
-      const uint32_t q_addr = ptx::smem_u32(sQ);
-      auto issue_s = [&](int j) {
+      auto issue_s = [&](int qi, int j) {
         ptx::mbar_wait(&bar_k[j], 0);
         ptx::tc_fence_after();
+        const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
         const uint32_t k_addr = ptx::smem_u32(sK + j * kTileBytes);
 #pragma unroll
         for (int k = 0; k < D / 16; ++k)
-          ptx::mma_bf16_ss(tmem + (j & 1) * AK, ptx::desc_k_sw128(q_addr + k * 32),
-                           ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
-        ptx::mma_commit(&s_full[j & 1]);
+          ptx::mma_bf16_ss(tmem + qi * AK, ptx::desc_k_sw128(q_addr + k * 32), ptx::desc_k_sw128(k_addr + k * 32),
+                           idesc_s, k > 0);
+        ptx::mma_commit(&s_full[qi]);
       };
-      issue_s(0);
-      if (n_kt > 1) issue_s(1);
+      for (int qi = 0; qi < nq; ++qi) issue_s(qi, 0);
       for (int j = 0; j < n_kt; ++j) {
-        ptx::mbar_wait(&p_full[j & 1], (j >> 1) & 1);
-        ptx::mbar_wait(&bar_v[j], 0);
-        ptx::tc_fence_after();
-        const uint32_t p_addr = ptx::smem_u32(sP + (j & 1) * kPBytes);
-        const uint32_t v_addr = ptx::smem_u32(sV + j * kTileBytes);
+        for (int qi = 0; qi < nq; ++qi) {
+          ptx::mbar_wait(&p_full[qi], j & 1);  // P_qi,j written, S_qi buffer consumed
+          ptx::mbar_wait(&bar_v[j], 0);
+          ptx::tc_fence_after();
+          const uint32_t p_addr = ptx::smem_u32(sP + qi * kPBytes);
+          const uint32_t v_addr = ptx::smem_u32(sV + j * kTileBytes);
 #pragma unroll
-        for (int ks = 0; ks < AK / 16; ++ks)
-          ptx::mma_bf16_ss(tmem + kOCol, ptx::desc_k_sw128(p_addr + (ks >> 2) * kTileBytes + (ks & 3) * 32),
-                           ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (j | ks) != 0);
-        ptx::mma_commit(&pv_done[j & 1]);
-        if (j + 2 < n_kt) issue_s(j + 2);
+          for (int ks = 0; ks < AK / 16; ++ks)
+            ptx::mma_bf16_ss(tmem + kOCol + qi * D,
+                             ptx::desc_k_sw128(p_addr + (ks >> 2) * kTileBytes + (ks & 3) * 32),
+                             ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (j | ks) != 0);
+          ptx::mma_commit(&pv_done[qi]);
+          if (j + 1 < n_kt) issue_s(qi, j + 1);
+        }
       }
     }
   } else {
     // ----------------------------------------------------------------- softmax
-    const int r = warp * 32 + lane;  // query row within the tile == TMEM lane
-    const uint32_t t_lane = tmem + ((uint32_t)(warp * 32) << 16);
-    const float c = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
-    float m = -INFINITY, l = 0.f;
-    for (int j = 0; j < n_kt; ++j) {
-      ptx::mbar_wait(&s_full[j & 1], (j >> 1) & 1);
-      ptx::tc_fence_after();
-      const uint32_t t_s = t_lane + (j & 1) * AK;
-      const bool full_tile = (j + 1) * AK <= len;
-      float tmax = -INFINITY;
-#pragma unroll
-      for (int ch = 0; ch < AK / 32; ++ch) {
-        uint32_t v[32];
-        ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
-        ptx::tmem_wait_ld();
-#pragma unroll
-        for (int e = 0; e < 32; ++e) {
-          const float sv = __uint_as_float(v[e]);
-          if (full_tile || valid_key(j * AK + ch * 32 + e, len)) tmax = fmaxf(tmax, sv);
-        }
-      }
-      if (j == 0) {
-        m = tmax;
-      } else if (__any_sync(0xffffffffu, (tmax - m) * c > kRescaleLog2)) {
-        // warp-uniform branch (tcgen05.ld/st are warp-collective): rows whose max
-        // rose by > 2^8 rescale, the others multiply by 1
-        float alpha = 1.f;
-        if ((tmax - m) * c > kRescaleLog2) {
-          alpha = ex2_approx((m - tmax) * c);
-          l *= alpha;
-          m = tmax;
-        }
-        // O holds PV_0..PV_{j-1}: wait for PV_{j-1}, rescale it in TMEM
-        ptx::mbar_wait(&pv_done[(j - 1) & 1], ((j - 1) >> 1) & 1);
+    const int qi = warp >> 2, quarter = warp & 3;
+    const int r = quarter * 32 + lane;  // query row within q-tile qi == TMEM lane
+    const int qrow = q0 + qi * AQ + r;
+    if (qi < nq) {
+      const uint32_t t_lane = tmem + ((uint32_t)(quarter * 32) << 16);
+      const uint32_t t_s = t_lane + qi * AK;
+      const uint32_t t_o = t_lane + kOCol + qi * D;
+      const float c = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
+      float m = -INFINITY, l = 0.f;
+      uint8_t* pbuf = sP + qi * kPBytes;
+      for (int j = 0; j < n_kt; ++j) {
+        ptx::mbar_wait(&s_full[qi], j & 1);
         ptx::tc_fence_after();
+        const bool full_tile = (j + 1) * AK <= len;
+        float tmax = -INFINITY;
 #pragma unroll
-        for (int half = 0; half < 2; ++half) {
+        for (int ch = 0; ch < AK / 32; ++ch) {
           uint32_t v[32];
-          ptx::tmem_ld_32x32b_x32(t_lane + kOCol + half * 32, v);
+          ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
           ptx::tmem_wait_ld();
 #pragma unroll
-          for (int e = 0; e < 32; ++e) v[e] = __float_as_uint(__uint_as_float(v[e]) * alpha);
-          ptx::tmem_st_32x32b_x32(t_lane + kOCol + half * 32, v);
-        }
-        ptx::tmem_wait_st();
-      }
-      // P buffer (j & 1) was read by PV_{j-2}
-      if (j >= 2) ptx::mbar_wait(&pv_done[j & 1], ((j - 2) >> 1) & 1);
-      const float mc = m * c;
-      uint8_t* pbuf = sP + (j & 1) * kPBytes;
-#pragma unroll
-      for (int ch = 0; ch < AK / 32; ++ch) {
-        uint32_t v[32];
-        ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
-        ptx::tmem_wait_ld();
-        uint32_t pk[16];
-#pragma unroll
-        for (int e = 0; e < 32; e += 2) {
-          float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c, -mc));
-          float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c, -mc));
-          if (!full_tile) {
-            if (!valid_key(j * AK + ch * 32 + e, len)) p0 = 0.f;
-            if (!valid_key(j * AK + ch * 32 + e + 1, len)) p1 = 0.f;
+          for (int e = 0; e < 32; ++e) {
+            if (full_tile || valid_key(j * AK + ch * 32 + e, len)) tmax = fmaxf(tmax, __uint_as_float(v[e]));
           }
-          l += p0 + p1;
-          pk[e >> 1] = pack_bf16x2(p0, p1);
         }
-        // keys ch*32 .. ch*32+31 -> K-block ch/2, 16-byte chunks (ch%2)*4 .. +3 of row r
-        uint8_t* rowp = pbuf + (ch >> 1) * kTileBytes + r * 128;
+        // P buffer (and O) are read / accumulated by PV_{j-1}: wait for it
+        if (j > 0) {
+          ptx::mbar_wait(&pv_done[qi], (j - 1) & 1);
+          ptx::tc_fence_after();
+        }
+        if (j == 0) {
+          m = tmax;
+        } else if (__any_sync(0xffffffffu, (tmax - m) * c > kRescaleLog2)) {
+          // warp-uniform branch (tcgen05.ld/st are warp-collective): rows whose
+          // max rose by > 2^8 rescale O and l, the others multiply by 1
+          float alpha = 1.f;
+          if ((tmax - m) * c > kRescaleLog2) {
+            alpha = ex2_approx((m - tmax) * c);
+            l *= alpha;
+            m = tmax;
+          }
 #pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          const int chunk = (ch & 1) * 4 + i;
-          *reinterpret_cast<uint4*>(rowp + ((chunk ^ (r & 7)) << 4)) =
-              make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+          for (int half = 0; half < 2; ++half) {
+            uint32_t v[32];
+            ptx::tmem_ld_32x32b_x32(t_o + half * 32, v);
+            ptx::tmem_wait_ld();
+#pragma unroll
+            for (int e = 0; e < 32; ++e) v[e] = __float_as_uint(__uint_as_float(v[e]) * alpha);
+            ptx::tmem_st_32x32b_x32(t_o + half * 32, v);
+          }
+          ptx::tmem_wait_st();
+        }
+        const float mc = m * c;
+#pragma unroll
+        for (int ch = 0; ch < AK / 32; ++ch) {
+          uint32_t v[32];
+          ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
+          ptx::tmem_wait_ld();
+          uint32_t pk[16];
+#pragma unroll
+          for (int e = 0; e < 32; e += 2) {
+            float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c, -mc));
+            float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c, -mc));
+            if (!full_tile) {
+              if (!valid_key(j * AK + ch * 32 + e, len)) p0 = 0.f;
+              if (!valid_key(j * AK + ch * 32 + e + 1, len)) p1 = 0.f;
+            }
+            l += p0 + p1;
+            pk[e >> 1] = pack_bf16x2(p0, p1);
+          }
+          // keys ch*32 .. +31 -> K-block ch/2, 16-byte chunks (ch%2)*4 .. +3 of row r
+          uint8_t* rowp = pbuf + (ch >> 1) * kTileBytes + r * 128;
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            const int chunk = (ch & 1) * 4 + i;
+            *reinterpret_cast<uint4*>(rowp + ((chunk ^ (r & 7)) << 4)) =
+                make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+          }
+        }
+        ptx::fence_proxy_async_smem();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&p_full[qi]);
+      }
+      // O = (sum_j P_j V_j) / l
+      ptx::mbar_wait(&pv_done[qi], (n_kt - 1) & 1);
+      ptx::tc_fence_after();
+      const float inv = 1.f / l;
+      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
+#pragma unroll
+      for (int half = 0; half < 2; ++half) {
+        uint32_t v[32];
+        ptx::tmem_ld_32x32b_x32(t_o + half * 32, v);
+        ptx::tmem_wait_ld();
+        if (qrow < L) {
+#pragma unroll
+          for (int i = 0; i < 4; ++i) {
+            uint4 u;
+            u.x = pack_bf16x2(__uint_as_float(v[8 * i + 0]) * inv, __uint_as_float(v[8 * i + 1]) * inv);
+            u.y = pack_bf16x2(__uint_as_float(v[8 * i + 2]) * inv, __uint_as_float(v[8 * i + 3]) * inv);
+            u.z = pack_bf16x2(__uint_as_float(v[8 * i + 4]) * inv, __uint_as_float(v[8 * i + 5]) * inv);
+            u.w = pack_bf16x2(__uint_as_float(v[8 * i + 6]) * inv, __uint_as_float(v[8 * i + 7]) * inv);
+            orow[half * 4 + i] = u;
+          }
         }
       }
-      ptx::fence_proxy_async_smem();
-      ptx::tc_fence_before();
-      __syncwarp();
-      if (lane == 0) ptx::mbar_arrive(&p_full[j & 1]);
-    }
-    // O = (sum_j P_j V_j) / l
-    ptx::mbar_wait(&pv_done[(n_kt - 1) & 1], ((n_kt - 1) >> 1) & 1);
-    ptx::tc_fence_after();
-    const float inv = 1.f / l;
-    const int row = q0 + r;
-    uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + row) * H + h * D);
+    } else if (qrow < L) {
+      // second q-tile wholly padded: zero rows
+      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
 #pragma unroll
-    for (int half = 0; half < 2; ++half) {
-      uint32_t v[32];
-      ptx::tmem_ld_32x32b_x32(t_lane + kOCol + half * 32, v);
-      ptx::tmem_wait_ld();
-      if (row < L) {
-#pragma unroll
-        for (int i = 0; i < 4; ++i) {
-          uint4 u;
-          u.x = pack_bf16x2(__uint_as_float(v[8 * i + 0]) * inv, __uint_as_float(v[8 * i + 1]) * inv);
-          u.y = pack_bf16x2(__uint_as_float(v[8 * i + 2]) * inv, __uint_as_float(v[8 * i + 3]) * inv);
-          u.z = pack_bf16x2(__uint_as_float(v[8 * i + 4]) * inv, __uint_as_float(v[8 * i + 5]) * inv);
-          u.w = pack_bf16x2(__uint_as_float(v[8 * i + 6]) * inv, __uint_as_float(v[8 * i + 7]) * inv);
-          orow[half * 4 + i] = u;
-        }
-      }
+      for (int i = 0; i < 8; ++i) orow[i] = make_uint4(0, 0, 0, 0);
     }
   }
   ptx::tc_fence_before();
   __syncthreads();
-  if (warp == 5) {
+  if (warp == kMmaWarp) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem, kTmemCols);
   }
@@ -271,7 +289,7 @@ __global__ void __launch_bounds__(128) attn_f32_kernel(int B, int L, int heads, 
   const int b = row / L, t = row - b * L;
   const int len = __ldg(lengths + b);
   float* orow = o + (size_t)row * H + h * D;
-  if ((t / AQ) * AQ >= len) {  // same zero rule as the bf16 path
+  if ((t / AQ) * AQ >= len) {  // same zero rule as the bf16 path (128-row q-tiles)
     orow[2 * lane] = 0.f;
     orow[2 * lane + 1] = 0.f;
     return;
@@ -312,7 +330,7 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
       if (e != cudaSuccess) return e;
       attr = true;
     }
-    dim3 grid((p.L + AQ - 1) / AQ, p.heads, p.B);
+    dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
     attn_tc_kernel<<<grid, kAttnThreads, kAttnSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
