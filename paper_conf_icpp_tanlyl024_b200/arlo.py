@@ -30,7 +30,7 @@ EXPORTED = [
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
     "arlo_op_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
-    "arlo_debug_gemm_trace", "arlo_gemm_tile_choice",
+    "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
 ]
 
 
@@ -76,6 +76,7 @@ _sig("arlo_op_layernorm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _
 _sig("arlo_op_embed", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp, _vp)
 _sig("arlo_op_attention", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp)
 _sig("arlo_debug_gemm_trace", C.c_int, _vp)
+_sig("arlo_debug_attn_trace", C.c_int, _vp)
 _sig("arlo_gemm_tile_choice", _i32, _i32, _i32, _i32)
 _sig("arlo_op_head", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp)
 

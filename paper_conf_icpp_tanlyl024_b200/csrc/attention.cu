@@ -24,38 +24,70 @@ namespace {
 
 constexpr int D = 64;        // head dim (all configs)
 constexpr int AQ = 128;      // queries per q-tile (TMEM lanes)
-constexpr int NQ = 2;        // q-tiles per CTA: their softmax and MMAs interleave
-constexpr int AK = 128;      // keys per tile
-constexpr int kMaxKT = 4;    // L <= 512
-constexpr int kSoftWarps = 4 * NQ;            // warps 0..7: q-tile w/4, TMEM lane quarter w%4
-constexpr int kProdWarp = kSoftWarps;         // warp 8: TMA
-constexpr int kMmaWarp = kSoftWarps + 1;      // warp 9: MMA
-constexpr int kAttnThreads = 32 * (kSoftWarps + 2);
+constexpr int AK = 128;      // keys per K/V tile (TMA unit)
+constexpr int KC = 64;       // keys per softmax chunk (S MMA N)
 constexpr int kTileBytes = 128 * 128;         // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
-constexpr int kPBytes = 2 * kTileBytes;       // P: 128 queries x 128 keys = two 64-key K-blocks
-constexpr int kAttnSmem = 1024 + kTileBytes * (NQ + 2 * kMaxKT) + NQ * kPBytes + 256;
-constexpr uint32_t kTmemCols = 512;           // S (NQ x 128) + O (NQ x 64)
-constexpr uint32_t kOCol = NQ * AK;
-// lazy rescale: keep a stale row max unless a tile's max exceeds it by > 2^8 in p
+constexpr int kPBytes = 128 * 128;            // P chunk: 128 queries x 64 keys (one K-block)
+// lazy rescale: keep a stale row max unless a chunk's max exceeds it by > 2^8 in p
 constexpr float kRescaleLog2 = 8.0f;
-static_assert(kAttnSmem <= 232448, "attention smem");
 
-__device__ __forceinline__ bool valid_key(int key, int len) { return key < len; }
+// Launch shape per runtime length: NQ q-tiles per CTA, up to MAXKT 128-key
+// K/V tiles (L <= 128 * MAXKT).  NQ = 1 (L <= 128) keeps smem (80 KB) and TMEM
+// (256 columns) small enough for two CTAs per SM.
+template <int NQ_, int MAXKT_>
+struct AttnCfg {
+  static constexpr int NQ = NQ_;
+  static constexpr int kMaxKT = MAXKT_;
+  static constexpr int kKSlots = MAXKT_ < 2 ? MAXKT_ : 2;  // K tiles ring; V stays resident
+  static constexpr int kSoftWarps = 4 * NQ;   // warp w: q-tile w/4, TMEM lane quarter w%4
+  static constexpr int kProdWarp = kSoftWarps;
+  static constexpr int kMmaWarp = kSoftWarps + 1;
+  static constexpr int kThreads = 32 * (kSoftWarps + 2);
+  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + NQ * 2 * kPBytes + 256;
+  // TMEM columns: q-tile qi: S slots at qi*128 + {0, 64}, O at NQ*128 + qi*64
+  static constexpr uint32_t kOCol = NQ * 128;
+  static constexpr uint32_t kTmemCols = NQ == 1 ? 256 : 512;
+  static constexpr int kMinBlocks = NQ == 1 ? 2 : 1;
+  static_assert(kSmem * kMinBlocks <= 232448, "attention smem");
+};
 
-// One CTA = (two 128-query tiles, head, sequence), 128-key tiles.  Per q-tile
-// qi: S_qi,j = Q_qi K_j^T (M=128, N=128, K=64) and O_qi += P_qi,j V_j (M=128,
-// N=64, K=128; V is an MN-major B operand) on tcgen05 with S_qi and O_qi in
-// TMEM.  Four softmax warps per q-tile (thread = query row) read S from TMEM,
-// keep a lazily-rescaled running max (O rescaled in TMEM only when a tile
-// raises a row max by > 2^8 in p), write P as bf16 into 128B-swizzled smem
-// (the A operand of the PV MMA) and accumulate the fp32 row sum.  The two
-// q-tiles' softmax and MMAs interleave (one's softmax runs while the other's
-// S/PV MMAs execute); Q, every K_j and V_j (<= 4 tiles, L <= 512) are loaded
-// once by TMA and shared by both q-tiles.  Key tiles starting at >= len are
-// never loaded or multiplied; keys >= len inside the last tile get p = 0.
-__global__ void __launch_bounds__(kAttnThreads, 1)
+// Profiling hook (arlo_debug_attn_trace): the TRACE=true instantiation writes
+// %globaltimer stamps of the first 2048 CTAs into g_atrace[cta * 32 + slot].
+__device__ unsigned long long* g_atrace = nullptr;
+template <bool TRACE>
+__device__ __forceinline__ void atrace(int slot) {
+  if (TRACE) {
+    const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+    if (cta < 2048 && slot < 32) {
+      unsigned long long t;
+      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+      g_atrace[cta * 32 + slot] = t;
+    }
+  }
+}
+
+// One CTA = (two 128-query tiles, head, sequence).  Keys are processed in
+// 64-key chunks: S_qi,c = Q_qi K_c^T (M=128, N=64, K=64) into a double-buffered
+// TMEM S slot, O_qi += P_qi,c V_c (M=128, N=64, K=64; V an MN-major B operand)
+// into TMEM.  Four softmax warps per q-tile (thread = query row = TMEM lane);
+// at head dim 64 the TMEM->RF reads of S and the exp2 (MUFU) work, not the
+// tensor pipe, bound attention.  A lazily-rescaled
+// running max is kept (O rescaled in TMEM only when a chunk raises a row max
+// by > 2^8 in p); P is written as bf16 into a 128B-swizzled smem K-block (the
+// PV MMA's A operand).  S slots are double-buffered so S(c+1) is computed
+// while chunk c is in the exp stage.  Q, K (2-tile ring) and V (resident, <= 4 tiles) come
+// in by TMA once per CTA and are shared by both q-tiles.  Key chunks starting
+// at >= len are never loaded or multiplied; keys >= len inside the last chunk
+// get p = 0.
+template <int NQ_, int MAXKT_, bool TRACE>
+__global__ void __launch_bounds__(AttnCfg<NQ_, MAXKT_>::kThreads, AttnCfg<NQ_, MAXKT_>::kMinBlocks)
 attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const int32_t* __restrict__ lengths,
                bf16* __restrict__ o) {
+  using Cfg = AttnCfg<NQ_, MAXKT_>;
+  constexpr int NQ = Cfg::NQ, kMaxKT = Cfg::kMaxKT, kKSlots = Cfg::kKSlots;
+  constexpr int kSoftWarps = Cfg::kSoftWarps, kProdWarp = Cfg::kProdWarp, kMmaWarp = Cfg::kMmaWarp;
+  constexpr int kAttnThreads = Cfg::kThreads;
+  constexpr uint32_t kOCol = Cfg::kOCol, kTmemCols = Cfg::kTmemCols;
   const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
   const int len = __ldg(lengths + b);
@@ -70,21 +102,24 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     }
     return;
   }
-  const int n_kt = (len + AK - 1) / AK;
-  const int nq = (q0 + AQ < len) ? 2 : 1;  // live q-tiles (the second may be wholly padded)
+  const int n_kt = (len + AK - 1) / AK;  // K/V tiles
+  const int n_ch = (len + KC - 1) / KC;  // 64-key chunks
+  const int nq = (NQ == 2 && q0 + AQ < len) ? 2 : 1;  // live q-tiles (the second may be wholly padded)
 
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + NQ * kTileBytes;
-  uint8_t* sV = sK + kMaxKT * kTileBytes;
-  uint8_t* sP = sV + kMaxKT * kTileBytes;
-  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * kPBytes);
+  uint8_t* sV = sK + kKSlots * kTileBytes;
+  uint8_t* sP = sV + kMaxKT * kTileBytes;  // [NQ][2][128 x 64 bf16]
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * 2 * kPBytes);
   uint64_t* bar_v = bar_k + kMaxKT;
-  uint64_t* s_full = bar_v + kMaxKT;
-  uint64_t* p_full = s_full + NQ;
-  uint64_t* pv_done = p_full + NQ;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + NQ);
+  uint64_t* k_free = bar_v + kMaxKT;
+  uint64_t* s_full = k_free + kKSlots;  // [NQ][2]
+  uint64_t* s_free = s_full + 2 * NQ;
+  uint64_t* p_full = s_free + 2 * NQ;
+  uint64_t* pv_done = p_full + 2 * NQ;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2 * NQ);
 
   if (warp == kProdWarp && lane == 0) {
     ptx::tma_prefetch_desc(&tm);
@@ -92,8 +127,10 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       ptx::mbar_init(&bar_k[j], 1);
       ptx::mbar_init(&bar_v[j], 1);
     }
-    for (int i = 0; i < NQ; ++i) {
+    for (int i = 0; i < kKSlots; ++i) ptx::mbar_init(&k_free[i], 1);
+    for (int i = 0; i < 2 * NQ; ++i) {
       ptx::mbar_init(&s_full[i], 1);
+      ptx::mbar_init(&s_free[i], 4);
       ptx::mbar_init(&p_full[i], 4);
       ptx::mbar_init(&pv_done[i], 1);
     }
@@ -104,55 +141,68 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  if (threadIdx.x == 0) atrace<TRACE>(0);
 
   if (warp == kProdWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
       ptx::mbar_arrive_expect_tx(&bar_k[0], (nq + 1) * kTileBytes);
-      for (int qi = 0; qi < nq; ++qi) ptx::tma_load_2d(sQ + qi * kTileBytes, &tm, &bar_k[0], h * D, row_base + q0 + qi * AQ);
+      for (int qi = 0; qi < nq; ++qi)
+        ptx::tma_load_2d(sQ + qi * kTileBytes, &tm, &bar_k[0], h * D, row_base + q0 + qi * AQ);
       ptx::tma_load_2d(sK, &tm, &bar_k[0], H + h * D, row_base);
-      for (int j = 1; j < n_kt; ++j) {
-        ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
-        ptx::tma_load_2d(sK + j * kTileBytes, &tm, &bar_k[j], H + h * D, row_base + j * AK);
+      if (n_kt > 1) {
+        ptx::mbar_arrive_expect_tx(&bar_k[1], kTileBytes);
+        ptx::tma_load_2d(sK + kTileBytes, &tm, &bar_k[1], H + h * D, row_base + AK);
       }
       for (int j = 0; j < n_kt; ++j) {
         ptx::mbar_arrive_expect_tx(&bar_v[j], kTileBytes);
         ptx::tma_load_2d(sV + j * kTileBytes, &tm, &bar_v[j], 2 * H + h * D, row_base + j * AK);
       }
+      for (int j = kKSlots; j < n_kt; ++j) {  // K ring: slot j%2 frees when S(., tile j-2) completes
+        ptx::mbar_wait(&k_free[j & 1], ((j - kKSlots) >> 1) & 1);
+        ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
+        ptx::tma_load_2d(sK + (j & 1) * kTileBytes, &tm, &bar_k[j], H + h * D, row_base + j * AK);
+      }
     }
   } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------- MMA issuer
     if (lane == 0) {
-      constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, AK);
+      constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
       constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
-      auto issue_s = [&](int qi, int j) {
-        ptx::mbar_wait(&bar_k[j], 0);
+      auto issue_s = [&](int qi, int c) {
+        const int t = c >> 1, sl = c & 1;
+        if (c >= 2) ptx::mbar_wait(&s_free[qi * 2 + sl], ((c - 2) >> 1) & 1);
+        ptx::mbar_wait(&bar_k[t], 0);
         ptx::tc_fence_after();
         const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
-        const uint32_t k_addr = ptx::smem_u32(sK + j * kTileBytes);
+        const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
         for (int k = 0; k < D / 16; ++k)
-          ptx::mma_bf16_ss(tmem + qi * AK, ptx::desc_k_sw128(q_addr + k * 32), ptx::desc_k_sw128(k_addr + k * 32),
-                           idesc_s, k > 0);
-        ptx::mma_commit(&s_full[qi]);
+          ptx::mma_bf16_ss(tmem + qi * 128 + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
+                           ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
+        ptx::mma_commit(&s_full[qi * 2 + sl]);
       };
-      for (int qi = 0; qi < nq; ++qi) issue_s(qi, 0);
-      for (int j = 0; j < n_kt; ++j) {
-        for (int qi = 0; qi < nq; ++qi) {
-          ptx::mbar_wait(&p_full[qi], j & 1);  // P_qi,j written, S_qi buffer consumed
-          ptx::mbar_wait(&bar_v[j], 0);
-          ptx::tc_fence_after();
-          const uint32_t p_addr = ptx::smem_u32(sP + qi * kPBytes);
-          const uint32_t v_addr = ptx::smem_u32(sV + j * kTileBytes);
+      auto issue_pv = [&](int qi, int c) {
+        const int t = c >> 1, sl = c & 1;
+        ptx::mbar_wait(&p_full[qi * 2 + sl], (c >> 1) & 1);
+        ptx::mbar_wait(&bar_v[t], 0);
+        ptx::tc_fence_after();
+        const uint32_t p_addr = ptx::smem_u32(sP + (qi * 2 + sl) * kPBytes);
+        const uint32_t v_addr = ptx::smem_u32(sV + t * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
-          for (int ks = 0; ks < AK / 16; ++ks)
-            ptx::mma_bf16_ss(tmem + kOCol + qi * D,
-                             ptx::desc_k_sw128(p_addr + (ks >> 2) * kTileBytes + (ks & 3) * 32),
-                             ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (j | ks) != 0);
-          ptx::mma_commit(&pv_done[qi]);
-          if (j + 1 < n_kt) issue_s(qi, j + 1);
-        }
+        for (int ks = 0; ks < KC / 16; ++ks)
+          ptx::mma_bf16_ss(tmem + kOCol + qi * D, ptx::desc_k_sw128(p_addr + ks * 32),
+                           ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (c | ks) != 0);
+        ptx::mma_commit(&pv_done[qi * 2 + sl]);
+      };
+      for (int c = 0; c < n_ch; ++c) {
+        for (int qi = 0; qi < nq; ++qi) issue_s(qi, c);
+        if ((c & 1) || c == n_ch - 1) ptx::mma_commit(&k_free[(c >> 1) & 1]);  // K tile c/2 fully used
+        if (c == 0) atrace<TRACE>(2);
+        if (c >= 1)
+          for (int qi = 0; qi < nq; ++qi) issue_pv(qi, c - 1);
       }
+      for (int qi = 0; qi < nq; ++qi) issue_pv(qi, n_ch - 1);
     }
   } else {
     // ----------------------------------------------------------------- softmax
@@ -161,104 +211,112 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     const int qrow = q0 + qi * AQ + r;
     if (qi < nq) {
       const uint32_t t_lane = tmem + ((uint32_t)(quarter * 32) << 16);
-      const uint32_t t_s = t_lane + qi * AK;
+      const uint32_t t_s = t_lane + qi * 128;
       const uint32_t t_o = t_lane + kOCol + qi * D;
-      const float c = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
+      const float c2 = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
       float m = -INFINITY, l = 0.f;
-      uint8_t* pbuf = sP + qi * kPBytes;
-      for (int j = 0; j < n_kt; ++j) {
-        ptx::mbar_wait(&s_full[qi], j & 1);
+#pragma unroll 1
+      for (int c = 0; c < n_ch; ++c) {
+        const int cur = c & 1;
+        // pull S chunk c out of TMEM and hand the slot back to the MMA warp
+        // (S(c+2) then overlaps this chunk's exp2 work; the other q-tile's warps
+        // on the same SM sub-partitions overlap this warp's TMEM-load latency)
+        ptx::mbar_wait(&s_full[qi * 2 + cur], (c >> 1) & 1);
         ptx::tc_fence_after();
-        const bool full_tile = (j + 1) * AK <= len;
-        float tmax = -INFINITY;
+        if (warp == 0 && lane == 0) atrace<TRACE>(3 + 3 * (c & 7));
+        uint32_t vc[KC];
+        ptx::tmem_ld_32x32b_x32(t_s + cur * KC, *reinterpret_cast<uint32_t(*)[32]>(&vc[0]));
+        ptx::tmem_ld_32x32b_x32(t_s + cur * KC + 32, *reinterpret_cast<uint32_t(*)[32]>(&vc[32]));
+        ptx::tmem_wait_ld();
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(&s_free[qi * 2 + cur]);
+        const int kbase = c * KC;
+        const bool full = kbase + KC <= len;
+        float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
-        for (int ch = 0; ch < AK / 32; ++ch) {
-          uint32_t v[32];
-          ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
-          ptx::tmem_wait_ld();
-#pragma unroll
-          for (int e = 0; e < 32; ++e) {
-            if (full_tile || valid_key(j * AK + ch * 32 + e, len)) tmax = fmaxf(tmax, __uint_as_float(v[e]));
-          }
-        }
-        // P buffer (and O) are read / accumulated by PV_{j-1}: wait for it
-        if (j > 0) {
-          ptx::mbar_wait(&pv_done[qi], (j - 1) & 1);
-          ptx::tc_fence_after();
-        }
-        if (j == 0) {
-          m = tmax;
-        } else if (__any_sync(0xffffffffu, (tmax - m) * c > kRescaleLog2)) {
+        for (int e = 0; e < KC; ++e)
+          if (full || kbase + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vc[e]));
+        const float cmax = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+        if (c == 0) {
+          m = cmax;
+        } else if (__any_sync(0xffffffffu, (cmax - m) * c2 > kRescaleLog2)) {
           // warp-uniform branch (tcgen05.ld/st are warp-collective): rows whose
           // max rose by > 2^8 rescale O and l, the others multiply by 1
           float alpha = 1.f;
-          if ((tmax - m) * c > kRescaleLog2) {
-            alpha = ex2_approx((m - tmax) * c);
+          if ((cmax - m) * c2 > kRescaleLog2) {
+            alpha = ex2_approx((m - cmax) * c2);
             l *= alpha;
-            m = tmax;
+            m = cmax;
           }
-#pragma unroll
-          for (int half = 0; half < 2; ++half) {
-            uint32_t v[32];
-            ptx::tmem_ld_32x32b_x32(t_o + half * 32, v);
+          ptx::mbar_wait(&pv_done[qi * 2 + ((c - 1) & 1)], ((c - 1) >> 1) & 1);  // O holds PV_0..c-1
+          ptx::tc_fence_after();
+#pragma unroll 1
+          for (int hh = 0; hh < 4; ++hh) {
+            uint32_t ov[16];
+            ptx::tmem_ld_32x32b_x16(t_o + hh * 16, ov);
             ptx::tmem_wait_ld();
 #pragma unroll
-            for (int e = 0; e < 32; ++e) v[e] = __float_as_uint(__uint_as_float(v[e]) * alpha);
-            ptx::tmem_st_32x32b_x32(t_o + half * 32, v);
+            for (int e = 0; e < 16; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
+            ptx::tmem_st_32x32b_x16(t_o + hh * 16, ov);
           }
           ptx::tmem_wait_st();
         }
-        const float mc = m * c;
+        if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
+        // P slot `cur` was read by PV(c-2)
+        if (c >= 2) ptx::mbar_wait(&pv_done[qi * 2 + cur], ((c - 2) >> 1) & 1);
+        const float mc = m * c2;
+        uint8_t* prow = sP + (qi * 2 + cur) * kPBytes + r * 128;
+        float ls[2] = {0.f, 0.f};
 #pragma unroll
-        for (int ch = 0; ch < AK / 32; ++ch) {
-          uint32_t v[32];
-          ptx::tmem_ld_32x32b_x32(t_s + ch * 32, v);
-          ptx::tmem_wait_ld();
+        for (int ch = 0; ch < 2; ++ch) {
           uint32_t pk[16];
 #pragma unroll
           for (int e = 0; e < 32; e += 2) {
-            float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c, -mc));
-            float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c, -mc));
-            if (!full_tile) {
-              if (!valid_key(j * AK + ch * 32 + e, len)) p0 = 0.f;
-              if (!valid_key(j * AK + ch * 32 + e + 1, len)) p1 = 0.f;
+            const int k = ch * 32 + e;
+            float p0 = ex2_approx(fmaf(__uint_as_float(vc[k]), c2, -mc));
+            float p1 = ex2_approx(fmaf(__uint_as_float(vc[k + 1]), c2, -mc));
+            if (!full) {
+              if (kbase + k >= len) p0 = 0.f;
+              if (kbase + k + 1 >= len) p1 = 0.f;
             }
-            l += p0 + p1;
+            ls[0] += p0;
+            ls[1] += p1;
             pk[e >> 1] = pack_bf16x2(p0, p1);
           }
-          // keys ch*32 .. +31 -> K-block ch/2, 16-byte chunks (ch%2)*4 .. +3 of row r
-          uint8_t* rowp = pbuf + (ch >> 1) * kTileBytes + r * 128;
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
-            const int chunk = (ch & 1) * 4 + i;
-            *reinterpret_cast<uint4*>(rowp + ((chunk ^ (r & 7)) << 4)) =
+            const int chunk16 = ch * 4 + i;
+            *reinterpret_cast<uint4*>(prow + ((chunk16 ^ (r & 7)) << 4)) =
                 make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
           }
         }
+        l += ls[0] + ls[1];
         ptx::fence_proxy_async_smem();
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&p_full[qi]);
+        if (lane == 0) ptx::mbar_arrive(&p_full[qi * 2 + cur]);
+        if (warp == 0 && lane == 0) atrace<TRACE>(5 + 3 * (c & 7));
       }
-      // O = (sum_j P_j V_j) / l
-      ptx::mbar_wait(&pv_done[qi], (n_kt - 1) & 1);
+      // O = (sum_c P_c V_c) / l
+      ptx::mbar_wait(&pv_done[qi * 2 + ((n_ch - 1) & 1)], ((n_ch - 1) >> 1) & 1);
       ptx::tc_fence_after();
       const float inv = 1.f / l;
       uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
 #pragma unroll
-      for (int half = 0; half < 2; ++half) {
-        uint32_t v[32];
-        ptx::tmem_ld_32x32b_x32(t_o + half * 32, v);
+      for (int hh = 0; hh < 2; ++hh) {
+        uint32_t ov[32];
+        ptx::tmem_ld_32x32b_x32(t_o + hh * 32, ov);
         ptx::tmem_wait_ld();
         if (qrow < L) {
 #pragma unroll
           for (int i = 0; i < 4; ++i) {
             uint4 u;
-            u.x = pack_bf16x2(__uint_as_float(v[8 * i + 0]) * inv, __uint_as_float(v[8 * i + 1]) * inv);
-            u.y = pack_bf16x2(__uint_as_float(v[8 * i + 2]) * inv, __uint_as_float(v[8 * i + 3]) * inv);
-            u.z = pack_bf16x2(__uint_as_float(v[8 * i + 4]) * inv, __uint_as_float(v[8 * i + 5]) * inv);
-            u.w = pack_bf16x2(__uint_as_float(v[8 * i + 6]) * inv, __uint_as_float(v[8 * i + 7]) * inv);
-            orow[half * 4 + i] = u;
+            u.x = pack_bf16x2(__uint_as_float(ov[8 * i + 0]) * inv, __uint_as_float(ov[8 * i + 1]) * inv);
+            u.y = pack_bf16x2(__uint_as_float(ov[8 * i + 2]) * inv, __uint_as_float(ov[8 * i + 3]) * inv);
+            u.z = pack_bf16x2(__uint_as_float(ov[8 * i + 4]) * inv, __uint_as_float(ov[8 * i + 5]) * inv);
+            u.w = pack_bf16x2(__uint_as_float(ov[8 * i + 6]) * inv, __uint_as_float(ov[8 * i + 7]) * inv);
+            orow[hh * 4 + i] = u;
           }
         }
       }
@@ -271,6 +329,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   }
   ptx::tc_fence_before();
   __syncthreads();
+  if (threadIdx.x == 0) atrace<TRACE>(1);
   if (warp == kMmaWarp) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc(tmem, kTmemCols);
@@ -314,24 +373,47 @@ __global__ void __launch_bounds__(128) attn_f32_kernel(int B, int L, int heads, 
 
 }  // namespace
 
+static bool g_attn_trace_on = false;
+
+int set_attn_trace(unsigned long long* buf) {
+  g_attn_trace_on = buf != nullptr;
+  return (int)cudaMemcpyToSymbol(g_atrace, &buf, sizeof(buf));
+}
+
+template <int NQ, int MAXKT>
+cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
+  using Cfg = AttnCfg<NQ, MAXKT>;
+  static bool attr = false;
+  if (!attr) {
+    cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, false>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               Cfg::kSmem);
+    if (e != cudaSuccess) return e;
+    attr = true;
+  }
+  dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
+  if (g_attn_trace_on)
+    attn_tc_kernel<NQ, MAXKT, true><<<grid, Cfg::kThreads, Cfg::kSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
+  else
+    attn_tc_kernel<NQ, MAXKT, false><<<grid, Cfg::kThreads, Cfg::kSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
+  return cudaGetLastError();
+}
+
 bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) {
   p->B = B; p->L = L; p->heads = heads; p->dt = dt; p->qkv = qkv;
   if (dt != DT_BF16) return true;
-  if (L > AK * kMaxKT) return false;
+  if (L > AK * 4) return false;
   return encode_tmap_bf16_2d(&p->tm, qkv, (uint64_t)3 * heads * D, (uint64_t)B * L, 64, 128, 128);
 }
 
 cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
   if (p.B <= 0 || p.L <= 0) return cudaSuccess;
   if (p.dt == DT_BF16) {
-    static bool attr = false;
-    if (!attr) {
-      cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, kAttnSmem);
-      if (e != cudaSuccess) return e;
-      attr = true;
-    }
-    dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
-    attn_tc_kernel<<<grid, kAttnThreads, kAttnSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
+    if (p.L <= 128) return attn_launch_cfg<1, 1>(p, lengths, o, s);
+    if (p.L <= 256) return attn_launch_cfg<2, 2>(p, lengths, o, s);
+    return attn_launch_cfg<2, 4>(p, lengths, o, s);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
     attn_f32_kernel<<<(unsigned)((warps + 3) / 4), 128, 0, s>>>(p.B, p.L, p.heads, (const float*)p.qkv, lengths,

@@ -15,6 +15,7 @@ enum Epi { EPI_BIAS = 0, EPI_BIAS_GELU = 1, EPI_BIAS_RESID = 2 };
 
 int num_sms();
 int set_gemm_trace(unsigned long long* buf);  // profiling hook, nullptr = off
+int set_attn_trace(unsigned long long* buf);  // profiling hook, nullptr = off
 
 // ---- a1: embedding + LN;  a5/a8: LN ------------------------------------------------------
 cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int32_t* ids,

@@ -523,3 +523,8 @@ extern "C" int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K) {
   if (M < 1 || N % 64 || K % 64 || N < 64 || K < 64) return 0;
   return tc_choose_bn(M, N, K);
 }
+
+extern "C" int arlo_debug_attn_trace(void* buf) {
+  cudaError_t e = (cudaError_t)set_attn_trace((unsigned long long*)buf);
+  return e == cudaSuccess ? ARLO_OK : cuda_fail(e, "arlo_debug_attn_trace");
+}

@@ -155,6 +155,8 @@ def test_embedding_ln(arlo_lib, dtype):
     (512, 2, [512, 300, 7]),
     (32, 2, [32, 5, 1, 17]),
     (64, 16, [63, 64]),
+    (256, 4, [256, 200, 129, 1, 128]),
+    (384, 2, [384, 257, 100]),
 ])
 @pytest.mark.parametrize("dtype", [0, 1])
 def test_attention_masked(arlo_lib, L, heads, lengths, dtype):
