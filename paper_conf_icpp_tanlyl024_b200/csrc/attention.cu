@@ -88,6 +88,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   constexpr int kSoftWarps = Cfg::kSoftWarps, kProdWarp = Cfg::kProdWarp, kMmaWarp = Cfg::kMmaWarp;
   constexpr int kAttnThreads = Cfg::kThreads;
   constexpr uint32_t kOCol = Cfg::kOCol, kTmemCols = Cfg::kTmemCols;
+  pdl_begin();
   const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
   const int len = __ldg(lengths + b);
@@ -395,10 +396,10 @@ cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, 
   }
   dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
   if (g_attn_trace_on)
-    attn_tc_kernel<NQ, MAXKT, true><<<grid, Cfg::kThreads, Cfg::kSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
-  else
-    attn_tc_kernel<NQ, MAXKT, false><<<grid, Cfg::kThreads, Cfg::kSmem, s>>>(p.tm, p.L, p.heads, lengths, (bf16*)o);
-  return cudaGetLastError();
+    return launch_k(attn_tc_kernel<NQ, MAXKT, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
+                    lengths, (bf16*)o);
+  return launch_k(attn_tc_kernel<NQ, MAXKT, false>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
+                  lengths, (bf16*)o);
 }
 
 bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) {

@@ -98,6 +98,7 @@ __global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* _
                                                         const float* __restrict__ b, float eps,
                                                         T* __restrict__ out) {
   constexpr int VN = Vec<T>::N;
+  pdl_begin();
   const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
   if (row >= M) return;
@@ -121,6 +122,7 @@ __global__ void __launch_bounds__(256) embed_ln_kernel(int B, int L, int H, int 
                                                        const float* __restrict__ b, float eps,
                                                        T* __restrict__ out, int32_t* err_flag) {
   constexpr int VN = Vec<T>::N;
+  pdl_begin();
   const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
   if (row >= B * L) return;
@@ -181,10 +183,10 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
   const int maxv = round_maxv(H / vn);
   dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
   if (dt == DT_BF16) {
-    ARLO_MAXV_SWITCH(maxv, layernorm_kernel<bf16, MV><<<grid, block, 0, s>>>(
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, 0, s,
         M, H, (const bf16*)in, g, b, eps, (bf16*)out));
   } else {
-    ARLO_MAXV_SWITCH(maxv, layernorm_kernel<float, MV><<<grid, block, 0, s>>>(
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<float, MV>, grid, block, 0, s,
         M, H, (const float*)in, g, b, eps, (float*)out));
   }
   return cudaGetLastError();
@@ -200,11 +202,11 @@ cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int3
   const int maxv = round_maxv(H / vn);
   dim3 grid((B * L + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
   if (dt == DT_BF16) {
-    ARLO_MAXV_SWITCH(maxv, embed_ln_kernel<bf16, MV><<<grid, block, 0, s>>>(
+    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<bf16, MV>, grid, block, 0, s,
         B, L, H, vocab, ids, lengths, (const bf16*)word, (const bf16*)pos, (const bf16*)type, g, b,
         eps, (bf16*)out, err_flag));
   } else {
-    ARLO_MAXV_SWITCH(maxv, embed_ln_kernel<float, MV><<<grid, block, 0, s>>>(
+    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<float, MV>, grid, block, 0, s,
         B, L, H, vocab, ids, lengths, (const float*)word, (const float*)pos, (const float*)type, g,
         b, eps, (float*)out, err_flag));
   }

@@ -201,6 +201,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_begin();  // setup above overlapped the previous kernel's tail
   if (threadIdx.x == 0) trace(0);
 
   if (warp == kProducerWarp) {
@@ -338,6 +339,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  pdl_begin();  // setup above overlapped the previous kernel's tail
 
   if (warp == kProducerWarp) {
     if (lane == 0) {
@@ -439,8 +441,8 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  kern<<<p.grid, kThreads, C::SMEM, s>>>(p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias, (const bf16*)p.resid);
-  return cudaGetLastError();
+  return launch_k(kern, dim3(p.grid), dim3(kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias,
+                  (const bf16*)p.resid);
 }
 
 template <int BN, bool PAIR>

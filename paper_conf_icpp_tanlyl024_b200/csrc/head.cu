@@ -40,6 +40,7 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
                                                      float* __restrict__ pooled) {
   extern __shared__ float xs[];  // [kRows][H]
+  pdl_begin();
   const int b0 = blockIdx.y * kRows;
   const int nb = min(kRows, B - b0);
   for (int i = threadIdx.x; i < kRows * H; i += blockDim.x) {
@@ -75,6 +76,7 @@ template <typename T>
 __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const float* __restrict__ pooled,
                                                         const T* __restrict__ w_c, const float* __restrict__ b_c,
                                                         float* __restrict__ logits) {
+  pdl_begin();
   const int b = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const float* p = pooled + (size_t)b * H;
@@ -98,9 +100,11 @@ cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p,
     attr = true;
   }
   dim3 grid((H + kFeat - 1) / kFeat, (B + kRows - 1) / kRows);
-  pooler_kernel<T><<<grid, 256, smem, s>>>(B, L, H, (const T*)x, (const T*)w_p, b_p, pooled);
-  classifier_kernel<T><<<B, 64, 0, s>>>(H, C, pooled, (const T*)w_c, b_c, logits);
-  return cudaGetLastError();
+  cudaError_t e = launch_k(pooler_kernel<T>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p, b_p,
+                           pooled);
+  if (e != cudaSuccess) return e;
+  return launch_k(classifier_kernel<T>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c, b_c,
+                  logits);
 }
 
 }  // namespace

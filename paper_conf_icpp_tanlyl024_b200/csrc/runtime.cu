@@ -13,6 +13,7 @@
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <mutex>
 #include <new>
@@ -40,6 +41,11 @@ int set_error(int code, const char* fmt, ...) {
   return code;
 }
 void clear_error() { g_err.clear(); }
+
+bool pdl_enabled() {
+  static const bool on = getenv("ARLO_NO_PDL") == nullptr;
+  return on;
+}
 
 static int cuda_fail(cudaError_t e, const char* what) {
   return set_error(ARLO_ECUDA, "%s: %s (%s)", what, cudaGetErrorName(e), cudaGetErrorString(e));
