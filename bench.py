@@ -31,6 +31,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 from paper_conf_icpp_tanlyl024_b200 import metrics  # noqa: E402
+from paper_conf_icpp_tanlyl024_b200 import replicas  # noqa: E402
 from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
 
 RUNTIME_LS = (64, 128, 256, 512)
@@ -52,7 +53,7 @@ def parse():
 
 # ------------------------------------------------------------------------- workload plan
 def make_step_requests(step: int, rank: int, R: int, cfg):
-    lengths = wl.sample_lengths(R, seed=wl.SEED_LENGTHS + 7919 * step + 104729 * rank)
+    lengths = wl.sample_lengths(R, seed=replicas.step_seed(wl.SEED_LENGTHS, step, rank))
     return lengths
 
 
@@ -256,12 +257,11 @@ def main():
             lat[L] += [a.elapsed_time(b)] * n
             done[L] += [st.elapsed_time(b)] * n
     total_req = R * args.steps
-    t_max = total_ms
-    if world > 1:
-        t = torch.tensor([total_ms], device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        t_max = float(t.item())
-    value = world * total_req / (t_max / 1e3)
+    # whole job: requests summed over ranks / max over ranks of the timed region
+    value, t_max, _ = replicas.aggregate_throughput(float(total_req), total_ms)
+    e2e_res = None
+    if not args.no_extras:
+        e2e_res = e2e(runtimes, torch, stream, steps[args.warmup:], R, cfg, flush)
 
     result = None
     if rank == 0:
@@ -292,7 +292,8 @@ def main():
         result["roofline"] = roofline_dominant(arlo, torch, dev, stream, step_times)
         result["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
         result["uniform_512"] = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
-        result["e2e"] = e2e(runtimes, torch, stream, steps[args.warmup:], R, cfg, flush)
+        result["e2e"] = e2e_res
+        result["bert_large"] = bert_large_per_L(arlo, torch, dev, stream, local_rank)
         if not args.no_cpu_baseline:
             result["cpu_baseline"] = cpu_baseline()
     if rank == 0:
@@ -301,6 +302,50 @@ def main():
         rt.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def bert_large_per_L(arlo, torch, dev, stream, device_index):
+    """north_star target: per-L bf16 BERT-large forward at L >= 256 as a fraction of
+    the B200 tensor peak (BASELINE configs[2]: L in {128,256,512}, batch up to 64).
+    One forward per (L, b) replayed back to back from the runtime's CUDA graph."""
+    cfg = wl.BERT_LARGE
+    W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg, seed=wl.SEED_WEIGHTS), arlo.BF16, dev),
+                     arlo.BF16, device_index)
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    peak = peaks.get("bf16_tflops", 1590.0)
+    peak_sus = peaks.get("bf16_tflops_sustained", 1400.0)
+    out = {}
+    for L in (128, 256, 512):
+        rt = arlo.Runtime(W, L, 64)
+        rt.set_stream(stream)
+        row = {}
+        for b in (1, 16, 64):
+            lens = np.full(b, L, np.int32)
+            ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
+            ld = torch.from_numpy(lens).to(dev)
+            o = torch.empty((b, cfg.num_labels), device=dev)
+            for _ in range(3):
+                rt.enqueue(b, ids, ld, o)
+            reps = 5
+            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            for _ in range(reps):
+                rt.enqueue(b, ids, ld, o)
+            e.record(stream)
+            torch.cuda.synchronize()
+            ms = a.elapsed_time(e) / reps
+            tf = metrics.forward_flops(cfg, b, L) / (ms / 1e3) / 1e12
+            row[str(b)] = {"ms": ms, "static_tflops": tf, "frac_of_peak": tf / peak,
+                           "frac_of_sustained_peak": tf / peak_sus}
+        out[str(L)] = row
+        rt.close()
+    W.close()
+    return {"per_L": out, "peak_tflops": peak, "peak_sustained_tflops": peak_sus,
+            "note": "static FLOPs = layers*(24bLH^2+4bL^2H)+b(2H^2+2HC); back-to-back graph replays"}
 
 
 def roofline_dominant(arlo, torch, dev, stream, step_times):
@@ -435,7 +480,8 @@ def e2e(runtimes, torch, stream, steps, R, cfg, flush):
             d2h += 4 * n * cfg.num_labels + 4
     h2d /= len(host)
     d2h /= len(host)
-    return {"value": len(host) * R / (tot / 1e3), "unit": "req/s", "h2d_bytes_per_step": int(h2d),
+    value, _, _ = replicas.aggregate_throughput(float(len(host) * R), tot)  # all ranks, max time
+    return {"value": value, "unit": "req/s", "h2d_bytes_per_step": int(h2d),
             "d2h_bytes_per_step": int(d2h), "api": "arlo_infer (synchronous, pinned host buffers)"}
 
 
