@@ -33,6 +33,16 @@ int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, const void* A, 
                  const float* bias, const void* residual, void* out, int32_t epi,
                  int32_t force_bn, void* stream);
 
+/*
+ * Steps a4+a5 / a7+a8 fused (bf16): out[M,N] = LN(A W^T + bias + residual; gamma, beta, eps)
+ * over full rows, N = hidden size (multiple of 192 or 256 with <= 8 column tiles, or 128).
+ * A cluster of N/BN CTAs shares per-row statistics through distributed shared memory.
+ * `out` may alias `residual`.  Errors: ARLO_EINVAL for unsupported N / bad pointers.
+ */
+int arlo_op_gemm_ln(int32_t M, int32_t N, int32_t K, const void* A, const void* W, const float* bias,
+                    const void* residual, const float* gamma, const float* beta, float eps, void* out,
+                    void* stream);
+
 /* Step a5/a8: out[M,H] = LN(in[M,H]; gamma, beta, eps) per row (biased variance). */
 int arlo_op_layernorm(int32_t dtype, int32_t M, int32_t H, const void* in, const float* gamma,
                       const float* beta, float eps, void* out, void* stream);

@@ -29,7 +29,7 @@ EXPORTED = [
     "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
-    "arlo_op_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
+    "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
     "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
 ]
 
@@ -72,6 +72,7 @@ _sig("arlo_dispatch", C.c_int, _vp, _i32, _P(_i32), _P(_i32))
 _sig("arlo_complete", C.c_int, _vp, _i32, _i32)
 _sig("arlo_sched_outstanding", _i32, _vp, _i32, _i32)
 _sig("arlo_op_gemm", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _i32, _i32, _vp)
+_sig("arlo_op_gemm_ln", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp)
 _sig("arlo_op_layernorm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp)
 _sig("arlo_op_embed", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp, _vp)
 _sig("arlo_op_attention", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp)
@@ -239,6 +240,14 @@ def op_gemm(dtype, A, W, bias, out, epi=EPI_BIAS, residual=None, force_bn=0, str
     N = W.shape[0]
     check(lib.arlo_op_gemm(dtype, M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(residual), _ptr(out), epi,
                            force_bn, _stream_ptr(stream)))
+    return out
+
+
+def op_gemm_ln(A, W, bias, residual, gamma, beta, eps, out, stream=None):
+    M, K = A.shape
+    N = W.shape[0]
+    check(lib.arlo_op_gemm_ln(M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(residual), _ptr(gamma), _ptr(beta), eps,
+                              _ptr(out), _stream_ptr(stream)))
     return out
 
 

@@ -60,17 +60,17 @@ constexpr int tmem_cols_for(int n) {
 // PAIR = false: one CTA computes a 128 x BN tile; PAIR = true: a CTA pair
 // (cluster of 2, cta_group::2) computes a 256 x BN tile, each CTA holding 128
 // rows of A, BN/2 rows of W and its 128 x BN half of the accumulator.
-template <int BN, bool PAIR>
+template <int BN, bool PAIR, int RESERVE = 0>
 struct TcCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
   static constexpr int B_BYTES = B_ROWS * BK * 2;
   static constexpr int STAGE_BYTES = A_BYTES + B_BYTES;
-  static constexpr int STAGES_FIT = (kSmemBudget - kStagingBytes) / STAGE_BYTES;
+  static constexpr int STAGES_FIT = (kSmemBudget - kStagingBytes - RESERVE) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int TMEM_COLS = tmem_cols_for(kAccStages * BN);
   static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages) + 16;
-  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + kStagingBytes + BAR_BYTES;
+  static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + kStagingBytes + BAR_BYTES + RESERVE;
   static_assert(SMEM <= 232448, "shared memory budget");
 };
 
@@ -412,6 +412,269 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   }
 }
 
+// ---------------------------------------------------------------------------------------------
+// GEMM + bias + residual + LayerNorm over the full row (steps a4+a5 and a7+a8 fused):
+//   out[M,N] = LN(A W^T + bias + resid; gamma, beta, eps),  N = hidden (768 / 1024 / 128).
+// A cluster of NT = N / BN single-CTA tiles covers whole rows: CTA rank r owns
+// columns [r*BN, (r+1)*BN) of the same 128-row block.  The epilogue keeps
+// y = acc + bias + resid in TMEM (tcgen05.st back over the accumulator), and
+// the per-row sum and sum of squared deviations are combined across the
+// cluster through distributed shared memory (each warp publishes its partial
+// row sums, arrives on every CTA's stat barrier with release.cluster
+// semantics, waits on its own with acquire.cluster, then reads the NT x 2
+// partials with ld.shared::cluster).  Two-pass statistics (mean, then
+// sum (y-mean)^2) in fp32 as in the unfused LayerNorm; the normalised row is
+// written once (TMA store).  Removes the LayerNorm kernels and the y round
+// trip through memory.
+template <int BN>
+__device__ __forceinline__ float cluster_row_sum(float v, float* red, uint64_t* stat_bar, int& use, int cg,
+                                                 int r_local, int lane, uint32_t nt) {
+  const int set = use & 1;
+  float* slot = red + (set * 2 + cg) * BM + r_local;  // red[set][half][row]
+  *slot = v;
+  __syncwarp();
+  if (lane == 0) {
+    for (uint32_t k = 0; k < nt; ++k) ptx::mbar_arrive_cluster(ptx::mapa_shared(&stat_bar[set], k));
+  }
+  ptx::mbar_wait_cluster(&stat_bar[set], (use >> 1) & 1);
+  float tot = 0.f;
+  for (uint32_t k = 0; k < nt; ++k) {
+    tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * 2 + 0) * BM + r_local, k));
+    tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * 2 + 1) * BM + r_local, k));
+  }
+  ++use;
+  return tot;
+}
+
+template <int BN, typename Release>
+__device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
+                                                 int N, float eps, const float* __restrict__ bias,
+                                                 const bf16* __restrict__ resid, const float* __restrict__ gamma,
+                                                 const float* __restrict__ beta, const CUtensorMap* tmC, uint8_t* stg,
+                                                 int& sc, float* red, uint64_t* stat_bar, int& use, uint32_t nt,
+                                                 Release release) {
+  constexpr int COLS = BN / 2;
+  constexpr int NC = COLS / 32;
+  const int r_local = q * 32 + lane;
+  const int row = row0 + lane;
+  const bool row_ok = row < M;
+  const int col0 = n0 + cg * COLS;
+  const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
+  const float4* g4 = reinterpret_cast<const float4*>(gamma + col0);
+  const float4* be4 = reinterpret_cast<const float4*>(beta + col0);
+  const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
+  const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16) + cg * COLS;
+  // pass 1: y = acc + bias + resid, kept in TMEM; partial row sum
+  float s1 = 0.f;
+#pragma unroll 1
+  for (int c = 0; c < NC; ++c) {
+    uint32_t r[32];
+    uint4 rv[4];
+    if (row_ok) {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) rv[j] = __ldg(res4 + c * 4 + j);
+    } else {
+#pragma unroll
+      for (int j = 0; j < 4; ++j) rv[j] = make_uint4(0, 0, 0, 0);
+    }
+    ptx::tmem_ld_32x32b_x32(t_row + c * 32, r);
+    ptx::tmem_wait_ld();
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float4 b4 = __ldg(bias4 + c * 8 + j);
+      const uint4 u = rv[j >> 1];
+      const float2 fa = unpack_bf16x2((j & 1) ? u.z : u.x), fb = unpack_bf16x2((j & 1) ? u.w : u.y);
+      const float y0 = __uint_as_float(r[4 * j + 0]) + b4.x + fa.x;
+      const float y1 = __uint_as_float(r[4 * j + 1]) + b4.y + fa.y;
+      const float y2 = __uint_as_float(r[4 * j + 2]) + b4.z + fb.x;
+      const float y3 = __uint_as_float(r[4 * j + 3]) + b4.w + fb.y;
+      s1 += (y0 + y1) + (y2 + y3);
+      r[4 * j + 0] = __float_as_uint(y0);
+      r[4 * j + 1] = __float_as_uint(y1);
+      r[4 * j + 2] = __float_as_uint(y2);
+      r[4 * j + 3] = __float_as_uint(y3);
+    }
+    ptx::tmem_st_32x32b_x32(t_row + c * 32, r);
+  }
+  ptx::tmem_wait_st();
+  const float mean = cluster_row_sum<BN>(s1, red, stat_bar, use, cg, r_local, lane, nt) / (float)N;
+  // pass 2: sum of squared deviations
+  float s2 = 0.f;
+#pragma unroll 1
+  for (int c = 0; c < NC; ++c) {
+    uint32_t r[32];
+    ptx::tmem_ld_32x32b_x32(t_row + c * 32, r);
+    ptx::tmem_wait_ld();
+#pragma unroll
+    for (int j = 0; j < 32; ++j) {
+      const float d = __uint_as_float(r[j]) - mean;
+      s2 = fmaf(d, d, s2);
+    }
+  }
+  const float var = cluster_row_sum<BN>(s2, red, stat_bar, use, cg, r_local, lane, nt) / (float)N;
+  const float rstd = 1.0f / sqrtf(var + eps);
+  // pass 3: normalise, affine, bf16, TMA store
+#pragma unroll 1
+  for (int c = 0; c < NC; ++c) {
+    uint32_t r[32];
+    ptx::tmem_ld_32x32b_x32(t_row + c * 32, r);
+    ptx::tmem_wait_ld();
+    if (c == NC - 1) {
+      ptx::tc_fence_before();
+      __syncwarp();
+      if (lane == 0) release();
+    }
+    uint32_t pk[16];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float4 g = __ldg(g4 + c * 8 + j), be = __ldg(be4 + c * 8 + j);
+      const float o0 = (__uint_as_float(r[4 * j + 0]) - mean) * rstd * g.x + be.x;
+      const float o1 = (__uint_as_float(r[4 * j + 1]) - mean) * rstd * g.y + be.y;
+      const float o2 = (__uint_as_float(r[4 * j + 2]) - mean) * rstd * g.z + be.z;
+      const float o3 = (__uint_as_float(r[4 * j + 3]) - mean) * rstd * g.w + be.w;
+      pk[2 * j] = pack_bf16x2(o0, o1);
+      pk[2 * j + 1] = pack_bf16x2(o2, o3);
+    }
+    uint8_t* buf = stg + (sc & 1) * kStgBytes;
+    if (sc >= 2) {
+      if (lane == 0) ptx::bulk_wait_read<1>();
+      __syncwarp();
+    }
+#pragma unroll
+    for (int j = 0; j < 4; ++j) {
+      const int sw = j ^ ((lane >> 1) & 3);
+      *reinterpret_cast<uint4*>(buf + lane * 64 + sw * 16) =
+          make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+    }
+    ptx::fence_proxy_async_smem();
+    __syncwarp();
+    if (lane == 0) {
+      ptx::tma_store_2d(tmC, buf, col0 + c * 32, row0);
+      ptx::bulk_commit();
+    }
+    ++sc;
+  }
+}
+
+constexpr int kLnReserve = 4 * BM * 4 + 16;  // row-statistics exchange buffers + 2 stat barriers
+
+template <int BN>
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+               const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
+               const bf16* __restrict__ resid, const float* __restrict__ gamma, const float* __restrict__ beta,
+               float eps) {
+  using C = TcCfg<BN, false, kLnReserve>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
+  float* red = reinterpret_cast<float*>(sStg + kStagingBytes);  // [2 sets][2 halves][128 rows]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red + 4 * BM);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint64_t* tempty = tfull + kAccStages;
+  uint64_t* stat_bar = tempty + kAccStages;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(stat_bar + 2);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  uint32_t nt;
+  asm volatile("mov.u32 %0, %%cluster_nctarank;" : "=r"(nt));
+  const uint32_t rank = ptx::cluster_ctarank();
+  const int cid = blockIdx.x / nt, ncl = gridDim.x / nt;
+  const int num_m = (M + BM - 1) / BM;
+  const int n0 = rank * BN;
+  const int kblocks = K / BK;
+
+  if (warp == kProducerWarp && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    ptx::tma_prefetch_desc(&tmC);
+    for (int s = 0; s < C::STAGES; ++s) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int a = 0; a < kAccStages; ++a) {
+      ptx::mbar_init(&tfull[a], 1);
+      ptx::mbar_init(&tempty[a], kEpiWarps);
+    }
+    for (int i = 0; i < 2; ++i) ptx::mbar_init(&stat_bar[i], kEpiWarps * nt);
+    ptx::fence_mbar_init();
+  }
+  if (warp == kMmaWarp) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
+  ptx::tc_fence_before();
+  ptx::cluster_sync();  // peers' stat barriers are initialised before any remote arrive
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  pdl_begin();
+
+  if (warp == kProducerWarp) {
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int mb = cid; mb < num_m; mb += ncl) {
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait(&empty[stage], phase ^ 1);
+          ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+          ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, mb * BM);
+          ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+      }
+    }
+  } else if (warp == kMmaWarp) {
+    if (lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      int acc = 0;
+      uint32_t acc_phase = 0;
+      for (int mb = cid; mb < num_m; mb += ncl) {
+        ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
+        ptx::tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * BN;
+        for (int kb = 0; kb < kblocks; ++kb) {
+          ptx::mbar_wait(&full[stage], phase);
+          ptx::tc_fence_after();
+          const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+          const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
+#pragma unroll
+          for (int k = 0; k < BK / 16; ++k)
+            ptx::mma_bf16_ss(d_tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32), idesc,
+                             (kb | k) != 0);
+          ptx::mma_commit(&empty[stage]);
+          if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+        }
+        ptx::mma_commit(&tfull[acc]);
+        if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+      }
+    }
+  } else {
+    const int q = warp & 3, cg = warp >> 2;
+    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    int sc = 0, use = 0;
+    int acc = 0;
+    uint32_t acc_phase = 0;
+    for (int mb = cid; mb < num_m; mb += ncl) {
+      ptx::mbar_wait(&tfull[acc], acc_phase);
+      ptx::tc_fence_after();
+      uint64_t* te = &tempty[acc];
+      epilogue_ln_tile<BN>(tmem_base + acc * BN, q, cg, lane, mb * BM + q * 32, n0, M, N, eps, bias, resid, gamma,
+                           beta, &tmC, stg, sc, red, stat_bar, use, nt, [te]() { ptx::mbar_arrive(te); });
+      if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
+    }
+    if (lane == 0) ptx::bulk_wait<0>();
+  }
+
+  ptx::tc_fence_before();
+  ptx::cluster_sync();  // no CTA leaves while a peer may still read its stats or arrive on its barriers
+  if (warp == kMmaWarp) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem_base, C::TMEM_COLS);
+  }
+}
+
 typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*,
                                   const cuuint64_t*, const cuuint64_t*, const cuuint32_t*,
                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
@@ -526,7 +789,7 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn == 64) return false;
   if (N % bn) return false;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi; p->ln = false;
   p->bias = bias; p->resid = resid; p->out = out;
   const int tile_m = pair ? 2 * BM : BM;
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
@@ -538,7 +801,67 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   return true;
 }
 
+template <int BN>
+cudaError_t launch_ln(const TcGemmPlan& p, cudaStream_t s) {
+  using C = TcCfg<BN, false, kLnReserve>;
+  constexpr int SMEM = C::SMEM;
+  static_assert(SMEM <= 232448, "fused LN smem");
+  auto kern = gemm_ln_kernel<BN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+    if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3(p.grid);
+  cfg.blockDim = dim3(kThreads);
+  cfg.dynamicSmemBytes = SMEM;
+  cfg.stream = s;
+  cudaLaunchAttribute attr[2];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = p.N / BN;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = pdl_enabled() ? 2 : 1;
+  return cudaLaunchKernelEx(&cfg, kern, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias, (const bf16*)p.resid, p.gamma,
+                            p.beta, p.eps);
+}
+
+// Fused GEMM + bias + residual + LayerNorm over full rows (N = hidden).
+bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W, const float* bias,
+                     const void* resid, const float* gamma, const float* beta, float eps, void* out) {
+  if (M <= 0 || K % 64 || K <= 0) return false;
+  int bn = 0;
+  if (N % 192 == 0 && N / 192 <= 8 && N > 256) bn = 192;
+  if (N % 256 == 0 && N / 256 <= 8) bn = 256;
+  if (N == 128) bn = 128;
+  if (!bn) return false;
+  const int nt = N / bn;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->bias = bias; p->resid = resid; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
+  const int num_m = (M + BM - 1) / BM;
+  const int clusters = num_sms() / nt;
+  p->grid = (num_m < clusters ? num_m : clusters) * nt;
+  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, 32, 32, 64)) return false;
+  return true;
+}
+
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
+  if (p.ln) {
+    switch (p.BN) {
+      case 128: return launch_ln<128>(p, s);
+      case 192: return launch_ln<192>(p, s);
+      case 256: return launch_ln<256>(p, s);
+    }
+    return cudaErrorInvalidValue;
+  }
   if (p.pair) {
     switch (p.BN) {
       case 128: return launch_bn<128, true>(p, s);

@@ -34,6 +34,10 @@ struct TcGemmPlan {
   CUtensorMap tmC;  // output      [M, N] bf16, box {32, 32}, 64B swizzle (epilogue TMA stores)
   int M, N, K, BN, epi, grid;
   bool pair;  // CTA-pair (cta_group::2) kernel, 256-row tiles
+  bool ln;    // fused residual + LayerNorm epilogue over full rows (cluster of N/BN CTAs)
+  const float* gamma;
+  const float* beta;
+  float eps;
   const float* bias;
   const void* resid;
   void* out;
@@ -42,6 +46,10 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
                   const float* bias, const void* resid, void* out, int epi, int force_bn);
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s);
 int tc_choose_bn(int M, int N, int K);
+// out = LN(A W^T + bias + resid; gamma, beta, eps), N = hidden size (128 / 768 / 1024 ...).
+// `out` may alias `resid` (each tile reads its residual before storing the same region).
+bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W, const float* bias,
+                     const void* resid, const float* gamma, const float* beta, float eps, void* out);
 
 cudaError_t launch_gemm_simt(DType dt, int M, int N, int K, const void* A, const void* W,
                              const float* bias, const void* resid, void* out, int epi,

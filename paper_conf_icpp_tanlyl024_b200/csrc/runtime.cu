@@ -159,6 +159,7 @@ struct LayerPlans {
 struct Bucket {
   int b = 0;
   std::vector<LayerPlans> plans;  // bf16 only
+  bool fused_ln = false;          // o / f2 plans carry residual + LayerNorm (no separate LN kernels)
   AttnPlan attn;
   cudaGraphExec_t exec = nullptr;
   size_t nodes = 0;
@@ -214,9 +215,10 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "out-proj gemm launch");
     }
-    ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
-                               c.ln_eps, rt->X, s),
-              "ln1 launch");
+    if (!bk.fused_ln)
+      ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
+                                 c.ln_eps, rt->X, s),
+                "ln1 launch");
     if (dt == DT_BF16) {
       ARLO_CUDA(tc_launch_gemm(bk.plans[l].f1, s), "ffn1 gemm launch");
       ARLO_CUDA(tc_launch_gemm(bk.plans[l].f2, s), "ffn2 gemm launch");
@@ -228,9 +230,10 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "ffn2 gemm launch");
     }
-    ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
-                               c.ln_eps, rt->X, s),
-              "ln2 launch");
+    if (!bk.fused_ln)
+      ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
+                                 c.ln_eps, rt->X, s),
+                "ln2 launch");
   }
   ARLO_CUDA(launch_head(dt, b, L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
                         (const float*)w->hd(3), rt->pooled, rt->logits, s),
@@ -243,16 +246,31 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
   const arlo_model_config& c = w->cfg;
   const int M = bk.b * rt->L, H = c.hidden, F = c.ffn;
   bk.plans.resize(c.layers);
+  // residual + LayerNorm fused into the out-proj / FFN2 GEMM epilogues when the
+  // hidden size splits into a cluster of <= 8 column tiles (all BERT configs)
+  TcGemmPlan probe;
+  bk.fused_ln = getenv("ARLO_NO_FUSED_LN") == nullptr &&
+                tc_plan_gemm_ln(&probe, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X,
+                                (const float*)w->lt(0, LN1_G), (const float*)w->lt(0, LN1_B), c.ln_eps, rt->X);
   for (int l = 0; l < c.layers; ++l) {
     LayerPlans& p = bk.plans[l];
     bool ok = tc_plan_gemm(&p.qkv, M, 3 * H, H, rt->X, w->lt(l, LW_QKV), (const float*)w->lt(l, LB_QKV), nullptr,
                            rt->QKV, EPI_BIAS, 0) &&
-              tc_plan_gemm(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y,
-                           EPI_BIAS_RESID, 0) &&
               tc_plan_gemm(&p.f1, M, F, H, rt->X, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, rt->F,
-                           EPI_BIAS_GELU, 0) &&
-              tc_plan_gemm(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
-                           EPI_BIAS_RESID, 0);
+                           EPI_BIAS_GELU, 0);
+    if (bk.fused_ln) {
+      ok = ok &&
+           tc_plan_gemm_ln(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X,
+                           (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B), c.ln_eps, rt->X) &&
+           tc_plan_gemm_ln(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X,
+                           (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B), c.ln_eps, rt->X);
+    } else {
+      ok = ok &&
+           tc_plan_gemm(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y,
+                        EPI_BIAS_RESID, 0) &&
+           tc_plan_gemm(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
+                        EPI_BIAS_RESID, 0);
+    }
     if (!ok) return set_error(ARLO_ECUDA, "tensor-map encoding failed (cuTensorMapEncodeTiled unavailable?)");
   }
   return ARLO_OK;
@@ -533,4 +551,17 @@ extern "C" int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K) {
 extern "C" int arlo_debug_attn_trace(void* buf) {
   cudaError_t e = (cudaError_t)set_attn_trace((unsigned long long*)buf);
   return e == cudaSuccess ? ARLO_OK : cuda_fail(e, "arlo_debug_attn_trace");
+}
+
+extern "C" int arlo_op_gemm_ln(int32_t M, int32_t N, int32_t K, const void* A, const void* W, const float* bias,
+                               const void* residual, const float* gamma, const float* beta, float eps, void* out,
+                               void* stream) {
+  clear_error();
+  if (M < 1 || K % 64 || K < 64 || !A || !W || !bias || !residual || !gamma || !beta || !out)
+    return set_error(ARLO_EINVAL, "arlo_op_gemm_ln: bad arguments");
+  TcGemmPlan p;
+  if (!tc_plan_gemm_ln(&p, M, N, K, A, W, bias, residual, gamma, beta, eps, out))
+    return set_error(ARLO_EINVAL, "arlo_op_gemm_ln: N = %d not supported (needs N/192 or N/256 <= 8, or 128)", N);
+  ARLO_CUDA(tc_launch_gemm(p, (cudaStream_t)stream), "fused gemm+layernorm");
+  return ARLO_OK;
 }

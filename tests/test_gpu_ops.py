@@ -224,3 +224,25 @@ def test_attention_lazy_rescale_path(arlo_lib, dtype):
         xx = qkv[i * L:(i + 1) * L].astype(np.float64)
         ref = orc.attention(xx[:n, :H], xx[:n, H:2 * H], xx[:n, 2 * H:], heads)
         np.testing.assert_allclose(got[i, :n], ref, rtol=0, atol=tol)
+
+
+@pytest.mark.parametrize("M,N,K", [(4096, 768, 768), (333, 768, 3072), (64, 1024, 1024), (700, 1024, 4096),
+                                   (100, 128, 512), (2048, 768, 768)])
+def test_gemm_fused_layernorm(arlo_lib, M, N, K):
+    """Residual + LayerNorm fused into the GEMM epilogue (cluster row statistics)."""
+    A = rnd((M, K), 1)
+    W = rnd((N, K), 2, 0.02)
+    b = rnd((N,), 3, 0.02)
+    R = rnd((M, N), 4)
+    g = wl.round_to_bf16(rnd((N,), 5, 0.1) + 1)
+    be = rnd((N,), 6, 0.02)
+    ref = orc.layer_norm(orc.linear(A, W, b) + R, g, be, 1e-12)
+    out = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_gemm_ln(bf16_dev(A), bf16_dev(W), f32_dev(b), bf16_dev(R), f32_dev(g), f32_dev(be), 1e-12, out)
+    torch.cuda.synchronize()
+    np.testing.assert_allclose(host64(out), ref, rtol=0, atol=3e-2)
+    # in place (out aliases the residual), as the runtime uses it
+    Rd = bf16_dev(R)
+    arlo_lib.op_gemm_ln(bf16_dev(A), bf16_dev(W), f32_dev(b), Rd, f32_dev(g), f32_dev(be), 1e-12, Rd)
+    torch.cuda.synchronize()
+    assert torch.equal(Rd, out)

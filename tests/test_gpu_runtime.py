@@ -178,5 +178,5 @@ def test_enqueue_matches_infer(arlo_lib):
     rt.enqueue(12, torch.from_numpy(ids).cuda(), torch.from_numpy(lengths).cuda(), out)
     s.synchronize()
     np.testing.assert_array_equal(out.cpu().numpy(), a[:12])
-    assert rt.kernel_count(12) == 3 + 7 * cfg.layers
+    assert rt.kernel_count(12) in (3 + 5 * cfg.layers, 3 + 7 * cfg.layers)  # fused / unfused LayerNorm
     rt.close()
