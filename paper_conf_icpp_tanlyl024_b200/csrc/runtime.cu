@@ -246,10 +246,12 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
   const arlo_model_config& c = w->cfg;
   const int M = bk.b * rt->L, H = c.hidden, F = c.ffn;
   bk.plans.resize(c.layers);
-  // residual + LayerNorm fused into the out-proj / FFN2 GEMM epilogues when the
-  // hidden size splits into a cluster of <= 8 column tiles (all BERT configs)
+  // Residual + LayerNorm fused into the out-proj / FFN2 GEMM epilogues (cluster
+  // row statistics).  Opt-in (ARLO_FUSED_LN=1): measured slower than GEMM + LN
+  // kernel on B200 in round 1 (one tile per CTA leaves its three-pass epilogue
+  // exposed; small M runs on N/BN CTAs only), see DESIGN.md.
   TcGemmPlan probe;
-  bk.fused_ln = getenv("ARLO_NO_FUSED_LN") == nullptr &&
+  bk.fused_ln = getenv("ARLO_FUSED_LN") != nullptr &&
                 tc_plan_gemm_ln(&probe, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X,
                                 (const float*)w->lt(0, LN1_G), (const float*)w->lt(0, LN1_B), c.ln_eps, rt->X);
   for (int l = 0; l < c.layers; ++l) {
