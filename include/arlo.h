@@ -99,10 +99,10 @@ typedef struct arlo_runtime arlo_runtime;
  * "compiled into multiple runtimes, each with a different max_length"; the
  * static (batch, length) shape, L77 §2.1).  Requires 16 <= L <= max_pos,
  * L % 16 == 0, 1 <= max_batch <= 64.  Allocates the activation arena for
- * (max_batch, L) and captures one CUDA graph per batch bucket
- * b in {1, 2, 4, ..., max_batch} (max_batch itself included): embedding+LN,
+ * (max_batch, L) and captures one CUDA graph per batch bucket: embedding+LN,
  * layers x {QKV GEMM, masked attention, out-proj GEMM+residual, LN, FFN1
- * GEMM+GELU, FFN2 GEMM+residual, LN}, CLS pooler + classifier.
+ * GEMM+GELU, FFN2 GEMM+residual, LN}, CLS pooler + classifier.  Buckets are
+ * b in {1, 2, 4} then every multiple of 8 below max_batch, plus max_batch.
  * The runtime uses its own non-blocking stream until arlo_runtime_set_stream.
  * Errors: EINVAL, ENOMEM, ECUDA, ENODEV.
  */

@@ -81,41 +81,61 @@ struct TcCfg {
 // st.shared into a 64-byte-swizzled 32x32 staging tile, then one TMA bulk
 // tensor store of the tile (coalesced, asynchronous; rows >= M clipped by the
 // tensor map).  `release()` fires once the last TMEM load has completed.
+template <int BN>
+struct EpiShape {
+  static constexpr int COLS = BN / 2;            // columns per epilogue warp
+  static constexpr int CW = COLS >= 32 ? 32 : 16;  // chunk width: TMEM load / staging tile / TMA box
+  static constexpr int NC = COLS / CW;
+  static constexpr int SWZ = CW * 2;             // staging row bytes == TMA swizzle mode (64B / 32B)
+};
+
+template <int CW>
+__device__ __forceinline__ void tmem_ld_chunk(uint32_t taddr, uint32_t (&r)[CW]);
+template <>
+__device__ __forceinline__ void tmem_ld_chunk<32>(uint32_t taddr, uint32_t (&r)[32]) {
+  ptx::tmem_ld_32x32b_x32(taddr, r);
+}
+template <>
+__device__ __forceinline__ void tmem_ld_chunk<16>(uint32_t taddr, uint32_t (&r)[16]) {
+  ptx::tmem_ld_32x32b_x16(taddr, r);
+}
+
 template <int BN, int EPI, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int N, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
                                               uint8_t* stg, int& sc, Release release) {
-  constexpr int COLS = BN / 2;
-  constexpr int NC = COLS / 32;
+  using S = EpiShape<BN>;
+  constexpr int COLS = S::COLS, CW = S::CW, NC = S::NC;
+  constexpr int RV = CW / 8;  // 16-byte residual vectors per row per chunk
   const int row = row0 + lane;
   const bool row_ok = row < M;
   const int col0 = n0 + cg * COLS;
   const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
   const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
   const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16) + cg * COLS;
-  uint32_t r[2][32];
-  uint4 rv[2][4];
+  uint32_t r[2][CW];
+  uint4 rv[2][RV];
   if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-    for (int j = 0; j < 4; ++j) rv[0][j] = __ldg(res4 + j);
+    for (int j = 0; j < RV; ++j) rv[0][j] = __ldg(res4 + j);
   }
-  ptx::tmem_ld_32x32b_x32(t_row, r[0]);
+  tmem_ld_chunk<CW>(t_row, r[0]);
   ptx::tmem_wait_ld();
 #pragma unroll
   for (int c = 0; c < NC; ++c) {
     const int cur = c & 1, nxt = cur ^ 1;
     if (c + 1 < NC) {
-      ptx::tmem_ld_32x32b_x32(t_row + (c + 1) * 32, r[nxt]);
+      tmem_ld_chunk<CW>(t_row + (c + 1) * CW, r[nxt]);
       if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-        for (int j = 0; j < 4; ++j) rv[nxt][j] = __ldg(res4 + (c + 1) * 4 + j);
+        for (int j = 0; j < RV; ++j) rv[nxt][j] = __ldg(res4 + (c + 1) * RV + j);
       }
     }
-    uint32_t pk[16];
+    uint32_t pk[CW / 2];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      const float4 b4 = __ldg(bias4 + c * 8 + j);
+    for (int j = 0; j < CW / 4; ++j) {
+      const float4 b4 = __ldg(bias4 + c * (CW / 4) + j);
       float v0 = __uint_as_float(r[cur][4 * j + 0]) + b4.x;
       float v1 = __uint_as_float(r[cur][4 * j + 1]) + b4.y;
       float v2 = __uint_as_float(r[cur][4 * j + 2]) + b4.z;
@@ -138,15 +158,16 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       __syncwarp();
     }
 #pragma unroll
-    for (int j = 0; j < 4; ++j) {
-      const int sw = j ^ ((lane >> 1) & 3);  // SWIZZLE_64B: 16-byte chunk ^= address bits [7:8]
-      *reinterpret_cast<uint4*>(buf + lane * 64 + sw * 16) =
+    for (int j = 0; j < CW / 8; ++j) {
+      // TMA swizzle of a (CW*2)-byte row: 16-byte chunk index ^= address bits [7:8] (64B) / [7] (32B)
+      const int sw = CW == 32 ? (j ^ ((lane >> 1) & 3)) : (j ^ ((lane >> 2) & 1));
+      *reinterpret_cast<uint4*>(buf + lane * (CW * 2) + sw * 16) =
           make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
     }
     ptx::fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) {
-      ptx::tma_store_2d(tmC, buf, col0 + c * 32, row0);
+      ptx::tma_store_2d(tmC, buf, col0 + c * CW, row0);
       ptx::bulk_commit();
     }
     ++sc;
@@ -763,7 +784,7 @@ int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
   double best = 1e30;
   int best_bn = 0;
-  const int cands[7] = {-256, -192, 256, 192, -128, 128, 64};
+  const int cands[8] = {-256, -192, 256, 192, -128, 128, 64, 32};
   for (int c : cands) {
     const bool pair = c < 0;
     const int bn = pair ? -c : c;
@@ -773,7 +794,7 @@ int tc_choose_bn(int M, int N, int K) {
     const long slots = pair ? sms / 2 : sms;
     const long waves = (tiles + slots - 1) / slots;
     const double mma_us = (double)BM * bn * K * 2 / 8192.0 / 1.9e3;
-    double eff = bn >= 192 ? (pair ? 1.0 : 0.92) : (bn == 128 ? 0.68 : 0.5);
+    double eff = bn >= 192 ? (pair ? 1.0 : 0.92) : (bn == 128 ? 0.68 : (bn == 64 ? 0.5 : 0.3));
     const double t = waves * (mma_us / eff + 1.0);
     if (t < best * 0.999) { best = t; best_bn = c; }
   }
@@ -786,8 +807,8 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
   const bool pair = choice < 0;
   const int bn = pair ? -choice : choice;
-  if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
-  if (pair && bn == 64) return false;
+  if (bn != 32 && bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
+  if (pair && bn < 128) return false;
   if (N % bn) return false;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi; p->ln = false;
   p->bias = bias; p->resid = resid; p->out = out;
@@ -849,7 +870,8 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   p->grid = (num_m < clusters ? num_m : clusters) * nt;
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
-  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, 32, 32, 64)) return false;
+  const int cw = bn / 2 >= 32 ? 32 : 16;  // EpiShape<bn>::CW
+  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, cw, 32, cw * 2)) return false;
   return true;
 }
 
@@ -871,6 +893,7 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
     return cudaErrorInvalidValue;
   }
   switch (p.BN) {
+    case 32: return launch_bn<32, false>(p, s);
     case 64: return launch_bn<64, false>(p, s);
     case 128: return launch_bn<128, false>(p, s);
     case 192: return launch_bn<192, false>(p, s);

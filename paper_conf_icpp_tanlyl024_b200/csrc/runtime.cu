@@ -337,9 +337,11 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
   e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
   if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "pinned staging: %s", cudaGetErrorString(e)));
 
-  // batch buckets 1, 2, 4, ..., max_batch
+  // batch buckets 1, 2, 4, 8, then every multiple of 8, and max_batch: a partly
+  // filled batch pads to at most 7 (or b-1 below 8) empty slots
   std::vector<int> bs;
-  for (int b = 1; b < max_batch; b *= 2) bs.push_back(b);
+  for (int b = 1; b < max_batch && b < 8; b *= 2) bs.push_back(b);
+  for (int b = 8; b < max_batch; b += 8) bs.push_back(b);
   bs.push_back(max_batch);
   rt->buckets.resize(bs.size());
   for (size_t i = 0; i < bs.size(); ++i) {
