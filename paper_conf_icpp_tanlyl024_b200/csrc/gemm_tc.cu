@@ -784,7 +784,7 @@ int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
   double best = 1e30;
   int best_bn = 0;
-  const int cands[8] = {-256, -192, 256, 192, -128, 128, 64, 32};
+  const int cands[7] = {-256, -192, 256, 192, -128, 128, 64};
   for (int c : cands) {
     const bool pair = c < 0;
     const int bn = pair ? -c : c;
@@ -807,7 +807,7 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
   const bool pair = choice < 0;
   const int bn = pair ? -choice : choice;
-  if (bn != 32 && bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
+  if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn < 128) return false;
   if (N % bn) return false;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi; p->ln = false;
@@ -893,7 +893,6 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
     return cudaErrorInvalidValue;
   }
   switch (p.BN) {
-    case 32: return launch_bn<32, false>(p, s);
     case 64: return launch_bn<64, false>(p, s);
     case 128: return launch_bn<128, false>(p, s);
     case 192: return launch_bn<192, false>(p, s);

@@ -35,7 +35,7 @@ GEMM_SHAPES = [
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
 @pytest.mark.parametrize("epi", [0, 1, 2])
-@pytest.mark.parametrize("force", [0, 32, 128, -128, -256, 192, -192])
+@pytest.mark.parametrize("force", [0, 128, -128, -256, 192, -192])
 def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
     if N % abs(force or 64):
         pytest.skip("tile width does not divide N")
@@ -57,7 +57,7 @@ def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
     np.testing.assert_allclose(got, ref, rtol=8e-3, atol=8e-3)
 
 
-@pytest.mark.parametrize("bn", [32, 64, 128, 192, 256, -128, -192, -256])
+@pytest.mark.parametrize("bn", [64, 128, 192, 256, -128, -192, -256])
 def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
     """Row results do not depend on the tile width (cross-L invariance contract)."""
     M, N, K = 300, 768, 768
