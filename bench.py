@@ -294,6 +294,7 @@ def main():
         result["uniform_512"] = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
         result["e2e"] = e2e_res
         result["bert_large"] = bert_large_per_L(arlo, torch, dev, stream, local_rank)
+        result["trace_replay"] = trace_replay(arlo, torch, runtimes, cfg, stream, result)
         if not args.no_cpu_baseline:
             result["cpu_baseline"] = cpu_baseline()
     if rank == 0:
@@ -302,6 +303,21 @@ def main():
         rt.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def trace_replay(arlo, torch, runtimes, cfg, stream, result):
+    """Mean / p98 / p99 latency per length bucket under Poisson and MMPP arrivals at
+    70% of the measured saturation throughput, requests dispatched by Algorithm 1
+    (replay.py); SLO 150 ms for BERT-base."""
+    from paper_conf_icpp_tanlyl024_b200 import replay
+    per_L = {int(L): {int(b): v["median"] for b, v in row.items()} for L, row in result["per_L_latency_ms"].items()}
+    rate = 0.7 * result["value"] / max(1, result["n_gpus"])
+    out = {}
+    for bursty in (False, True):
+        out["bursty" if bursty else "stable"] = replay.replay(arlo, torch, runtimes, cfg, 20000, rate, bursty=bursty,
+                                                              slo_ms=150.0, max_batch=MAX_BATCH, per_L_ms=per_L,
+                                                              stream=stream)
+    return out
 
 
 def bert_large_per_L(arlo, torch, dev, stream, device_index):
