@@ -34,20 +34,22 @@ constexpr float kRescaleLog2 = 8.0f;
 // Launch shape per runtime length: NQ q-tiles per CTA, up to MAXKT 128-key
 // K/V tiles (L <= 128 * MAXKT).  NQ = 1 (L <= 128) keeps smem (80 KB) and TMEM
 // (256 columns) small enough for two CTAs per SM.
-template <int NQ_, int MAXKT_>
+template <int NQ_, int MAXKT_, int NS_>
 struct AttnCfg {
   static constexpr int NQ = NQ_;
+  static constexpr int NS = NS_;  // S (TMEM) and P (smem) slots per q-tile
   static constexpr int kMaxKT = MAXKT_;
   static constexpr int kKSlots = MAXKT_ < 2 ? MAXKT_ : 2;  // K tiles ring; V stays resident
   static constexpr int kSoftWarps = 4 * NQ;   // warp w: q-tile w/4, TMEM lane quarter w%4
   static constexpr int kProdWarp = kSoftWarps;
   static constexpr int kMmaWarp = kSoftWarps + 1;
   static constexpr int kThreads = 32 * (kSoftWarps + 2);
-  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + NQ * 2 * kPBytes + 256;
-  // TMEM columns: q-tile qi: S slots at qi*128 + {0, 64}, O at NQ*128 + qi*64
-  static constexpr uint32_t kOCol = NQ * 128;
-  static constexpr uint32_t kTmemCols = NQ == 1 ? 256 : 512;
-  static constexpr int kMinBlocks = NQ == 1 ? 2 : 1;
+  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + NQ * NS * kPBytes + 256;
+  // TMEM columns: q-tile qi: S slots at qi*NS*64 + slot*64, O at NQ*NS*64 + qi*64
+  static constexpr uint32_t kOCol = NQ * NS * KC;
+  static constexpr uint32_t kUsedCols = NQ * (NS * KC + 64);
+  static constexpr uint32_t kTmemCols = kUsedCols <= 128 ? 128 : kUsedCols <= 256 ? 256 : 512;
+  static constexpr int kMinBlocks = (NQ == 1 && NS == 1) ? 3 : (NQ == 1 ? 2 : 1);
   static_assert(kSmem * kMinBlocks <= 232448, "attention smem");
 };
 
@@ -79,11 +81,12 @@ __device__ __forceinline__ void atrace(int slot) {
 // in by TMA once per CTA and are shared by both q-tiles.  Key chunks starting
 // at >= len are never loaded or multiplied; keys >= len inside the last chunk
 // get p = 0.
-template <int NQ_, int MAXKT_, bool TRACE>
-__global__ void __launch_bounds__(AttnCfg<NQ_, MAXKT_>::kThreads, AttnCfg<NQ_, MAXKT_>::kMinBlocks)
+template <int NQ_, int MAXKT_, int NS_, bool TRACE>
+__global__ void __launch_bounds__(AttnCfg<NQ_, MAXKT_, NS_>::kThreads, AttnCfg<NQ_, MAXKT_, NS_>::kMinBlocks)
 attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const int32_t* __restrict__ lengths,
                bf16* __restrict__ o) {
-  using Cfg = AttnCfg<NQ_, MAXKT_>;
+  using Cfg = AttnCfg<NQ_, MAXKT_, NS_>;
+  constexpr int NS = Cfg::NS;
   constexpr int NQ = Cfg::NQ, kMaxKT = Cfg::kMaxKT, kKSlots = Cfg::kKSlots;
   constexpr int kSoftWarps = Cfg::kSoftWarps, kProdWarp = Cfg::kProdWarp, kMmaWarp = Cfg::kMmaWarp;
   constexpr int kAttnThreads = Cfg::kThreads;
@@ -113,14 +116,14 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   uint8_t* sK = sQ + NQ * kTileBytes;
   uint8_t* sV = sK + kKSlots * kTileBytes;
   uint8_t* sP = sV + kMaxKT * kTileBytes;  // [NQ][2][128 x 64 bf16]
-  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * 2 * kPBytes);
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * NS * kPBytes);
   uint64_t* bar_v = bar_k + kMaxKT;
   uint64_t* k_free = bar_v + kMaxKT;
   uint64_t* s_full = k_free + kKSlots;  // [NQ][2]
-  uint64_t* s_free = s_full + 2 * NQ;
-  uint64_t* p_full = s_free + 2 * NQ;
-  uint64_t* pv_done = p_full + 2 * NQ;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + 2 * NQ);
+  uint64_t* s_free = s_full + NS * NQ;
+  uint64_t* p_full = s_free + NS * NQ;
+  uint64_t* pv_done = p_full + NS * NQ;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(pv_done + NS * NQ);
 
   if (warp == kProdWarp && lane == 0) {
     ptx::tma_prefetch_desc(&tm);
@@ -129,7 +132,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       ptx::mbar_init(&bar_v[j], 1);
     }
     for (int i = 0; i < kKSlots; ++i) ptx::mbar_init(&k_free[i], 1);
-    for (int i = 0; i < 2 * NQ; ++i) {
+    for (int i = 0; i < NS * NQ; ++i) {
       ptx::mbar_init(&s_full[i], 1);
       ptx::mbar_init(&s_free[i], 4);
       ptx::mbar_init(&p_full[i], 4);
@@ -171,30 +174,30 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
       constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
       auto issue_s = [&](int qi, int c) {
-        const int t = c >> 1, sl = c & 1;
-        if (c >= 2) ptx::mbar_wait(&s_free[qi * 2 + sl], ((c - 2) >> 1) & 1);
+        const int t = c >> 1, sl = c % NS;
+        if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
         ptx::mbar_wait(&bar_k[t], 0);
         ptx::tc_fence_after();
         const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
         const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
         for (int k = 0; k < D / 16; ++k)
-          ptx::mma_bf16_ss(tmem + qi * 128 + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
+          ptx::mma_bf16_ss(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
                            ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
-        ptx::mma_commit(&s_full[qi * 2 + sl]);
+        ptx::mma_commit(&s_full[qi * NS + sl]);
       };
       auto issue_pv = [&](int qi, int c) {
-        const int t = c >> 1, sl = c & 1;
-        ptx::mbar_wait(&p_full[qi * 2 + sl], (c >> 1) & 1);
+        const int t = c >> 1, sl = c % NS;
+        ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
         ptx::mbar_wait(&bar_v[t], 0);
         ptx::tc_fence_after();
-        const uint32_t p_addr = ptx::smem_u32(sP + (qi * 2 + sl) * kPBytes);
+        const uint32_t p_addr = ptx::smem_u32(sP + (qi * NS + sl) * kPBytes);
         const uint32_t v_addr = ptx::smem_u32(sV + t * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
         for (int ks = 0; ks < KC / 16; ++ks)
           ptx::mma_bf16_ss(tmem + kOCol + qi * D, ptx::desc_k_sw128(p_addr + ks * 32),
                            ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (c | ks) != 0);
-        ptx::mma_commit(&pv_done[qi * 2 + sl]);
+        ptx::mma_commit(&pv_done[qi * NS + sl]);
       };
       for (int c = 0; c < n_ch; ++c) {
         for (int qi = 0; qi < nq; ++qi) issue_s(qi, c);
@@ -212,17 +215,17 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     const int qrow = q0 + qi * AQ + r;
     if (qi < nq) {
       const uint32_t t_lane = tmem + ((uint32_t)(quarter * 32) << 16);
-      const uint32_t t_s = t_lane + qi * 128;
+      const uint32_t t_s = t_lane + qi * NS * KC;
       const uint32_t t_o = t_lane + kOCol + qi * D;
       const float c2 = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
       float m = -INFINITY, l = 0.f;
 #pragma unroll 1
       for (int c = 0; c < n_ch; ++c) {
-        const int cur = c & 1;
+        const int cur = c % NS;
         // pull S chunk c out of TMEM and hand the slot back to the MMA warp
         // (S(c+2) then overlaps this chunk's exp2 work; the other q-tile's warps
         // on the same SM sub-partitions overlap this warp's TMEM-load latency)
-        ptx::mbar_wait(&s_full[qi * 2 + cur], (c >> 1) & 1);
+        ptx::mbar_wait(&s_full[qi * NS + cur], (c / NS) & 1);
         ptx::tc_fence_after();
         if (warp == 0 && lane == 0) atrace<TRACE>(3 + 3 * (c & 7));
         uint32_t vc[KC];
@@ -231,7 +234,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         ptx::tmem_wait_ld();
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&s_free[qi * 2 + cur]);
+        if (lane == 0) ptx::mbar_arrive(&s_free[qi * NS + cur]);
         const int kbase = c * KC;
         const bool full = kbase + KC <= len;
         float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
@@ -250,7 +253,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
             l *= alpha;
             m = cmax;
           }
-          ptx::mbar_wait(&pv_done[qi * 2 + ((c - 1) & 1)], ((c - 1) >> 1) & 1);  // O holds PV_0..c-1
+          ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);  // O holds PV_0..c-1
           ptx::tc_fence_after();
 #pragma unroll 1
           for (int hh = 0; hh < 4; ++hh) {
@@ -265,9 +268,9 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
         // P slot `cur` was read by PV(c-2)
-        if (c >= 2) ptx::mbar_wait(&pv_done[qi * 2 + cur], ((c - 2) >> 1) & 1);
+        if (c >= NS) ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
         const float mc = m * c2;
-        uint8_t* prow = sP + (qi * 2 + cur) * kPBytes + r * 128;
+        uint8_t* prow = sP + (qi * NS + cur) * kPBytes + r * 128;
         float ls[2] = {0.f, 0.f};
 #pragma unroll
         for (int ch = 0; ch < 2; ++ch) {
@@ -296,11 +299,11 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         ptx::fence_proxy_async_smem();
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&p_full[qi * 2 + cur]);
+        if (lane == 0) ptx::mbar_arrive(&p_full[qi * NS + cur]);
         if (warp == 0 && lane == 0) atrace<TRACE>(5 + 3 * (c & 7));
       }
       // O = (sum_c P_c V_c) / l
-      ptx::mbar_wait(&pv_done[qi * 2 + ((n_ch - 1) & 1)], ((n_ch - 1) >> 1) & 1);
+      ptx::mbar_wait(&pv_done[qi * NS + ((n_ch - 1) % NS)], ((n_ch - 1) / NS) & 1);
       ptx::tc_fence_after();
       const float inv = 1.f / l;
       uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
@@ -381,24 +384,24 @@ int set_attn_trace(unsigned long long* buf) {
   return (int)cudaMemcpyToSymbol(g_atrace, &buf, sizeof(buf));
 }
 
-template <int NQ, int MAXKT>
+template <int NQ, int MAXKT, int NS>
 cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
-  using Cfg = AttnCfg<NQ, MAXKT>;
+  using Cfg = AttnCfg<NQ, MAXKT, NS>;
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, false>,
+    cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, false>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
     if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+      e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                Cfg::kSmem);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
   if (g_attn_trace_on)
-    return launch_k(attn_tc_kernel<NQ, MAXKT, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
+    return launch_k(attn_tc_kernel<NQ, MAXKT, NS, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
                     lengths, (bf16*)o);
-  return launch_k(attn_tc_kernel<NQ, MAXKT, false>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
+  return launch_k(attn_tc_kernel<NQ, MAXKT, NS, false>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
                   lengths, (bf16*)o);
 }
 
@@ -412,9 +415,9 @@ bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) 
 cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
   if (p.B <= 0 || p.L <= 0) return cudaSuccess;
   if (p.dt == DT_BF16) {
-    if (p.L <= 128) return attn_launch_cfg<1, 1>(p, lengths, o, s);
-    if (p.L <= 256) return attn_launch_cfg<2, 2>(p, lengths, o, s);
-    return attn_launch_cfg<2, 4>(p, lengths, o, s);
+    if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
+    if (p.L <= 256) return attn_launch_cfg<2, 2, 2>(p, lengths, o, s);
+    return attn_launch_cfg<2, 4, 2>(p, lengths, o, s);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
     attn_f32_kernel<<<(unsigned)((warps + 3) / 4), 128, 0, s>>>(p.B, p.L, p.heads, (const float*)p.qkv, lengths,
