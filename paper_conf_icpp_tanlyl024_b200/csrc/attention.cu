@@ -19,6 +19,8 @@
 #include "kernels.h"
 #include "ptx.cuh"
 
+#include <cstdlib>
+
 namespace arlo {
 namespace {
 
@@ -108,7 +110,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   }
   const int n_kt = (len + AK - 1) / AK;  // K/V tiles
   const int n_ch = (len + KC - 1) / KC;  // 64-key chunks
-  const int nq = (NQ == 2 && q0 + AQ < len) ? 2 : 1;  // live q-tiles (the second may be wholly padded)
+  int nq = 1;  // live q-tiles (trailing ones may be wholly padded)
+  while (nq < NQ && q0 + nq * AQ < len) ++nq;
 
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -219,87 +222,123 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       const uint32_t t_o = t_lane + kOCol + qi * D;
       const float c2 = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
       float m = -INFINITY, l = 0.f;
+      // 16 keys of chunk c: p = 2^(s*c2 - mc) (0 past len), fp32 partial sum,
+      // running max of p, bf16 pack into the row's two 16-byte P chunks
+      auto exp_piece = [&](const uint32_t (&v)[16], int k, float mc, bool full, int kbase, uint8_t* prow, float& ls,
+                           float& pmax) {
+        uint32_t pk[8];
+#pragma unroll
+        for (int e = 0; e < 16; e += 2) {
+          float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c2, -mc));
+          float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c2, -mc));
+          if (!full) {
+            if (kbase + k * 16 + e >= len) p0 = 0.f;
+            if (kbase + k * 16 + e + 1 >= len) p1 = 0.f;
+          }
+          ls += p0 + p1;
+          pmax = fmaxf(pmax, fmaxf(p0, p1));
+          pk[e >> 1] = pack_bf16x2(p0, p1);
+        }
+#pragma unroll
+        for (int i = 0; i < 2; ++i) {
+          const int chunk16 = k * 2 + i;
+          *reinterpret_cast<uint4*>(prow + ((chunk16 ^ (r & 7)) << 4)) =
+              make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
+        }
+      };
+      // all 64 keys of chunk c against a given max (S re-read from TMEM, pieces double-buffered)
+      auto exp_chunk = [&](uint32_t t_chunk, float mc, bool full, int kbase, uint8_t* prow, float& ls, float& pmax) {
+        uint32_t va[16], vb[16];
+        ptx::tmem_ld_32x32b_x16(t_chunk, va);
+        ptx::tmem_wait_ld();
+        ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);  // in flight while piece 0 is computed
+        exp_piece(va, 0, mc, full, kbase, prow, ls, pmax);
+        ptx::tmem_wait_ld();
+        ptx::tmem_ld_32x32b_x16(t_chunk + 32, va);
+        exp_piece(vb, 1, mc, full, kbase, prow, ls, pmax);
+        ptx::tmem_wait_ld();
+        ptx::tmem_ld_32x32b_x16(t_chunk + 48, vb);
+        exp_piece(va, 2, mc, full, kbase, prow, ls, pmax);
+        ptx::tmem_wait_ld();
+        exp_piece(vb, 3, mc, full, kbase, prow, ls, pmax);
+      };
 #pragma unroll 1
       for (int c = 0; c < n_ch; ++c) {
         const int cur = c % NS;
-        // pull S chunk c out of TMEM and hand the slot back to the MMA warp
-        // (S(c+2) then overlaps this chunk's exp2 work; the other q-tile's warps
-        // on the same SM sub-partitions overlap this warp's TMEM-load latency)
         ptx::mbar_wait(&s_full[qi * NS + cur], (c / NS) & 1);
         ptx::tc_fence_after();
         if (warp == 0 && lane == 0) atrace<TRACE>(3 + 3 * (c & 7));
-        uint32_t vc[KC];
-        ptx::tmem_ld_32x32b_x32(t_s + cur * KC, *reinterpret_cast<uint32_t(*)[32]>(&vc[0]));
-        ptx::tmem_ld_32x32b_x32(t_s + cur * KC + 32, *reinterpret_cast<uint32_t(*)[32]>(&vc[32]));
-        ptx::tmem_wait_ld();
-        ptx::tc_fence_before();
-        __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&s_free[qi * NS + cur]);
         const int kbase = c * KC;
         const bool full = kbase + KC <= len;
-        float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-#pragma unroll
-        for (int e = 0; e < KC; ++e)
-          if (full || kbase + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vc[e]));
-        const float cmax = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+        const uint32_t t_chunk = t_s + cur * KC;
+        uint8_t* prow = sP + (qi * NS + cur) * kPBytes + r * 128;
+        // P slot `cur` was read by PV(c - NS)
+        if (c >= NS) ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
+        float ls = 0.f, pmax = 0.f;
         if (c == 0) {
-          m = cmax;
-        } else if (__any_sync(0xffffffffu, (cmax - m) * c2 > kRescaleLog2)) {
-          // warp-uniform branch (tcgen05.ld/st are warp-collective): rows whose
-          // max rose by > 2^8 rescale O and l, the others multiply by 1
-          float alpha = 1.f;
-          if ((cmax - m) * c2 > kRescaleLog2) {
-            alpha = ex2_approx((m - cmax) * c2);
-            l *= alpha;
-            m = cmax;
-          }
-          ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);  // O holds PV_0..c-1
-          ptx::tc_fence_after();
-#pragma unroll 1
-          for (int hh = 0; hh < 4; ++hh) {
-            uint32_t ov[16];
-            ptx::tmem_ld_32x32b_x16(t_o + hh * 16, ov);
+          // first chunk: row max from a first pass over S
+          float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+          for (int k = 0; k < 4; ++k) {
+            uint32_t v[16];
+            ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
             ptx::tmem_wait_ld();
 #pragma unroll
-            for (int e = 0; e < 16; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
-            ptx::tmem_st_32x32b_x16(t_o + hh * 16, ov);
+            for (int e = 0; e < 16; ++e)
+              if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
           }
-          ptx::tmem_wait_st();
+          m = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+          exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
+        } else {
+          // single streaming pass against the (possibly stale) running max: exact
+          // as long as no p exceeds 2^8; otherwise redo the chunk with its max
+          exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
+          if (__any_sync(0xffffffffu, pmax > 256.0f)) {
+            float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+            for (int k = 0; k < 4; ++k) {
+              uint32_t v[16];
+              ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
+              ptx::tmem_wait_ld();
+#pragma unroll
+              for (int e = 0; e < 16; ++e)
+                if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
+            }
+            const float cmax = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+            float alpha = 1.f;
+            if (pmax > 256.0f) {  // this row's max rose by > 2^8: rescale O and l
+              alpha = ex2_approx((m - cmax) * c2);
+              l *= alpha;
+              m = cmax;
+            }
+            // O holds PV_0..c-1 (warp-collective TMEM traffic: every row takes part)
+            ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);
+            ptx::tc_fence_after();
+#pragma unroll 1
+            for (int hh = 0; hh < 4; ++hh) {
+              uint32_t ov[16];
+              ptx::tmem_ld_32x32b_x16(t_o + hh * 16, ov);
+              ptx::tmem_wait_ld();
+#pragma unroll
+              for (int e = 0; e < 16; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
+              ptx::tmem_st_32x32b_x16(t_o + hh * 16, ov);
+            }
+            ptx::tmem_wait_st();
+            ls = 0.f;
+            pmax = 0.f;
+            exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
+          }
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
-        // P slot `cur` was read by PV(c-2)
-        if (c >= NS) ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
-        const float mc = m * c2;
-        uint8_t* prow = sP + (qi * NS + cur) * kPBytes + r * 128;
-        float ls[2] = {0.f, 0.f};
-#pragma unroll
-        for (int ch = 0; ch < 2; ++ch) {
-          uint32_t pk[16];
-#pragma unroll
-          for (int e = 0; e < 32; e += 2) {
-            const int k = ch * 32 + e;
-            float p0 = ex2_approx(fmaf(__uint_as_float(vc[k]), c2, -mc));
-            float p1 = ex2_approx(fmaf(__uint_as_float(vc[k + 1]), c2, -mc));
-            if (!full) {
-              if (kbase + k >= len) p0 = 0.f;
-              if (kbase + k + 1 >= len) p1 = 0.f;
-            }
-            ls[0] += p0;
-            ls[1] += p1;
-            pk[e >> 1] = pack_bf16x2(p0, p1);
-          }
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            const int chunk16 = ch * 4 + i;
-            *reinterpret_cast<uint4*>(prow + ((chunk16 ^ (r & 7)) << 4)) =
-                make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
-          }
-        }
-        l += ls[0] + ls[1];
+        l += ls;
+        // S slot back to the MMA warp, P chunk to the PV MMA
         ptx::fence_proxy_async_smem();
         ptx::tc_fence_before();
         __syncwarp();
-        if (lane == 0) ptx::mbar_arrive(&p_full[qi * NS + cur]);
+        if (lane == 0) {
+          ptx::mbar_arrive(&s_free[qi * NS + cur]);
+          ptx::mbar_arrive(&p_full[qi * NS + cur]);
+        }
         if (warp == 0 && lane == 0) atrace<TRACE>(5 + 3 * (c & 7));
       }
       // O = (sum_c P_c V_c) / l
@@ -417,6 +456,7 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
   if (p.dt == DT_BF16) {
     if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
     if (p.L <= 256) return attn_launch_cfg<2, 2, 2>(p, lengths, o, s);
+    if (getenv("ARLO_ATTN_NQ4")) return attn_launch_cfg<4, 4, 1>(p, lengths, o, s);
     return attn_launch_cfg<2, 4, 2>(p, lengths, o, s);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
