@@ -86,7 +86,7 @@ int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K);
  * %globaltimer stamps of their pipeline events into it; NULL turns it off.
  */
 int arlo_debug_gemm_trace(void* buf);
-/* Same for the bf16 attention kernel: >= 32 * 2048 uint64 entries. */
+/* Same for the bf16 attention kernel: >= 64 * 2048 uint64 entries. */
 int arlo_debug_attn_trace(void* buf);
 
 #ifdef __cplusplus

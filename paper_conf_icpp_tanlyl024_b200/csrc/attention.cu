@@ -19,7 +19,7 @@
 #include "kernels.h"
 #include "ptx.cuh"
 
-#include <cstdlib>
+#include <type_traits>
 
 namespace arlo {
 namespace {
@@ -29,43 +29,50 @@ constexpr int AQ = 128;      // queries per q-tile (TMEM lanes)
 constexpr int AK = 128;      // keys per K/V tile (TMA unit)
 constexpr int KC = 64;       // keys per softmax chunk (S MMA N)
 constexpr int kTileBytes = 128 * 128;         // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
-constexpr int kPBytes = 128 * 128;            // P chunk: 128 queries x 64 keys (one K-block)
-// lazy rescale: keep a stale row max unless a chunk's max exceeds it by > 2^8 in p
-constexpr float kRescaleLog2 = 8.0f;
 
 // Launch shape per runtime length: NQ q-tiles per CTA, up to MAXKT 128-key
-// K/V tiles (L <= 128 * MAXKT).  NQ = 1 (L <= 128) keeps smem (80 KB) and TMEM
-// (256 columns) small enough for two CTAs per SM.
+// K/V tiles (L <= 128 * MAXKT), NS S/P slots per q-tile.  NQ = 1 (L <= 128)
+// keeps smem (48 KB) and TMEM (256 columns) small enough for two CTAs per SM.
 template <int NQ_, int MAXKT_, int NS_>
 struct AttnCfg {
   static constexpr int NQ = NQ_;
-  static constexpr int NS = NS_;  // S (TMEM) and P (smem) slots per q-tile
+  static constexpr int NS = NS_;  // S and P (TMEM) slots per q-tile
   static constexpr int kMaxKT = MAXKT_;
   static constexpr int kKSlots = MAXKT_ < 2 ? MAXKT_ : 2;  // K tiles ring; V stays resident
   static constexpr int kSoftWarps = 4 * NQ;   // warp w: q-tile w/4, TMEM lane quarter w%4
   static constexpr int kProdWarp = kSoftWarps;
   static constexpr int kMmaWarp = kSoftWarps + 1;
   static constexpr int kThreads = 32 * (kSoftWarps + 2);
-  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + NQ * NS * kPBytes + 256;
-  // TMEM columns: q-tile qi: S slots at qi*NS*64 + slot*64, O at NQ*NS*64 + qi*64
+  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + 256;
+  // TMEM columns, q-tile qi: S slot sl (64 fp32) at qi*NS*64 + sl*64; O (64 fp32)
+  // at kOCol + qi*64; P slot sl (64 bf16 packed in 32 columns) at kPCol + (qi*NS + sl)*32
   static constexpr uint32_t kOCol = NQ * NS * KC;
-  static constexpr uint32_t kUsedCols = NQ * (NS * KC + 64);
+  static constexpr uint32_t kPCol = kOCol + NQ * D;
+  static constexpr uint32_t kUsedCols = NQ * (NS * KC + D + NS * KC / 2);
   static constexpr uint32_t kTmemCols = kUsedCols <= 128 ? 128 : kUsedCols <= 256 ? 256 : 512;
-  static constexpr int kMinBlocks = (NQ == 1 && NS == 1) ? 3 : (NQ == 1 ? 2 : 1);
+  static_assert(kUsedCols <= 512, "attention TMEM");
+  static constexpr int kMinBlocks = 512 / kTmemCols < 2 ? 1 : 2;
   static_assert(kSmem * kMinBlocks <= 232448, "attention smem");
 };
 
 // Profiling hook (arlo_debug_attn_trace): the TRACE=true instantiation writes
-// %globaltimer stamps of the first 2048 CTAs into g_atrace[cta * 32 + slot].
+// Timeline of the first 2048 CTAs into g_atrace[cta * 64 + slot]: slots 0/1 are
+// %globaltimer at start/end (cross-SM), 62/63 clock64 at start/end (to convert),
+// every other slot is clock64 (cycle resolution within the SM).
 __device__ unsigned long long* g_atrace = nullptr;
 template <bool TRACE>
 __device__ __forceinline__ void atrace(int slot) {
   if (TRACE) {
     const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-    if (cta < 2048 && slot < 32) {
+    if (cta < 2048 && slot < 64) {
       unsigned long long t;
-      asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
-      g_atrace[cta * 32 + slot] = t;
+      if (slot < 2) {
+        asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+        g_atrace[cta * 64 + 62 + slot] = clock64();
+      } else {
+        t = clock64();
+      }
+      g_atrace[cta * 64 + slot] = t;
     }
   }
 }
@@ -77,8 +84,9 @@ __device__ __forceinline__ void atrace(int slot) {
 // at head dim 64 the TMEM->RF reads of S and the exp2 (MUFU) work, not the
 // tensor pipe, bound attention.  A lazily-rescaled
 // running max is kept (O rescaled in TMEM only when a chunk raises a row max
-// by > 2^8 in p); P is written as bf16 into a 128B-swizzled smem K-block (the
-// PV MMA's A operand).  S slots are double-buffered so S(c+1) is computed
+// enough that its p sum passes 2^8); P is written as packed bf16 back into
+// TMEM (tcgen05.st) and read from there as the PV MMA's A operand, so P never
+// touches shared memory.  S/P slots are double-buffered so S(c+1) is computed
 // while chunk c is in the exp stage.  Q, K (2-tile ring) and V (resident, <= 4 tiles) come
 // in by TMA once per CTA and are shared by both q-tiles.  Key chunks starting
 // at >= len are never loaded or multiplied; keys >= len inside the last chunk
@@ -92,7 +100,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   constexpr int NQ = Cfg::NQ, kMaxKT = Cfg::kMaxKT, kKSlots = Cfg::kKSlots;
   constexpr int kSoftWarps = Cfg::kSoftWarps, kProdWarp = Cfg::kProdWarp, kMmaWarp = Cfg::kMmaWarp;
   constexpr int kAttnThreads = Cfg::kThreads;
-  constexpr uint32_t kOCol = Cfg::kOCol, kTmemCols = Cfg::kTmemCols;
+  constexpr uint32_t kOCol = Cfg::kOCol, kPCol = Cfg::kPCol, kTmemCols = Cfg::kTmemCols;
   pdl_begin();
   const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
@@ -118,8 +126,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + NQ * kTileBytes;
   uint8_t* sV = sK + kKSlots * kTileBytes;
-  uint8_t* sP = sV + kMaxKT * kTileBytes;  // [NQ][2][128 x 64 bf16]
-  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sP + NQ * NS * kPBytes);
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sV + kMaxKT * kTileBytes);
   uint64_t* bar_v = bar_k + kMaxKT;
   uint64_t* k_free = bar_v + kMaxKT;
   uint64_t* s_full = k_free + kKSlots;  // [NQ][2]
@@ -176,11 +183,11 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     if (lane == 0) {
       constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
       constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
+      // Event loop: each q-tile advances independently (no head-of-line blocking
+      // on the slower one); an S MMA is issued as soon as its TMEM slot is free
+      // and its K tile has landed, a PV MMA as soon as its P chunk is written.
       auto issue_s = [&](int qi, int c) {
         const int t = c >> 1, sl = c % NS;
-        if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
-        ptx::mbar_wait(&bar_k[t], 0);
-        ptx::tc_fence_after();
         const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
         const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
@@ -188,28 +195,72 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::mma_bf16_ss(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
                            ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
         ptx::mma_commit(&s_full[qi * NS + sl]);
+        if (qi == 0 && c < 16) atrace<TRACE>(32 + c);  // S(0, c) issued
       };
       auto issue_pv = [&](int qi, int c) {
         const int t = c >> 1, sl = c % NS;
-        ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
-        ptx::mbar_wait(&bar_v[t], 0);
-        ptx::tc_fence_after();
-        const uint32_t p_addr = ptx::smem_u32(sP + (qi * NS + sl) * kPBytes);
+        const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
         const uint32_t v_addr = ptx::smem_u32(sV + t * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
-        for (int ks = 0; ks < KC / 16; ++ks)
-          ptx::mma_bf16_ss(tmem + kOCol + qi * D, ptx::desc_k_sw128(p_addr + ks * 32),
-                           ptx::desc_mn_sw128(v_addr + ks * 2048, 0), idesc_pv, (c | ks) != 0);
+        for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
+          ptx::mma_bf16_ts(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
+                           idesc_pv, (c | ks) != 0);
         ptx::mma_commit(&pv_done[qi * NS + sl]);
+        // (slots 48..55: MMA loop iteration of S(0, c))
       };
-      for (int c = 0; c < n_ch; ++c) {
-        for (int qi = 0; qi < nq; ++qi) issue_s(qi, c);
-        if ((c & 1) || c == n_ch - 1) ptx::mma_commit(&k_free[(c >> 1) & 1]);  // K tile c/2 fully used
-        if (c == 0) atrace<TRACE>(2);
-        if (c >= 1)
-          for (int qi = 0; qi < nq; ++qi) issue_pv(qi, c - 1);
+      int s_next[NQ], pv_next[NQ];
+#pragma unroll
+      for (int qi = 0; qi < NQ; ++qi) s_next[qi] = pv_next[qi] = 0;
+      int k_done = 0;  // K tiles whose S MMAs have all been issued (k_free committed)
+      int pv_left = nq * n_ch;
+      int iter = 0;
+      long long it_clk[4] = {0, 0, 0, 0};
+      while (pv_left > 0) {
+        if (TRACE && iter >= 8 && iter < 12) it_clk[iter - 8] = clock64();  // MMA event-loop iterations 8..11
+        ++iter;
+#pragma unroll
+        for (int qi = 0; qi < NQ; ++qi) {
+          if (qi >= nq) continue;
+          const int cs = s_next[qi];
+          if (cs < n_ch && (cs < NS || ptx::mbar_test(&s_free[qi * NS + cs % NS], ((cs - NS) / NS) & 1)) &&
+              ptx::mbar_test(&bar_k[cs >> 1], 0)) {
+            ptx::tc_fence_after();
+            if (TRACE && cs == 3) atrace<TRACE>(56 + 2 * qi);  // before S(qi, 3) issue
+            issue_s(qi, cs);
+            if (TRACE && cs == 3) atrace<TRACE>(57 + 2 * qi);  // after
+            if (TRACE && qi == 0 && cs < 8) {
+              const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+              if (cta < 2048) g_atrace[cta * 64 + 48 + cs] = iter;  // loop iteration that issued S(0,cs)
+            }
+            s_next[qi] = cs + 1;
+          }
+          const int cp = pv_next[qi];
+          if (cp < s_next[qi] && ptx::mbar_test(&p_full[qi * NS + cp % NS], (cp / NS) & 1) &&
+              ptx::mbar_test(&bar_v[cp >> 1], 0)) {
+            ptx::tc_fence_after();
+            if (TRACE && cp == 2 && qi == 0) atrace<TRACE>(60);  // before PV(0, 2) issue
+            issue_pv(qi, cp);
+            if (TRACE && cp == 2 && qi == 0) atrace<TRACE>(61);
+            pv_next[qi] = cp + 1;
+            --pv_left;
+          }
+        }
+        // a K tile is free once every live q-tile has issued the S MMAs of both its chunks
+        int smin = n_ch;
+#pragma unroll
+        for (int qi = 0; qi < NQ; ++qi)
+          if (qi < nq) smin = min(smin, s_next[qi]);
+        const int tiles_done = (smin == n_ch) ? n_kt : (smin >> 1);
+        while (k_done < tiles_done) {
+          ptx::mma_commit(&k_free[k_done & 1]);
+          ++k_done;
+        }
       }
-      for (int qi = 0; qi < nq; ++qi) issue_pv(qi, n_ch - 1);
+      if (TRACE) {
+        const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
+        if (cta < 2048)
+          for (int i = 0; i < 4; ++i) g_atrace[cta * 64 + 27 + i] = it_clk[i];
+      }
     }
   } else {
     // ----------------------------------------------------------------- softmax
@@ -222,45 +273,62 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       const uint32_t t_o = t_lane + kOCol + qi * D;
       const float c2 = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
       float m = -INFINITY, l = 0.f;
-      // 16 keys of chunk c: p = 2^(s*c2 - mc) (0 past len), fp32 partial sum,
-      // running max of p, bf16 pack into the row's two 16-byte P chunks
-      auto exp_piece = [&](const uint32_t (&v)[16], int k, float mc, bool full, int kbase, uint8_t* prow, float& ls,
-                           float& pmax) {
+      // 16 keys of chunk c: p = 2^(s*c2 - mc) (0 past len when MASK), fp32 partial
+      // sums, packed bf16 into the row's 8 TMEM P columns for these keys.  MASK is
+      // a compile-time flag: only a chunk straddling len pays for masking.
+      auto exp_piece = [&](auto mask_tag, const uint32_t (&v)[16], int k, float mc, int kbase, uint32_t t_p,
+                           float (&ls)[2]) {
+        constexpr bool MASK = decltype(mask_tag)::value;
         uint32_t pk[8];
 #pragma unroll
         for (int e = 0; e < 16; e += 2) {
           float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c2, -mc));
           float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c2, -mc));
-          if (!full) {
+          if (MASK) {
             if (kbase + k * 16 + e >= len) p0 = 0.f;
             if (kbase + k * 16 + e + 1 >= len) p1 = 0.f;
           }
-          ls += p0 + p1;
-          pmax = fmaxf(pmax, fmaxf(p0, p1));
+          ls[0] += p0;
+          ls[1] += p1;
           pk[e >> 1] = pack_bf16x2(p0, p1);
         }
-#pragma unroll
-        for (int i = 0; i < 2; ++i) {
-          const int chunk16 = k * 2 + i;
-          *reinterpret_cast<uint4*>(prow + ((chunk16 ^ (r & 7)) << 4)) =
-              make_uint4(pk[4 * i], pk[4 * i + 1], pk[4 * i + 2], pk[4 * i + 3]);
-        }
+        ptx::tmem_st_32x32b_x8(t_p + k * 8, pk);
       };
-      // all 64 keys of chunk c against a given max (S re-read from TMEM, pieces double-buffered)
-      auto exp_chunk = [&](uint32_t t_chunk, float mc, bool full, int kbase, uint8_t* prow, float& ls, float& pmax) {
+      // all 64 keys of chunk c against a given max (S pieces double-buffered); returns the p sum
+      auto exp_chunk = [&](auto mask_tag, uint32_t t_chunk, float mc, int kbase, uint32_t t_p) {
+        float ls[2] = {0.f, 0.f};
         uint32_t va[16], vb[16];
         ptx::tmem_ld_32x32b_x16(t_chunk, va);
         ptx::tmem_wait_ld();
         ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);  // in flight while piece 0 is computed
-        exp_piece(va, 0, mc, full, kbase, prow, ls, pmax);
+        exp_piece(mask_tag, va, 0, mc, kbase, t_p, ls);
         ptx::tmem_wait_ld();
         ptx::tmem_ld_32x32b_x16(t_chunk + 32, va);
-        exp_piece(vb, 1, mc, full, kbase, prow, ls, pmax);
+        exp_piece(mask_tag, vb, 1, mc, kbase, t_p, ls);
         ptx::tmem_wait_ld();
         ptx::tmem_ld_32x32b_x16(t_chunk + 48, vb);
-        exp_piece(va, 2, mc, full, kbase, prow, ls, pmax);
+        exp_piece(mask_tag, va, 2, mc, kbase, t_p, ls);
         ptx::tmem_wait_ld();
-        exp_piece(vb, 3, mc, full, kbase, prow, ls, pmax);
+        exp_piece(mask_tag, vb, 3, mc, kbase, t_p, ls);
+        return ls[0] + ls[1];
+      };
+      auto exp_any = [&](bool full, uint32_t t_chunk, float mc, int kbase, uint32_t t_p) {
+        return full ? exp_chunk(std::false_type{}, t_chunk, mc, kbase, t_p)
+                    : exp_chunk(std::true_type{}, t_chunk, mc, kbase, t_p);
+      };
+      // row max of chunk c (first chunk, or the rare redo)
+      auto chunk_max = [&](bool full, uint32_t t_chunk, int kbase) {
+        float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          uint32_t v[16];
+          ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
+          ptx::tmem_wait_ld();
+#pragma unroll
+          for (int e = 0; e < 16; ++e)
+            if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
+        }
+        return fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
       };
 #pragma unroll 1
       for (int c = 0; c < n_ch; ++c) {
@@ -271,42 +339,26 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         const int kbase = c * KC;
         const bool full = kbase + KC <= len;
         const uint32_t t_chunk = t_s + cur * KC;
-        uint8_t* prow = sP + (qi * NS + cur) * kPBytes + r * 128;
+        const uint32_t t_p = t_lane + kPCol + (qi * NS + cur) * (KC / 2);
         // P slot `cur` was read by PV(c - NS)
-        if (c >= NS) ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
-        float ls = 0.f, pmax = 0.f;
+        if (c >= NS) {
+          ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
+          ptx::tc_fence_after();
+        }
+        float ls;
         if (c == 0) {
           // first chunk: row max from a first pass over S
-          float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-#pragma unroll
-          for (int k = 0; k < 4; ++k) {
-            uint32_t v[16];
-            ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
-            ptx::tmem_wait_ld();
-#pragma unroll
-            for (int e = 0; e < 16; ++e)
-              if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
-          }
-          m = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
-          exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
+          m = chunk_max(full, t_chunk, kbase);
+          ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
         } else {
-          // single streaming pass against the (possibly stale) running max: exact
-          // as long as no p exceeds 2^8; otherwise redo the chunk with its max
-          exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
-          if (__any_sync(0xffffffffu, pmax > 256.0f)) {
-            float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
-#pragma unroll
-            for (int k = 0; k < 4; ++k) {
-              uint32_t v[16];
-              ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
-              ptx::tmem_wait_ld();
-#pragma unroll
-              for (int e = 0; e < 16; ++e)
-                if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
-            }
-            const float cmax = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+          // single streaming pass against the (possibly stale) running max.  A row
+          // whose p sum passes 2^8 (necessary if any p > 2^8; impossible while every
+          // p <= 4) is redone against its new max, O and l rescaled.
+          ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
+          if (__any_sync(0xffffffffu, ls > 256.0f)) {
+            const float cmax = fmaxf(m, chunk_max(full, t_chunk, kbase));
             float alpha = 1.f;
-            if (pmax > 256.0f) {  // this row's max rose by > 2^8: rescale O and l
+            if (ls > 256.0f) {  // this row's max rose: rescale O and l
               alpha = ex2_approx((m - cmax) * c2);
               l *= alpha;
               m = cmax;
@@ -324,15 +376,13 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
               ptx::tmem_st_32x32b_x16(t_o + hh * 16, ov);
             }
             ptx::tmem_wait_st();
-            ls = 0.f;
-            pmax = 0.f;
-            exp_chunk(t_chunk, m * c2, full, kbase, prow, ls, pmax);
+            ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
           }
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
         l += ls;
-        // S slot back to the MMA warp, P chunk to the PV MMA
-        ptx::fence_proxy_async_smem();
+        // S slot back to the MMA warp, P chunk (TMEM stores complete) to the PV MMA
+        ptx::tmem_wait_st();
         ptx::tc_fence_before();
         __syncwarp();
         if (lane == 0) {
@@ -456,7 +506,6 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
   if (p.dt == DT_BF16) {
     if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
     if (p.L <= 256) return attn_launch_cfg<2, 2, 2>(p, lengths, o, s);
-    if (getenv("ARLO_ATTN_NQ4")) return attn_launch_cfg<4, 4, 1>(p, lengths, o, s);
     return attn_launch_cfg<2, 4, 2>(p, lengths, o, s);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
