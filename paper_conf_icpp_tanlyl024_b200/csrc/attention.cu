@@ -38,12 +38,13 @@ struct AttnCfg {
   static constexpr int NQ = NQ_;
   static constexpr int NS = NS_;  // S and P (TMEM) slots per q-tile
   static constexpr int kMaxKT = MAXKT_;
-  static constexpr int kKSlots = MAXKT_ < 2 ? MAXKT_ : 2;  // K tiles ring; V stays resident
-  static constexpr int kSoftWarps = 4 * NQ;   // warp w: q-tile w/4, TMEM lane quarter w%4
+  static constexpr int kKSlots = MAXKT_ < 2 ? MAXKT_ : 2;  // K and V tile rings (2 slots each)
+  // softmax warp w: q-tile w/8, key half (w/4)%2 of every chunk, TMEM lane quarter w%4
+  static constexpr int kSoftWarps = 8 * NQ;
   static constexpr int kProdWarp = kSoftWarps;
-  static constexpr int kMmaWarp = kSoftWarps + 1;
-  static constexpr int kThreads = 32 * (kSoftWarps + 2);
-  static constexpr int kSmem = 1024 + kTileBytes * (NQ + kKSlots + kMaxKT) + 256;
+  static constexpr int kMmaWarp = kSoftWarps + 1;  // MMA warp of q-tile qi: kMmaWarp + qi
+  static constexpr int kThreads = 32 * (kSoftWarps + 1 + NQ);
+  static constexpr int kSmem = 1024 + kTileBytes * (NQ + 2 * kKSlots) + 256;
   // TMEM columns, q-tile qi: S slot sl (64 fp32) at qi*NS*64 + sl*64; O (64 fp32)
   // at kOCol + qi*64; P slot sl (64 bf16 packed in 32 columns) at kPCol + (qi*NS + sl)*32
   static constexpr uint32_t kOCol = NQ * NS * KC;
@@ -122,14 +123,17 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   while (nq < NQ && q0 + nq * AQ < len) ++nq;
 
   extern __shared__ uint8_t smem_raw[];
+  __shared__ float xch[NQ][2][2 * AQ];  // softmax pair exchange: [q-tile][half][chunk parity][row]
+  __shared__ float xmax[NQ][2][AQ];     // redo maxima, final partial sums
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sK = sQ + NQ * kTileBytes;
   uint8_t* sV = sK + kKSlots * kTileBytes;
-  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sV + kMaxKT * kTileBytes);
+  uint64_t* bar_k = reinterpret_cast<uint64_t*>(sV + kKSlots * kTileBytes);
   uint64_t* bar_v = bar_k + kMaxKT;
   uint64_t* k_free = bar_v + kMaxKT;
-  uint64_t* s_full = k_free + kKSlots;  // [NQ][2]
+  uint64_t* v_free = k_free + kKSlots;
+  uint64_t* s_full = v_free + kKSlots;  // [NQ][NS]
   uint64_t* s_free = s_full + NS * NQ;
   uint64_t* p_full = s_free + NS * NQ;
   uint64_t* pv_done = p_full + NS * NQ;
@@ -141,11 +145,14 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       ptx::mbar_init(&bar_k[j], 1);
       ptx::mbar_init(&bar_v[j], 1);
     }
-    for (int i = 0; i < kKSlots; ++i) ptx::mbar_init(&k_free[i], 1);
+    for (int i = 0; i < kKSlots; ++i) {  // one commit per live q-tile
+      ptx::mbar_init(&k_free[i], nq);
+      ptx::mbar_init(&v_free[i], nq);
+    }
     for (int i = 0; i < NS * NQ; ++i) {
       ptx::mbar_init(&s_full[i], 1);
-      ptx::mbar_init(&s_free[i], 4);
-      ptx::mbar_init(&p_full[i], 4);
+      ptx::mbar_init(&s_free[i], 8);
+      ptx::mbar_init(&p_full[i], 8);
       ptx::mbar_init(&pv_done[i], 1);
     }
     ptx::fence_mbar_init();
@@ -164,119 +171,86 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       for (int qi = 0; qi < nq; ++qi)
         ptx::tma_load_2d(sQ + qi * kTileBytes, &tm, &bar_k[0], h * D, row_base + q0 + qi * AQ);
       ptx::tma_load_2d(sK, &tm, &bar_k[0], H + h * D, row_base);
-      if (n_kt > 1) {
-        ptx::mbar_arrive_expect_tx(&bar_k[1], kTileBytes);
-        ptx::tma_load_2d(sK + kTileBytes, &tm, &bar_k[1], H + h * D, row_base + AK);
-      }
+      // K and V rings: slot j%2 of K (V) frees when the S (PV) MMAs of tile j-2 complete
       for (int j = 0; j < n_kt; ++j) {
+        if (j > 0) {
+          if (j >= kKSlots) ptx::mbar_wait(&k_free[j & 1], ((j - kKSlots) >> 1) & 1);
+          ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
+          ptx::tma_load_2d(sK + (j & 1) * kTileBytes, &tm, &bar_k[j], H + h * D, row_base + j * AK);
+        }
+        if (j >= kKSlots) ptx::mbar_wait(&v_free[j & 1], ((j - kKSlots) >> 1) & 1);
         ptx::mbar_arrive_expect_tx(&bar_v[j], kTileBytes);
-        ptx::tma_load_2d(sV + j * kTileBytes, &tm, &bar_v[j], 2 * H + h * D, row_base + j * AK);
-      }
-      for (int j = kKSlots; j < n_kt; ++j) {  // K ring: slot j%2 frees when S(., tile j-2) completes
-        ptx::mbar_wait(&k_free[j & 1], ((j - kKSlots) >> 1) & 1);
-        ptx::mbar_arrive_expect_tx(&bar_k[j], kTileBytes);
-        ptx::tma_load_2d(sK + (j & 1) * kTileBytes, &tm, &bar_k[j], H + h * D, row_base + j * AK);
+        ptx::tma_load_2d(sV + (j & 1) * kTileBytes, &tm, &bar_v[j], 2 * H + h * D, row_base + j * AK);
       }
     }
-  } else if (warp == kMmaWarp) {
-    // ------------------------------------------------------------- MMA issuer
-    if (lane == 0) {
+  } else if (warp >= kMmaWarp) {
+    // ------------------------------------------------------------ MMA issuers
+    // One warp per q-tile (tcgen05.mma issue blocks the issuing thread for
+    // ~100 cycles per instruction while the tensor pipe is not streaming, so two
+    // issuers keep both q-tiles' chains moving).  In order per q-tile: S(c) as
+    // soon as its TMEM slot is free and its K tile has landed, then PV(c-1) once
+    // P(c-1) is written, so S(c) overlaps the softmax of chunk c-1.
+    const int qi = warp - kMmaWarp;
+    if (qi < nq) {
       constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
       constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
-      // Event loop: each q-tile advances independently (no head-of-line blocking
-      // on the slower one); an S MMA is issued as soon as its TMEM slot is free
-      // and its K tile has landed, a PV MMA as soon as its P chunk is written.
-      auto issue_s = [&](int qi, int c) {
+      const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
+      auto issue_pv = [&](int c) {
         const int t = c >> 1, sl = c % NS;
-        const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
+        ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
+        ptx::mbar_wait(&bar_v[t], 0);
+        ptx::tc_fence_after();
+        const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
+        const uint32_t v_addr = ptx::smem_u32(sV + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
+#pragma unroll
+        for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
+          ptx::mma_bf16_ts_w(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
+                             idesc_pv, (c | ks) != 0);
+        ptx::mma_commit_w(&pv_done[qi * NS + sl]);
+        if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&v_free[t & 1]);  // V tile t done for this q-tile
+        if (qi == 0 && c < 14 && lane == 0) atrace<TRACE>(48 + c);  // PV(0, c) issued
+      };
+#pragma unroll 1
+      for (int c = 0; c < n_ch; ++c) {
+        const int t = c >> 1, sl = c % NS;
+        if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
+        ptx::mbar_wait(&bar_k[t], 0);
+        ptx::tc_fence_after();
         const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
         for (int k = 0; k < D / 16; ++k)
-          ptx::mma_bf16_ss(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
-                           ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
-        ptx::mma_commit(&s_full[qi * NS + sl]);
-        if (qi == 0 && c < 16) atrace<TRACE>(32 + c);  // S(0, c) issued
-      };
-      auto issue_pv = [&](int qi, int c) {
-        const int t = c >> 1, sl = c % NS;
-        const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
-        const uint32_t v_addr = ptx::smem_u32(sV + t * kTileBytes + (c & 1) * (KC * 128));
-#pragma unroll
-        for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
-          ptx::mma_bf16_ts(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
-                           idesc_pv, (c | ks) != 0);
-        ptx::mma_commit(&pv_done[qi * NS + sl]);
-        // (slots 48..55: MMA loop iteration of S(0, c))
-      };
-      int s_next[NQ], pv_next[NQ];
-#pragma unroll
-      for (int qi = 0; qi < NQ; ++qi) s_next[qi] = pv_next[qi] = 0;
-      int k_done = 0;  // K tiles whose S MMAs have all been issued (k_free committed)
-      int pv_left = nq * n_ch;
-      int iter = 0;
-      long long it_clk[4] = {0, 0, 0, 0};
-      while (pv_left > 0) {
-        if (TRACE && iter >= 8 && iter < 12) it_clk[iter - 8] = clock64();  // MMA event-loop iterations 8..11
-        ++iter;
-#pragma unroll
-        for (int qi = 0; qi < NQ; ++qi) {
-          if (qi >= nq) continue;
-          const int cs = s_next[qi];
-          if (cs < n_ch && (cs < NS || ptx::mbar_test(&s_free[qi * NS + cs % NS], ((cs - NS) / NS) & 1)) &&
-              ptx::mbar_test(&bar_k[cs >> 1], 0)) {
-            ptx::tc_fence_after();
-            if (TRACE && cs == 3) atrace<TRACE>(56 + 2 * qi);  // before S(qi, 3) issue
-            issue_s(qi, cs);
-            if (TRACE && cs == 3) atrace<TRACE>(57 + 2 * qi);  // after
-            if (TRACE && qi == 0 && cs < 8) {
-              const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-              if (cta < 2048) g_atrace[cta * 64 + 48 + cs] = iter;  // loop iteration that issued S(0,cs)
-            }
-            s_next[qi] = cs + 1;
-          }
-          const int cp = pv_next[qi];
-          if (cp < s_next[qi] && ptx::mbar_test(&p_full[qi * NS + cp % NS], (cp / NS) & 1) &&
-              ptx::mbar_test(&bar_v[cp >> 1], 0)) {
-            ptx::tc_fence_after();
-            if (TRACE && cp == 2 && qi == 0) atrace<TRACE>(60);  // before PV(0, 2) issue
-            issue_pv(qi, cp);
-            if (TRACE && cp == 2 && qi == 0) atrace<TRACE>(61);
-            pv_next[qi] = cp + 1;
-            --pv_left;
-          }
-        }
-        // a K tile is free once every live q-tile has issued the S MMAs of both its chunks
-        int smin = n_ch;
-#pragma unroll
-        for (int qi = 0; qi < NQ; ++qi)
-          if (qi < nq) smin = min(smin, s_next[qi]);
-        const int tiles_done = (smin == n_ch) ? n_kt : (smin >> 1);
-        while (k_done < tiles_done) {
-          ptx::mma_commit(&k_free[k_done & 1]);
-          ++k_done;
-        }
+          ptx::mma_bf16_ss_w(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
+                             ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
+        ptx::mma_commit_w(&s_full[qi * NS + sl]);
+        // K tile t is released (for this q-tile) once the S MMAs of both its chunks complete
+        if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&k_free[t & 1]);
+        if (qi == 0 && c < 16 && lane == 0) atrace<TRACE>(32 + c);  // S(0, c) issued
+        if (c > 0) issue_pv(c - 1);
       }
-      if (TRACE) {
-        const unsigned cta = blockIdx.x + gridDim.x * (blockIdx.y + gridDim.y * blockIdx.z);
-        if (cta < 2048)
-          for (int i = 0; i < 4; ++i) g_atrace[cta * 64 + 27 + i] = it_clk[i];
-      }
+      issue_pv(n_ch - 1);
     }
   } else {
     // ----------------------------------------------------------------- softmax
-    const int qi = warp >> 2, quarter = warp & 3;
+    // Two warps per TMEM lane quarter (same 32 query rows): warp half hf owns
+    // keys [32 hf, 32 hf + 32) of every 64-key chunk, O columns [32 hf, 32 hf + 32)
+    // and a partial row sum.  The pair shares one running max per row through
+    // shared memory (a 64-thread named barrier per chunk), so both halves of a
+    // row's P use the same scale.
+    const int qi = warp >> 3, hf = (warp >> 2) & 1, quarter = warp & 3;
     const int r = quarter * 32 + lane;  // query row within q-tile qi == TMEM lane
     const int qrow = q0 + qi * AQ + r;
+    const int bar_id = 1 + qi * 4 + quarter;
+    auto pair_sync = [&]() { asm volatile("bar.sync %0, 64;" ::"r"(bar_id) : "memory"); };
     if (qi < nq) {
       const uint32_t t_lane = tmem + ((uint32_t)(quarter * 32) << 16);
-      const uint32_t t_s = t_lane + qi * NS * KC;
-      const uint32_t t_o = t_lane + kOCol + qi * D;
+      const uint32_t t_s = t_lane + qi * NS * KC + hf * (KC / 2);
+      const uint32_t t_o = t_lane + kOCol + qi * D + hf * (D / 2);
       const float c2 = 0.125f * 1.4426950408889634f;  // 1/sqrt(64) * log2(e)
       float m = -INFINITY, l = 0.f;
-      // 16 keys of chunk c: p = 2^(s*c2 - mc) (0 past len when MASK), fp32 partial
-      // sums, packed bf16 into the row's 8 TMEM P columns for these keys.  MASK is
-      // a compile-time flag: only a chunk straddling len pays for masking.
-      auto exp_piece = [&](auto mask_tag, const uint32_t (&v)[16], int k, float mc, int kbase, uint32_t t_p,
+      // 16 keys: p = 2^(s*c2 - mc) (0 past len when MASK), fp32 partial sums,
+      // packed bf16 into the row's 8 TMEM P columns for these keys.  MASK is a
+      // compile-time flag: only a chunk straddling len pays for masking.
+      auto exp_piece = [&](auto mask_tag, const uint32_t (&v)[16], int key0, float mc, uint32_t t_p,
                            float (&ls)[2]) {
         constexpr bool MASK = decltype(mask_tag)::value;
         uint32_t pk[8];
@@ -285,61 +259,56 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c2, -mc));
           float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c2, -mc));
           if (MASK) {
-            if (kbase + k * 16 + e >= len) p0 = 0.f;
-            if (kbase + k * 16 + e + 1 >= len) p1 = 0.f;
+            if (key0 + e >= len) p0 = 0.f;
+            if (key0 + e + 1 >= len) p1 = 0.f;
           }
           ls[0] += p0;
           ls[1] += p1;
           pk[e >> 1] = pack_bf16x2(p0, p1);
         }
-        ptx::tmem_st_32x32b_x8(t_p + k * 8, pk);
+        ptx::tmem_st_32x32b_x8(t_p, pk);
       };
-      // all 64 keys of chunk c against a given max (S pieces double-buffered); returns the p sum
-      auto exp_chunk = [&](auto mask_tag, uint32_t t_chunk, float mc, int kbase, uint32_t t_p) {
+      // this warp's 32 keys of a chunk against max mc; returns the partial p sum
+      auto exp_half = [&](auto mask_tag, uint32_t t_chunk, float mc, int key0, uint32_t t_p) {
         float ls[2] = {0.f, 0.f};
         uint32_t va[16], vb[16];
         ptx::tmem_ld_32x32b_x16(t_chunk, va);
+        ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);
         ptx::tmem_wait_ld();
-        ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);  // in flight while piece 0 is computed
-        exp_piece(mask_tag, va, 0, mc, kbase, t_p, ls);
-        ptx::tmem_wait_ld();
-        ptx::tmem_ld_32x32b_x16(t_chunk + 32, va);
-        exp_piece(mask_tag, vb, 1, mc, kbase, t_p, ls);
-        ptx::tmem_wait_ld();
-        ptx::tmem_ld_32x32b_x16(t_chunk + 48, vb);
-        exp_piece(mask_tag, va, 2, mc, kbase, t_p, ls);
-        ptx::tmem_wait_ld();
-        exp_piece(mask_tag, vb, 3, mc, kbase, t_p, ls);
+        exp_piece(mask_tag, va, key0, mc, t_p, ls);
+        exp_piece(mask_tag, vb, key0 + 16, mc, t_p + 8, ls);
         return ls[0] + ls[1];
       };
-      auto exp_any = [&](bool full, uint32_t t_chunk, float mc, int kbase, uint32_t t_p) {
-        return full ? exp_chunk(std::false_type{}, t_chunk, mc, kbase, t_p)
-                    : exp_chunk(std::true_type{}, t_chunk, mc, kbase, t_p);
+      auto exp_any = [&](bool full, uint32_t t_chunk, float mc, int key0, uint32_t t_p) {
+        return full ? exp_half(std::false_type{}, t_chunk, mc, key0, t_p)
+                    : exp_half(std::true_type{}, t_chunk, mc, key0, t_p);
       };
-      // row max of chunk c (first chunk, or the rare redo)
-      auto chunk_max = [&](bool full, uint32_t t_chunk, int kbase) {
+      // row max over this warp's 32 keys of a chunk (first chunk, or the rare redo)
+      auto half_max = [&](bool full, uint32_t t_chunk, int key0) {
         float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+        uint32_t va[16], vb[16];
+        ptx::tmem_ld_32x32b_x16(t_chunk, va);
+        ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);
+        ptx::tmem_wait_ld();
 #pragma unroll
-        for (int k = 0; k < 4; ++k) {
-          uint32_t v[16];
-          ptx::tmem_ld_32x32b_x16(t_chunk + k * 16, v);
-          ptx::tmem_wait_ld();
-#pragma unroll
-          for (int e = 0; e < 16; ++e)
-            if (full || kbase + k * 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(v[e]));
+        for (int e = 0; e < 16; ++e) {
+          if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+          if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
         }
         return fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
       };
+      float* xs = xch[qi][hf];        // this warp's exchange row (chunk-parity double-buffered)
+      float* xp = xch[qi][hf ^ 1];    // partner's
 #pragma unroll 1
       for (int c = 0; c < n_ch; ++c) {
-        const int cur = c % NS;
+        const int cur = c % NS, par = c & 1;
         ptx::mbar_wait(&s_full[qi * NS + cur], (c / NS) & 1);
         ptx::tc_fence_after();
         if (warp == 0 && lane == 0) atrace<TRACE>(3 + 3 * (c & 7));
-        const int kbase = c * KC;
-        const bool full = kbase + KC <= len;
+        const int key0 = c * KC + hf * (KC / 2);
+        const bool full = c * KC + KC <= len;
         const uint32_t t_chunk = t_s + cur * KC;
-        const uint32_t t_p = t_lane + kPCol + (qi * NS + cur) * (KC / 2);
+        const uint32_t t_p = t_lane + kPCol + (qi * NS + cur) * (KC / 2) + hf * (KC / 4);
         // P slot `cur` was read by PV(c - NS)
         if (c >= NS) {
           ptx::mbar_wait(&pv_done[qi * NS + cur], ((c - NS) / NS) & 1);
@@ -347,18 +316,26 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         }
         float ls;
         if (c == 0) {
-          // first chunk: row max from a first pass over S
-          m = chunk_max(full, t_chunk, kbase);
-          ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
+          // first chunk: row max from a first pass over S, shared by the pair
+          xs[par * AQ + r] = half_max(full, t_chunk, key0);
+          pair_sync();
+          m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
+          ls = exp_any(full, t_chunk, m * c2, key0, t_p);
         } else {
           // single streaming pass against the (possibly stale) running max.  A row
-          // whose p sum passes 2^8 (necessary if any p > 2^8; impossible while every
-          // p <= 4) is redone against its new max, O and l rescaled.
-          ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
-          if (__any_sync(0xffffffffu, ls > 256.0f)) {
-            const float cmax = fmaxf(m, chunk_max(full, t_chunk, kbase));
+          // whose p sum passes 2^8 in either half (necessary if any p > 2^8;
+          // impossible while every p <= 4) is redone by both halves against the
+          // new row max, O and l rescaled.
+          ls = exp_any(full, t_chunk, m * c2, key0, t_p);
+          xs[par * AQ + r] = ls;
+          pair_sync();
+          const bool need = ls > 256.0f || xp[par * AQ + r] > 256.0f;  // same in both warps
+          if (__any_sync(0xffffffffu, need)) {
+            xmax[qi][hf][r] = half_max(full, t_chunk, key0);
+            pair_sync();
+            const float cmax = fmaxf(m, fmaxf(xmax[qi][0][r], xmax[qi][1][r]));
             float alpha = 1.f;
-            if (ls > 256.0f) {  // this row's max rose: rescale O and l
+            if (need) {
               alpha = ex2_approx((m - cmax) * c2);
               l *= alpha;
               m = cmax;
@@ -366,17 +343,15 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
             // O holds PV_0..c-1 (warp-collective TMEM traffic: every row takes part)
             ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);
             ptx::tc_fence_after();
-#pragma unroll 1
-            for (int hh = 0; hh < 4; ++hh) {
-              uint32_t ov[16];
-              ptx::tmem_ld_32x32b_x16(t_o + hh * 16, ov);
-              ptx::tmem_wait_ld();
+            uint32_t ov[32];
+            ptx::tmem_ld_32x32b_x32(t_o, ov);
+            ptx::tmem_wait_ld();
 #pragma unroll
-              for (int e = 0; e < 16; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
-              ptx::tmem_st_32x32b_x16(t_o + hh * 16, ov);
-            }
+            for (int e = 0; e < 32; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
+            ptx::tmem_st_32x32b_x16(t_o, *reinterpret_cast<uint32_t(*)[16]>(&ov[0]));
+            ptx::tmem_st_32x32b_x16(t_o + 16, *reinterpret_cast<uint32_t(*)[16]>(&ov[16]));
             ptx::tmem_wait_st();
-            ls = exp_any(full, t_chunk, m * c2, kbase, t_p);
+            ls = exp_any(full, t_chunk, m * c2, key0, t_p);
           }
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
@@ -391,33 +366,32 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(5 + 3 * (c & 7));
       }
-      // O = (sum_c P_c V_c) / l
+      // l = l_half0 + l_half1 (fixed order); O = (sum_c P_c V_c) / l
+      xmax[qi][hf][r] = l;  // (every redo's reads of xmax finished before the last chunk's barrier)
+      pair_sync();
+      const float inv = 1.f / (xmax[qi][0][r] + xmax[qi][1][r]);
       ptx::mbar_wait(&pv_done[qi * NS + ((n_ch - 1) % NS)], ((n_ch - 1) / NS) & 1);
       ptx::tc_fence_after();
-      const float inv = 1.f / l;
-      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
+      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D) + hf * 4;
+      uint32_t ov[32];
+      ptx::tmem_ld_32x32b_x32(t_o, ov);
+      ptx::tmem_wait_ld();
+      if (qrow < L) {
 #pragma unroll
-      for (int hh = 0; hh < 2; ++hh) {
-        uint32_t ov[32];
-        ptx::tmem_ld_32x32b_x32(t_o + hh * 32, ov);
-        ptx::tmem_wait_ld();
-        if (qrow < L) {
-#pragma unroll
-          for (int i = 0; i < 4; ++i) {
-            uint4 u;
-            u.x = pack_bf16x2(__uint_as_float(ov[8 * i + 0]) * inv, __uint_as_float(ov[8 * i + 1]) * inv);
-            u.y = pack_bf16x2(__uint_as_float(ov[8 * i + 2]) * inv, __uint_as_float(ov[8 * i + 3]) * inv);
-            u.z = pack_bf16x2(__uint_as_float(ov[8 * i + 4]) * inv, __uint_as_float(ov[8 * i + 5]) * inv);
-            u.w = pack_bf16x2(__uint_as_float(ov[8 * i + 6]) * inv, __uint_as_float(ov[8 * i + 7]) * inv);
-            orow[hh * 4 + i] = u;
-          }
+        for (int i = 0; i < 4; ++i) {
+          uint4 u;
+          u.x = pack_bf16x2(__uint_as_float(ov[8 * i + 0]) * inv, __uint_as_float(ov[8 * i + 1]) * inv);
+          u.y = pack_bf16x2(__uint_as_float(ov[8 * i + 2]) * inv, __uint_as_float(ov[8 * i + 3]) * inv);
+          u.z = pack_bf16x2(__uint_as_float(ov[8 * i + 4]) * inv, __uint_as_float(ov[8 * i + 5]) * inv);
+          u.w = pack_bf16x2(__uint_as_float(ov[8 * i + 6]) * inv, __uint_as_float(ov[8 * i + 7]) * inv);
+          orow[i] = u;
         }
       }
     } else if (qrow < L) {
-      // second q-tile wholly padded: zero rows
-      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D);
+      // q-tile wholly padded: zero rows (each half writes its 32 columns)
+      uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D) + hf * 4;
 #pragma unroll
-      for (int i = 0; i < 8; ++i) orow[i] = make_uint4(0, 0, 0, 0);
+      for (int i = 0; i < 4; ++i) orow[i] = make_uint4(0, 0, 0, 0);
     }
   }
   ptx::tc_fence_before();
@@ -504,9 +478,11 @@ bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) 
 cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
   if (p.B <= 0 || p.L <= 0) return cudaSuccess;
   if (p.dt == DT_BF16) {
-    if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
-    if (p.L <= 256) return attn_launch_cfg<2, 2, 2>(p, lengths, o, s);
-    return attn_launch_cfg<2, 4, 2>(p, lengths, o, s);
+    // one 128-query tile per CTA, two CTAs per SM (TMEM 256 columns, ~83 KB smem
+    // each): one CTA's prologue/epilogue overlaps the other's exp stream
+    if (p.L <= 128) return attn_launch_cfg<1, 1, 2>(p, lengths, o, s);
+    if (p.L <= 256) return attn_launch_cfg<1, 2, 2>(p, lengths, o, s);
+    return attn_launch_cfg<1, 4, 2>(p, lengths, o, s);
   } else {
     const long warps = (long)p.B * p.L * p.heads;
     attn_f32_kernel<<<(unsigned)((warps + 3) / 4), 128, 0, s>>>(p.B, p.L, p.heads, (const float*)p.qkv, lengths,

@@ -2,7 +2,7 @@
 
     python tools/attn_trace.py B L heads len
 Slots: 0/1 start/end, per 64-key chunk c (c < 8): 3+3c S ready (softmax warp 0),
-4+3c exp done, 5+3c P handed over; 32+c S(0,c) issued, 48+c PV(0,c) issued.
+4+3c exp done, 5+3c P handed over; 32+c S(0,c) issued (c < 16), 48+c PV(0,c) issued (c < 14).
 """
 import os
 import sys
@@ -46,7 +46,4 @@ starts = np.sort((gt0 - t00) / 1e3)
 print("CTA start times (first 10 / every 148th):", np.round(starts[:10], 2), np.round(starts[::148], 2))
 mmed = np.nanmedian(d[:, 32:62], axis=0)
 print("S(0,c) issued:", " ".join(f"{x:.2f}" for x in mmed[:16] if not np.isnan(x)))
-print("MMA loop iteration of S(0,c):", " ".join(f"{x:.0f}" for x in np.median(t[:, 48:56], axis=0)))
-print("S(0,3) issue before/after, S(1,3) before/after, PV(0,2) before/after:",
-      " ".join(f"{x:.3f}" for x in mmed[24:30]))
-print("MMA loop iterations 8..11 start:", " ".join(f"{x:.3f}" for x in np.nanmedian(d[:, 27:31], axis=0)))
+print("PV(0,c) issued:", " ".join(f"{x:.2f}" for x in mmed[16:30] if not np.isnan(x)))

@@ -147,6 +147,70 @@ void run_multi(long long* d, int n_mma) {
   printf("  err=%s\n", cudaGetErrorString(cudaGetLastError()));
 }
 
+// Operand-source variants at M=128, N=64, K=16, long streams from one converged
+// warp: mode 0 SS (A, B K-major), 1 SS with B MN-major, 2 TS (A from TMEM) B
+// K-major, 3 TS B MN-major.  Cycles per MMA.
+__device__ __forceinline__ void mma_ts_elect(uint32_t d_tmem, uint32_t a_tmem, uint64_t b_desc, uint32_t idesc,
+                                             uint32_t acc) {
+  asm volatile(
+      "{\n\t.reg .pred p, e;\n\t"
+      "elect.sync _|e, 0xffffffff;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d_tmem),
+      "r"(a_tmem), "l"(b_desc), "r"(idesc), "r"(acc)
+      : "memory");
+}
+template <int MODE>
+__global__ void __launch_bounds__(128, 1) kmode(int n_mma, long long* out) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  __shared__ uint64_t bar;
+  __shared__ uint32_t slot;
+  for (int i = threadIdx.x; i < 65536 / 16; i += blockDim.x) reinterpret_cast<uint4*>(smem)[i] = make_uint4(0, 0, 0, 0);
+  if (threadIdx.x == 0) {
+    ptx::mbar_init(&bar, 1);
+    ptx::fence_mbar_init();
+  }
+  if (threadIdx.x < 32) ptx::tmem_alloc(&slot, 256);
+  ptx::fence_proxy_async_smem();
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = slot;
+  if (threadIdx.x < 32) {
+    const uint32_t a = ptx::smem_u32(smem), b = ptx::smem_u32(smem + 32768);
+    constexpr bool bmn = MODE == 1 || MODE == 3;
+    constexpr uint32_t idesc = bmn ? ptx::idesc_bf16_f32_bmn(128, 64) : ptx::idesc_bf16_f32(128, 64);
+    long long t0 = clock64();
+    for (int i = 0; i < n_mma; ++i) {
+      const uint64_t bd = bmn ? ptx::desc_mn_sw128(b + (i & 3) * 2048, 0) : ptx::desc_k_sw128(b + (i & 3) * 32);
+      if (MODE < 2)
+        mma_elect(tmem, ptx::desc_k_sw128(a + (i & 3) * 32), bd, idesc, i > 0);
+      else
+        mma_ts_elect(tmem, tmem + 128 + (i & 3) * 8, bd, idesc, i > 0);
+    }
+    commit_elect(&bar);
+    ptx::mbar_wait(&bar, 0);
+    long long t1 = clock64();
+    if (blockIdx.x == 0 && threadIdx.x == 0) out[0] = t1 - t0;
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  if (threadIdx.x < 32) ptx::tmem_dealloc(tmem, 256);
+}
+template <int MODE>
+void run_mode(long long* d, int n) {
+  const int smem = 65536 + 2048;
+  cudaFuncSetAttribute(kmode<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  kmode<MODE><<<148, 128, smem>>>(n, d);
+  long long h = 0;
+  cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost);
+  const char* names[] = {"SS  B K-major", "SS  B MN-major", "TS  B K-major", "TS  B MN-major"};
+  printf("M=128 N=64 %s: %d MMAs %.1f cyc/mma  err=%s\n", names[MODE], n, (double)h / n,
+         cudaGetErrorString(cudaGetLastError()));
+}
+
 int main() {
   long long* d;
   cudaMalloc(&d, 32);
@@ -155,6 +219,12 @@ int main() {
     run<64, true>(d, n, 148);
     run<128>(d, n, 148);
     run<128, true>(d, n, 148);
+  }
+  for (int n : {4, 256}) {
+    run_mode<0>(d, n);
+    run_mode<1>(d, n);
+    run_mode<2>(d, n);
+    run_mode<3>(d, n);
   }
   for (int n : {4, 8}) {
     run_multi<1>(d, n);
