@@ -26,8 +26,10 @@ enum { ARLO_EPI_BIAS = 0, ARLO_EPI_BIAS_GELU = 1, ARLO_EPI_BIAS_RESIDUAL = 2 };
  * epi = identity | GELU_erf | (+ residual[M,N]).  Row-major, K-major operands
  * (PyTorch Linear layout).  Requires N % 64 == 0, K % 64 == 0, 1 <= M.
  * ARLO_BF16 runs the tcgen05/TMEM/TMA kernel; ARLO_FP32 the FFMA kernel.
- * force_bn: 0 = automatic tile choice; 64/128/256 = single-CTA kernel with that tile
- * width; -128/-256 = CTA-pair (cta_group::2, 256-row tiles) kernel (tests).
+ * force_bn: 0 = automatic tile choice; 64/128/192/256 = single-CTA kernel with that tile
+ * width; -128/-192/-256 = CTA-pair (cta_group::2, 256-row tiles) kernel; 1016/1032/1064 =
+ * skinny small-M kernel (one CTA per 128 x BN tile, BN = 16/32/64) (tests, sweeps).
+ * Every choice gives bitwise the same rows (same K order per output element).
  */
 int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, const void* A, const void* W,
                  const float* bias, const void* residual, void* out, int32_t epi,
@@ -77,7 +79,8 @@ int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, cons
                  float* pooled, float* logits, void* stream);
 
 /* The tile configuration arlo_op_gemm / the runtime graphs use for (M, N, K):
- * BN for the single-CTA kernel, -BN for the CTA-pair kernel, 0 if unsupported. */
+ * BN for the single-CTA kernel, -BN for the CTA-pair kernel, 1000 + BN for the
+ * skinny small-M kernel, 0 if unsupported. */
 int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K);
 
 /*

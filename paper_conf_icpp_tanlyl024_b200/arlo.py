@@ -14,6 +14,10 @@ import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "libarlo.so")
+# A/B hook for kernel experiments: ARLO_LIB_VARIANT=name loads build/libarlo_<name>.so, an
+# in-tree variant built by `python -m paper_conf_icpp_tanlyl024_b200.build --variant name -D...`.
+if os.environ.get("ARLO_LIB_VARIANT"):
+    LIB_PATH = os.path.join(_HERE, "build", f"libarlo_{os.environ['ARLO_LIB_VARIANT']}.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(f"{LIB_PATH} is missing: build it with `python -m paper_conf_icpp_tanlyl024_b200.build` "

@@ -1,6 +1,8 @@
 """Build libarlo.so in-tree with nvcc for sm_100a (B200) only.
 
     python -m paper_conf_icpp_tanlyl024_b200.build [--verbose-ptxas]
+    python -m paper_conf_icpp_tanlyl024_b200.build --variant NAME -DMACRO=V ...   (A/B experiments:
+        build/libarlo_NAME.so with extra defines, loaded when ARLO_LIB_VARIANT=NAME)
 
 Each translation unit under csrc/ is compiled to an object with
 ``-gencode arch=compute_100a,code=sm_100a -lineinfo -O3`` (in parallel), then
@@ -33,9 +35,9 @@ def nvcc() -> str:
     return p
 
 
-def _compile(src: str, verbose_ptxas: bool) -> tuple:
-    obj = os.path.join(BUILD, os.path.basename(src) + ".o")
-    cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3",
+def _compile(src: str, verbose_ptxas: bool, defines=(), tag="") -> tuple:
+    obj = os.path.join(BUILD, os.path.basename(src) + tag + ".o")
+    cmd = [nvcc(), *ARCH, "-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC,-O3", *defines,
            "-I", os.path.join(ROOT, "include"), "-c", os.path.join(CSRC, src), "-o", obj]
     if src.endswith(".cu"):
         cmd += ["--expt-relaxed-constexpr"]
@@ -80,5 +82,26 @@ def build(verbose_ptxas: bool = False, force: bool = False) -> str:
     return LIB
 
 
+def build_variant(name: str, defines) -> str:
+    """Compile every source with extra -D flags into build/libarlo_<name>.so (A/B runs)."""
+    os.makedirs(BUILD, exist_ok=True)
+    tag = "." + name
+    with cf.ThreadPoolExecutor(max_workers=len(SOURCES)) as ex:
+        for src, obj, rc, out in ex.map(lambda s: _compile(s, False, defines, tag), SOURCES):
+            if rc != 0:
+                raise RuntimeError(f"nvcc failed on {src}:\n{out}")
+    lib = os.path.join(BUILD, f"libarlo_{name}.so")
+    objs = [os.path.join(BUILD, s + tag + ".o") for s in SOURCES]
+    cmd = [nvcc(), *ARCH, "-shared", "-o", lib, *objs, "-cudart", "static", "-lpthread", "-ldl", "-lrt"]
+    r = subprocess.run(cmd, capture_output=True, text=True)
+    if r.returncode != 0:
+        raise RuntimeError(f"link failed:\n{r.stdout}{r.stderr}")
+    return lib
+
+
 if __name__ == "__main__":
-    print(build(verbose_ptxas="--verbose-ptxas" in sys.argv, force="--force" in sys.argv))
+    if "--variant" in sys.argv:
+        name = sys.argv[sys.argv.index("--variant") + 1]
+        print(build_variant(name, [a for a in sys.argv[1:] if a.startswith("-D")]))
+    else:
+        print(build(verbose_ptxas="--verbose-ptxas" in sys.argv, force="--force" in sys.argv))

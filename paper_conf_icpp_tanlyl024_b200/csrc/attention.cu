@@ -460,7 +460,7 @@ cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, 
     if (e != cudaSuccess) return e;
     attr = true;
   }
-  dim3 grid((p.L + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
+  dim3 grid((p.q_rows + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
   if (g_attn_trace_on)
     return launch_k(attn_tc_kernel<NQ, MAXKT, NS, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
                     lengths, (bf16*)o);
@@ -468,8 +468,10 @@ cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, 
                   lengths, (bf16*)o);
 }
 
-bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv) {
+bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv, int q_rows) {
   p->B = B; p->L = L; p->heads = heads; p->dt = dt; p->qkv = qkv;
+  p->q_rows = q_rows > 0 && q_rows < L ? q_rows : L;
+  if (dt != DT_BF16 && p->q_rows != L) return false;  // fp32 check mode always computes every row
   if (dt != DT_BF16) return true;
   if (L > AK * 4) return false;
   return encode_tmap_bf16_2d(&p->tm, qkv, (uint64_t)3 * heads * D, (uint64_t)B * L, 64, 128, 128);

@@ -31,13 +31,21 @@ namespace arlo {
 namespace {
 
 constexpr int BM = 128, BK = 64;
-constexpr int kEpiWarps = 8;                   // warps 0-7: two per TMEM lane quarter
+#ifndef ARLO_EPI_WARPS
+#define ARLO_EPI_WARPS 8
+#endif
+constexpr int kEpiWarps = ARLO_EPI_WARPS;      // warps 0..kEpiWarps-1: kEpiGroups per TMEM lane quarter
+constexpr int kEpiGroups = kEpiWarps / 4;      // column groups of an accumulator tile
 constexpr int kProducerWarp = kEpiWarps;       // warp 8: TMA producer
 constexpr int kMmaWarp = kEpiWarps + 1;        // warp 9: MMA issuer
 constexpr int kThreads = 32 * (kEpiWarps + 2);
 constexpr int kAccStages = 2;
 constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 staging tile (SWIZZLE_64B)
-constexpr int kStagingBytes = kEpiWarps * 2 * kStgBytes;  // double-buffered per epilogue warp
+#ifndef ARLO_STG_BUFS
+#define ARLO_STG_BUFS 2
+#endif
+constexpr int kStgBufs = ARLO_STG_BUFS;         // staging tiles per epilogue warp (TMA stores in flight)
+constexpr int kStagingBytes = kEpiWarps * kStgBufs * kStgBytes;
 constexpr int kSmemBudget = 229376;            // 224 KB of the 227 KB opt-in maximum
 
 // Optional event trace (tools/gemm_trace.py): when g_trace != nullptr every CTA
@@ -75,67 +83,60 @@ struct TcCfg {
 };
 
 // Epilogue of one accumulator tile for one warp: TMEM lane quarter q (32
-// rows), column half cg (BN/2 columns), processed in 32-column chunks.  For
-// each chunk: tcgen05.ld (the next chunk's load, bias and residual are issued
-// before this chunk is computed), bias / GELU / residual in fp32, RNE to bf16,
-// st.shared into a 64-byte-swizzled 32x32 staging tile, then one TMA bulk
-// tensor store of the tile (coalesced, asynchronous; rows >= M clipped by the
-// tensor map).  `release()` fires once the last TMEM load has completed.
-template <int BN>
-struct EpiShape {
-  static constexpr int COLS = BN / 2;            // columns per epilogue warp
-  static constexpr int CW = COLS >= 32 ? 32 : 16;  // chunk width: TMEM load / staging tile / TMA box
-  static constexpr int NC = COLS / CW;
-  static constexpr int SWZ = CW * 2;             // staging row bytes == TMA swizzle mode (64B / 32B)
-};
-
-template <int CW>
-__device__ __forceinline__ void tmem_ld_chunk(uint32_t taddr, uint32_t (&r)[CW]);
-template <>
-__device__ __forceinline__ void tmem_ld_chunk<32>(uint32_t taddr, uint32_t (&r)[32]) {
-  ptx::tmem_ld_32x32b_x32(taddr, r);
-}
-template <>
-__device__ __forceinline__ void tmem_ld_chunk<16>(uint32_t taddr, uint32_t (&r)[16]) {
-  ptx::tmem_ld_32x32b_x16(taddr, r);
-}
+// rows) and the 32-column chunks cg, cg + G, cg + 2G, ... of the tile (G =
+// kEpiGroups warps share a quarter).  For each chunk: tcgen05.ld (the next
+// chunk's load and residual are issued before this chunk is computed), bias /
+// GELU / residual in fp32, RNE to bf16, st.shared into a 64-byte-swizzled
+// 32x32 staging tile, then one TMA bulk tensor store of the tile (coalesced,
+// asynchronous; rows >= M clipped by the tensor map).  `release()` fires once
+// the warp's last TMEM load has completed.
+constexpr int CW = 32;  // chunk width: TMEM load / staging tile / TMA box (columns)
 
 template <int BN, int EPI, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
-                                              int N, const float* __restrict__ bias,
+                                              int ldr, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
                                               uint8_t* stg, int& sc, Release release) {
-  using S = EpiShape<BN>;
-  constexpr int COLS = S::COLS, CW = S::CW, NC = S::NC;
-  constexpr int RV = CW / 8;  // 16-byte residual vectors per row per chunk
+  static_assert(BN % CW == 0, "tile width must be a multiple of 32");
+  constexpr int NCH = BN / CW;                                 // chunks per row block
+  constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;  // chunks per warp (max)
+  constexpr int RV = CW / 8;                                   // 16-byte residual vectors per row per chunk
+  const int nc = (NCH - cg + kEpiGroups - 1) / kEpiGroups;     // this warp's chunks (warp-uniform)
   const int row = row0 + lane;
   const bool row_ok = row < M;
-  const int col0 = n0 + cg * COLS;
-  const float4* bias4 = reinterpret_cast<const float4*>(bias + col0);
-  const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * N + col0);
-  const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16) + cg * COLS;
+  const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)(row_ok ? row : 0) * ldr + n0);
+  const uint32_t t_row = t_acc + ((uint32_t)(q * 32) << 16);
+  if (nc <= 0) {
+    ptx::tc_fence_before();
+    __syncwarp();
+    if (lane == 0) release();
+    return;
+  }
   uint32_t r[2][CW];
   uint4 rv[2][RV];
   if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-    for (int j = 0; j < RV; ++j) rv[0][j] = __ldg(res4 + j);
+    for (int j = 0; j < RV; ++j) rv[0][j] = __ldg(res4 + cg * RV + j);
   }
-  tmem_ld_chunk<CW>(t_row, r[0]);
+  ptx::tmem_ld_32x32b_x32(t_row + cg * CW, r[0]);
   ptx::tmem_wait_ld();
 #pragma unroll
-  for (int c = 0; c < NC; ++c) {
-    const int cur = c & 1, nxt = cur ^ 1;
-    if (c + 1 < NC) {
-      tmem_ld_chunk<CW>(t_row + (c + 1) * CW, r[nxt]);
+  for (int k = 0; k < NCMAX; ++k) {
+    if (k >= nc) break;
+    const int c = cg + k * kEpiGroups;  // chunk index within the tile
+    const int cur = k & 1, nxt = cur ^ 1;
+    if (k + 1 < nc) {
+      ptx::tmem_ld_32x32b_x32(t_row + (c + kEpiGroups) * CW, r[nxt]);
       if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-        for (int j = 0; j < RV; ++j) rv[nxt][j] = __ldg(res4 + (c + 1) * RV + j);
+        for (int j = 0; j < RV; ++j) rv[nxt][j] = __ldg(res4 + (c + kEpiGroups) * RV + j);
       }
     }
+    const float4* bias4 = reinterpret_cast<const float4*>(bias + n0 + c * CW);
     uint32_t pk[CW / 2];
 #pragma unroll
     for (int j = 0; j < CW / 4; ++j) {
-      const float4 b4 = __ldg(bias4 + c * (CW / 4) + j);
+      const float4 b4 = __ldg(bias4 + j);
       float v0 = __uint_as_float(r[cur][4 * j + 0]) + b4.x;
       float v1 = __uint_as_float(r[cur][4 * j + 1]) + b4.y;
       float v2 = __uint_as_float(r[cur][4 * j + 2]) + b4.z;
@@ -151,28 +152,28 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       pk[2 * j] = pack_bf16x2(v0, v1);
       pk[2 * j + 1] = pack_bf16x2(v2, v3);
     }
-    // staging buffer (sc & 1) was last used two chunks ago: make sure its TMA store has read it
-    uint8_t* buf = stg + (sc & 1) * kStgBytes;
-    if (sc >= 2) {
-      if (lane == 0) ptx::bulk_wait_read<1>();
+    // staging buffer sc % kStgBufs was last used kStgBufs chunks ago: make sure its TMA store has read it
+    uint8_t* buf = stg + (sc % kStgBufs) * kStgBytes;
+    if (sc >= kStgBufs) {
+      if (lane == 0) ptx::bulk_wait_read<kStgBufs - 1>();
       __syncwarp();
     }
 #pragma unroll
     for (int j = 0; j < CW / 8; ++j) {
-      // TMA swizzle of a (CW*2)-byte row: 16-byte chunk index ^= address bits [7:8] (64B) / [7] (32B)
-      const int sw = CW == 32 ? (j ^ ((lane >> 1) & 3)) : (j ^ ((lane >> 2) & 1));
+      // TMA 64B swizzle of a 64-byte row: 16-byte chunk index ^= address bits [7:8]
+      const int sw = j ^ ((lane >> 1) & 3);
       *reinterpret_cast<uint4*>(buf + lane * (CW * 2) + sw * 16) =
           make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
     }
     ptx::fence_proxy_async_smem();
     __syncwarp();
     if (lane == 0) {
-      ptx::tma_store_2d(tmC, buf, col0 + c * CW, row0);
+      ptx::tma_store_2d(tmC, buf, n0 + c * CW, row0);
       ptx::bulk_commit();
     }
     ++sc;
     ptx::tmem_wait_ld();
-    if (c == (NC >= 2 ? NC - 2 : 0)) {
+    if (k == (nc >= 2 ? nc - 2 : 0)) {  // the last TMEM load of this warp has completed
       ptx::tc_fence_before();
       __syncwarp();
       if (lane == 0) release();
@@ -184,7 +185,7 @@ template <int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-               const bf16* __restrict__ resid) {
+               const bf16* __restrict__ resid, int ldr) {
   using C = TcCfg<BN, false>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -281,7 +282,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     // warp w may only touch TMEM lanes 32*(w%4)..+31 (rows of the tile); the
     // two warps sharing a quarter take one column half each.
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -292,7 +293,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, N, bias, resid, &tmC, stg,
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg,
                              sc, [te]() { ptx::mbar_arrive(te); });
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
@@ -320,7 +321,7 @@ template <int BN, int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-                    const bf16* __restrict__ resid) {
+                    const bf16* __restrict__ resid, int ldr) {
   using C = TcCfg<BN, true>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -361,12 +362,15 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
   pdl_begin();  // setup above overlapped the previous kernel's tail
+  if (threadIdx.x == 0) trace(0);
 
   if (warp == kProducerWarp) {
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      for (int tile = pair; tile < tiles; tile += npairs) {
+      int it = 0;
+      for (int tile = pair; tile < tiles; tile += npairs, ++it) {
+        trace(2 + 6 * it);
         const int m0 = (tile % num_m) * 2 * BM + rank * BM;
         const int n0 = (tile / num_m) * BN + rank * C::B_ROWS;
         for (int kb = 0; kb < kblocks; ++kb) {
@@ -386,13 +390,16 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       uint32_t phase = 0;
       int acc = 0;
       uint32_t acc_phase = 0;
-      for (int tile = pair; tile < tiles; tile += npairs) {
+      int it = 0;
+      for (int tile = pair; tile < tiles; tile += npairs, ++it) {
         ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
+        trace(3 + 6 * it);
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < kblocks; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
+          if (kb == 0) trace(4 + 6 * it);
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
@@ -404,22 +411,26 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
         ptx::mma_commit_pair(&tfull[acc]);
+        trace(5 + 6 * it);
         if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
       }
     }
   } else {
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
-    for (int tile = pair; tile < tiles; tile += npairs) {
+    int it = 0;
+    for (int tile = pair; tile < tiles; tile += npairs, ++it) {
       const int m0 = (tile % num_m) * 2 * BM + rank * BM, n0 = (tile / num_m) * BN;
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
+      if (warp == 0 && lane == 0) trace(6 + 6 * it);
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, N, bias, resid, &tmC, stg, sc,
+      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg, sc,
                              [te]() { ptx::mbar_arrive_cluster(te); });
+      if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) ptx::bulk_wait<0>();
@@ -427,9 +438,165 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
 
   ptx::tc_fence_before();
   ptx::cluster_sync();
+  if (threadIdx.x == 0) trace(1);
   if (warp == kMmaWarp) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc_pair(tmem_base, C::TMEM_COLS);
+  }
+}
+
+// ---------------------------------------------------------------------------------------------
+// Skinny GEMM for small M (batch-1/2 runtimes: M = b*L <= a few hundred rows).
+// At small M the projections are weight-streaming bound (b*L flop
+// per weight byte, below the ridge), so what matters is how many SMs pull W:
+// one non-persistent CTA per 128 x BN tile with BN in {16, 32, 64} (N/BN CTAs
+// per 128-row block, e.g. 144 CTAs for the BERT-base QKV at BN = 16).  Every
+// output element still accumulates the same K = 16 tcgen05.mma steps in the
+// same order as the wide kernels (M = 128 instruction, only N differs), so its
+// result is bitwise the wide kernels' (tests: tile widths agree bitwise).
+// Warps 0-3 epilogue (TMEM lane quarter = warp), warp 4 TMA producer, warp 5
+// MMA issuer.  The A box is min(128, M rounded up to 8) rows: TMEM lanes past
+// it hold rows that are never stored.  The epilogue stores straight from
+// registers (a row's BN*2 bytes per thread).
+constexpr int kSkThreads = 192;
+
+template <int BN>
+struct SkCfg {
+  static constexpr int A_BYTES = BM * BK * 2;
+  static constexpr int B_BYTES = BN * BK * 2;
+  static constexpr int STAGE = A_BYTES + B_BYTES;
+  static constexpr int STAGES = (kSmemBudget - 1024) / STAGE > 12 ? 12 : (kSmemBudget - 1024) / STAGE;
+  static constexpr int SMEM = 1024 + STAGES * STAGE + 8 * (2 * STAGES + 1) + 16;
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;
+  static_assert(SMEM <= 232448, "skinny smem");
+};
+
+template <int BN, int EPI>
+__global__ void __launch_bounds__(kSkThreads, 1)
+gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, bf16* __restrict__ out,
+                   int M, int N, int K, int a_rows, const float* __restrict__ bias, const bf16* __restrict__ resid,
+                   int ldr) {
+  using C = SkCfg<BN>;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sA = smem;
+  uint8_t* sB = smem + C::STAGES * C::A_BYTES;
+  uint64_t* full = reinterpret_cast<uint64_t*>(sB + C::STAGES * C::B_BYTES);
+  uint64_t* empty = full + C::STAGES;
+  uint64_t* tfull = empty + C::STAGES;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tfull + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int n0 = blockIdx.x * BN, m0 = blockIdx.y * BM;
+  const int kblocks = K / BK;
+  const uint32_t stage_tx = (uint32_t)(a_rows * BK * 2 + C::B_BYTES);
+
+  if (warp == 4 && lane == 0) {
+    ptx::tma_prefetch_desc(&tmA);
+    ptx::tma_prefetch_desc(&tmB);
+    for (int i = 0; i < C::STAGES; ++i) {
+      ptx::mbar_init(&full[i], 1);
+      ptx::mbar_init(&empty[i], 1);
+    }
+    ptx::mbar_init(tfull, 1);
+    ptx::fence_mbar_init();
+  }
+  if (warp == 5) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
+  ptx::tc_fence_before();
+  __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem = *tmem_slot;
+
+  if (warp == 4) {
+    if (lane == 0) {
+      // weights do not depend on the predecessor kernel: start streaming W before
+      // the PDL wait, then A once the producer of A has completed
+      const int pre = kblocks < C::STAGES ? kblocks : C::STAGES;
+      for (int kb = 0; kb < pre; ++kb) {
+        ptx::mbar_arrive_expect_tx(&full[kb], stage_tx);
+        ptx::tma_load_2d(sB + kb * C::B_BYTES, &tmB, &full[kb], kb * BK, n0);
+      }
+      pdl_begin();
+      for (int kb = 0; kb < pre; ++kb) ptx::tma_load_2d(sA + kb * C::A_BYTES, &tmA, &full[kb], kb * BK, m0);
+      int stage = pre % C::STAGES;
+      uint32_t phase = pre == C::STAGES ? 1 : 0;
+      for (int kb = pre; kb < kblocks; ++kb) {
+        ptx::mbar_wait(&empty[stage], phase ^ 1);
+        ptx::mbar_arrive_expect_tx(&full[stage], stage_tx);
+        ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+        ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
+        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+      }
+    }
+  } else if (warp == 5) {
+    pdl_begin();
+    if (lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int kb = 0; kb < kblocks; ++kb) {
+        ptx::mbar_wait(&full[stage], phase);
+        ptx::tc_fence_after();
+        const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+        const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
+#pragma unroll
+        for (int k = 0; k < BK / 16; ++k)
+          ptx::mma_bf16_ss(tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32), idesc,
+                           (kb | k) != 0);
+        ptx::mma_commit(&empty[stage]);
+        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+      }
+      ptx::mma_commit(tfull);
+    }
+  } else {
+    pdl_begin();
+    // epilogue: thread = row (TMEM lane), BN columns, straight 16-byte stores
+    const int row = m0 + warp * 32 + lane;
+    const bool row_ok = row < M;
+    ptx::mbar_wait(tfull, 0);
+    ptx::tc_fence_after();
+    const uint32_t t_row = tmem + ((uint32_t)(warp * 32) << 16);
+#pragma unroll
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      uint32_t r[16];
+      ptx::tmem_ld_32x32b_x16(t_row + c0, r);
+      ptx::tmem_wait_ld();
+      if (row_ok) {
+        uint4 rv[2];
+        if (EPI == EPI_BIAS_RESID) {
+          const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0 + c0);
+          rv[0] = __ldg(res4);
+          rv[1] = __ldg(res4 + 1);
+        }
+        uint32_t pk[8];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+          const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + n0 + c0) + j);
+          float v0 = __uint_as_float(r[4 * j + 0]) + b4.x;
+          float v1 = __uint_as_float(r[4 * j + 1]) + b4.y;
+          float v2 = __uint_as_float(r[4 * j + 2]) + b4.z;
+          float v3 = __uint_as_float(r[4 * j + 3]) + b4.w;
+          if (EPI == EPI_BIAS_GELU) {
+            v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
+          }
+          if (EPI == EPI_BIAS_RESID) {
+            const uint4 u = rv[j >> 1];
+            const float2 fa = unpack_bf16x2((j & 1) ? u.z : u.x), fb = unpack_bf16x2((j & 1) ? u.w : u.y);
+            v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
+          }
+          pk[2 * j] = pack_bf16x2(v0, v1);
+          pk[2 * j + 1] = pack_bf16x2(v2, v3);
+        }
+        uint4* o4 = reinterpret_cast<uint4*>(out + (size_t)row * N + n0 + c0);
+        o4[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        o4[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+      }
+    }
+  }
+  ptx::tc_fence_before();
+  __syncthreads();
+  if (warp == 5) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc(tmem, C::TMEM_COLS);
   }
 }
 
@@ -451,7 +618,7 @@ template <int BN>
 __device__ __forceinline__ float cluster_row_sum(float v, float* red, uint64_t* stat_bar, int& use, int cg,
                                                  int r_local, int lane, uint32_t nt) {
   const int set = use & 1;
-  float* slot = red + (set * 2 + cg) * BM + r_local;  // red[set][half][row]
+  float* slot = red + (set * kEpiGroups + cg) * BM + r_local;  // red[set][column group][row]
   *slot = v;
   __syncwarp();
   if (lane == 0) {
@@ -460,8 +627,9 @@ __device__ __forceinline__ float cluster_row_sum(float v, float* red, uint64_t* 
   ptx::mbar_wait_cluster(&stat_bar[set], (use >> 1) & 1);
   float tot = 0.f;
   for (uint32_t k = 0; k < nt; ++k) {
-    tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * 2 + 0) * BM + r_local, k));
-    tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * 2 + 1) * BM + r_local, k));
+#pragma unroll
+    for (int g = 0; g < kEpiGroups; ++g)
+      tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * kEpiGroups + g) * BM + r_local, k));
   }
   ++use;
   return tot;
@@ -474,7 +642,8 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
                                                  const float* __restrict__ beta, const CUtensorMap* tmC, uint8_t* stg,
                                                  int& sc, float* red, uint64_t* stat_bar, int& use, uint32_t nt,
                                                  Release release) {
-  constexpr int COLS = BN / 2;
+  constexpr int COLS = BN / kEpiGroups;
+  static_assert(COLS % 32 == 0, "fused LN epilogue: 32-column chunks");
   constexpr int NC = COLS / 32;
   const int r_local = q * 32 + lane;
   const int row = row0 + lane;
@@ -577,7 +746,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
   }
 }
 
-constexpr int kLnReserve = 4 * BM * 4 + 16;  // row-statistics exchange buffers + 2 stat barriers
+constexpr int kLnReserve = 2 * kEpiGroups * BM * 4 + 16;  // row-statistics exchange buffers + 2 stat barriers
 
 template <int BN>
 __global__ void __launch_bounds__(kThreads, 1)
@@ -591,8 +760,8 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
-  float* red = reinterpret_cast<float*>(sStg + kStagingBytes);  // [2 sets][2 halves][128 rows]
-  uint64_t* full = reinterpret_cast<uint64_t*>(red + 4 * BM);
+  float* red = reinterpret_cast<float*>(sStg + kStagingBytes);  // [2 sets][column groups][128 rows]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red + 2 * kEpiGroups * BM);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
@@ -673,7 +842,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
   } else {
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * 2 * kStgBytes;
+    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0, use = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -726,7 +895,7 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
     attr_set = true;
   }
   return launch_k(kern, dim3(p.grid), dim3(kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias,
-                  (const bf16*)p.resid);
+                  (const bf16*)p.resid, p.ldr);
 }
 
 template <int BN, bool PAIR>
@@ -735,6 +904,30 @@ cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
     case EPI_BIAS: return launch_cfg<BN, EPI_BIAS, PAIR>(p, s);
     case EPI_BIAS_GELU: return launch_cfg<BN, EPI_BIAS_GELU, PAIR>(p, s);
     case EPI_BIAS_RESID: return launch_cfg<BN, EPI_BIAS_RESID, PAIR>(p, s);
+  }
+  return cudaErrorInvalidValue;
+}
+
+template <int BN, int EPI>
+cudaError_t launch_skinny_cfg(const TcGemmPlan& p, cudaStream_t s) {
+  using C = SkCfg<BN>;
+  auto kern = gemm_skinny_kernel<BN, EPI>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  return launch_k(kern, dim3(p.N / BN, (p.M + BM - 1) / BM), dim3(kSkThreads), C::SMEM, s, p.tmA, p.tmB,
+                  (bf16*)p.out, p.M, p.N, p.K, p.a_rows, p.bias, (const bf16*)p.resid, p.ldr);
+}
+
+template <int BN>
+cudaError_t launch_skinny_bn(const TcGemmPlan& p, cudaStream_t s) {
+  switch (p.epi) {
+    case EPI_BIAS: return launch_skinny_cfg<BN, EPI_BIAS>(p, s);
+    case EPI_BIAS_GELU: return launch_skinny_cfg<BN, EPI_BIAS_GELU>(p, s);
+    case EPI_BIAS_RESID: return launch_skinny_cfg<BN, EPI_BIAS_RESID>(p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -756,11 +949,11 @@ int num_sms() {
 }
 
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
-                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes) {
+                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes, uint64_t row_elems) {
   EncodeTiledFn fn = get_encode_fn();
   if (!fn) return false;
   cuuint64_t dims[2] = {inner, outer};
-  cuuint64_t strides[1] = {inner * 2};
+  cuuint64_t strides[1] = {(row_elems ? row_elems : inner) * 2};
   cuuint32_t box[2] = {box_inner, box_outer};
   cuuint32_t estr[2] = {1, 1};
   CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box,
@@ -774,12 +967,16 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
 }
 
 // Tile choice: a function of (M, N, K) only (never of the data), minimising a
-// wave-quantised time estimate.  Per tile: MMA time of a 128 x BN x K slab at
-// 8192 flop/clk/SM divided by a feed efficiency measured on B200
-// (tools/gemm_sweep.py: CTA pairs and single CTAs at BN >= 192 sustain the
-// tensor pipe; BN = 128 tiles re-read A twice as often and run ~30% slower),
-// plus a fixed ~1 us tile prologue/epilogue cost.  Returns BN for the
-// single-CTA kernel, -BN for the CTA-pair kernel.
+// wave-quantised time estimate.  Wide kernels, per tile: MMA time of a
+// 128 x BN x K slab at 8192 flop/clk/SM divided by a feed efficiency measured
+// on B200 (tools/gemm_sweep.py: CTA pairs and single CTAs at BN >= 192 sustain
+// the tensor pipe; BN = 128 tiles re-read A twice as often and run ~30%
+// slower), plus a fixed ~1 us tile prologue/epilogue cost.  Skinny kernel (one
+// CTA per 128 x BN tile, M <= 512): the CTA's operand bytes at ~kSkFeed B/clk
+// per SM plus ~1.5 us of latency.  Returns BN for the single-CTA kernel, -BN
+// for the CTA-pair kernel, kSkinnyCode + BN for the skinny kernel.
+constexpr double kSkFeed = 96.0;
+
 int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
   double best = 1e30;
@@ -798,27 +995,54 @@ int tc_choose_bn(int M, int N, int K) {
     const double t = waves * (mma_us / eff + 1.0);
     if (t < best * 0.999) { best = t; best_bn = c; }
   }
+  if (M <= 512 && getenv("ARLO_NO_SKINNY") == nullptr) {
+    const int a_rows = M < BM ? ((M + 7) & ~7) : BM;
+    for (int bn : {16, 32, 64}) {
+      if (N % bn) continue;
+      const long ctas = (long)((M + BM - 1) / BM) * (N / bn);
+      const long waves = (ctas + sms - 1) / sms;
+      const double bytes = 2.0 * (double)(a_rows + bn) * K;
+      const double t = waves * (bytes / kSkFeed / 1.9e3 + 1.5);
+      if (t < best * 0.999) { best = t; best_bn = kSkinnyCode + bn; }
+    }
+  }
   return best_bn;
 }
 
 bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
                   const float* bias, const void* resid, void* out, int epi, int force_bn) {
-  if (M <= 0 || N % 64 || K % 64 || K <= 0) return false;
+  return tc_plan_gemm_strided(p, M, N, K, A, K, W, bias, resid, N, out, epi, force_bn);
+}
+
+bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int lda, const void* W,
+                          const float* bias, const void* resid, int ldr, void* out, int epi, int force_bn) {
+  if (M <= 0 || N % 64 || K % 64 || K <= 0 || lda < K || lda % 8 || ldr < N || ldr % 8) return false;
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
+  if (choice > kSkinnyCode) {
+    const int bn = choice - kSkinnyCode;
+    if ((bn != 16 && bn != 32 && bn != 64) || N % bn) return false;
+    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->epi = epi; p->ln = false;
+    p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
+    p->a_rows = M < BM ? ((M + 7) & ~7) : BM;
+    p->grid = (N / bn) * ((M + BM - 1) / BM);
+    if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, p->a_rows, 128, (uint64_t)lda)) return false;
+    if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
+    return true;
+  }
   const bool pair = choice < 0;
   const int bn = pair ? -choice : choice;
   if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn < 128) return false;
   if (N % bn) return false;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->epi = epi; p->ln = false;
-  p->bias = bias; p->resid = resid; p->out = out;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->epi = epi; p->ln = false;
+  p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
   const int tile_m = pair ? 2 * BM : BM;
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
   const int slots = pair ? num_sms() / 2 : num_sms();
   p->grid = (tiles < slots ? tiles : slots) * (pair ? 2 : 1);
-  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128, (uint64_t)lda)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn, 128)) return false;
-  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, 32, 32, 64)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
   return true;
 }
 
@@ -858,28 +1082,37 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
                      const void* resid, const float* gamma, const float* beta, float eps, void* out) {
   if (M <= 0 || K % 64 || K <= 0) return false;
   int bn = 0;
-  if (N % 192 == 0 && N / 192 <= 8 && N > 256) bn = 192;
+  if (N % 192 == 0 && N / 192 <= 8 && N > 256 && (192 / kEpiGroups) % 32 == 0) bn = 192;
   if (N % 256 == 0 && N / 256 <= 8) bn = 256;
   if (N == 128) bn = 128;
   if (!bn) return false;
   const int nt = N / bn;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->epi = EPI_BIAS_RESID; p->ln = true;
-  p->bias = bias; p->resid = resid; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->bias = bias; p->resid = resid; p->ldr = N; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
   const int num_m = (M + BM - 1) / BM;
   const int clusters = num_sms() / nt;
   p->grid = (num_m < clusters ? num_m : clusters) * nt;
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
-  const int cw = bn / 2 >= 32 ? 32 : 16;  // EpiShape<bn>::CW
-  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, cw, 32, cw * 2)) return false;
+  if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
   return true;
 }
 
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
+  if (p.skinny) {
+    switch (p.BN) {
+      case 16: return launch_skinny_bn<16>(p, s);
+      case 32: return launch_skinny_bn<32>(p, s);
+      case 64: return launch_skinny_bn<64>(p, s);
+    }
+    return cudaErrorInvalidValue;
+  }
   if (p.ln) {
     switch (p.BN) {
       case 128: return launch_ln<128>(p, s);
-      case 192: return launch_ln<192>(p, s);
+      case 192:
+        if constexpr ((192 / kEpiGroups) % 32 == 0) return launch_ln<192>(p, s);
+        return cudaErrorInvalidValue;
       case 256: return launch_ln<256>(p, s);
     }
     return cudaErrorInvalidValue;

@@ -33,18 +33,27 @@ struct TcGemmPlan {
   CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN (BN/2 for a pair)}, 128B swizzle
   CUtensorMap tmC;  // output      [M, N] bf16, box {32, 32}, 64B swizzle (epilogue TMA stores)
   int M, N, K, BN, epi, grid;
-  bool pair;  // CTA-pair (cta_group::2) kernel, 256-row tiles
+  bool pair;    // CTA-pair (cta_group::2) kernel, 256-row tiles
+  bool skinny;  // small-M kernel: one CTA per 128 x BN tile (BN 16/32/64), direct stores
+  int a_rows;   // skinny: A box rows (min(128, M rounded up to 8))
   bool ln;    // fused residual + LayerNorm epilogue over full rows (cluster of N/BN CTAs)
   const float* gamma;
   const float* beta;
   float eps;
   const float* bias;
   const void* resid;
+  int ldr;  // residual row stride (elements)
   void* out;
 };
 bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
                   const float* bias, const void* resid, void* out, int epi, int force_bn);
+// Row-strided variant: A row i at A + i*lda, residual row i at resid + i*ldr (elements).
+// The runtime's CLS-only last layer reads row 0 of every sequence (lda = ldr = L*H).
+bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int lda, const void* W,
+                          const float* bias, const void* resid, int ldr, void* out, int epi, int force_bn);
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s);
+// Tile choice codes: BN (single CTA), -BN (CTA pair), kSkinnyCode + BN (skinny kernel).
+constexpr int kSkinnyCode = 1000;
 int tc_choose_bn(int M, int N, int K);
 // out = LN(A W^T + bias + resid; gamma, beta, eps), N = hidden size (128 / 768 / 1024 ...).
 // `out` may alias `resid` (each tile reads its residual before storing the same region).
@@ -61,10 +70,11 @@ cudaError_t launch_gemm_simt(DType dt, int M, int N, int K, const void* A, const
 struct AttnPlan {
   CUtensorMap tm;  // QKV [B*L, 3H] bf16, box {64, 128}, 128B swizzle
   int B, L, heads;
+  int q_rows;  // queries computed per sequence: L, or 1 for the CLS-only last layer (one 128-row q-tile)
   DType dt;
   const void* qkv;
 };
-bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv);
+bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv, int q_rows = 0);
 cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s);
 
 // ---- a9: CLS pooler + classifier ----------------------------------------------------------
@@ -73,7 +83,8 @@ cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, con
                         float* logits, cudaStream_t s);
 
 // Resolve cuTensorMapEncodeTiled through the runtime (no link-time libcuda dependency).
+// row_elems = row stride in elements (0: rows are contiguous, stride = inner).
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
-                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes);
+                         uint32_t box_inner, uint32_t box_outer, int swizzle_bytes, uint64_t row_elems = 0);
 
 }  // namespace arlo

@@ -161,6 +161,14 @@ struct Bucket {
   std::vector<LayerPlans> plans;  // bf16 only
   bool fused_ln = false;          // o / f2 plans carry residual + LayerNorm (no separate LN kernels)
   AttnPlan attn;
+  // CLS-only last layer (bf16): only position 0 of each sequence feeds the pooler
+  // (reading S8), so after the last layer's QKV projection and the attention of
+  // q-tile 0, the out-projection, LayerNorms and FFN run on the b CLS rows
+  // (A and residual read with row stride L*H, outputs compact [b, H]).  Same
+  // K order per row => bitwise the rows the full layer would produce.
+  bool cls_prune = false;
+  LayerPlans cls;
+  AttnPlan attn_cls;
   cudaGraphExec_t exec = nullptr;
   size_t nodes = 0;
 };
@@ -200,6 +208,21 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                             w->emb_b(), c.ln_eps, rt->X, rt->err, s),
             "embed_ln launch");
   for (int l = 0; l < c.layers; ++l) {
+    if (bk.cls_prune && l == c.layers - 1) {
+      // last layer on the b CLS rows only (see Bucket::cls_prune)
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].qkv, s), "qkv gemm launch");
+      ARLO_CUDA(attn_launch(bk.attn_cls, rt->lengths, rt->O, s), "attention launch (CLS q-tile)");
+      ARLO_CUDA(tc_launch_gemm(bk.cls.o, s), "out-proj gemm launch (CLS rows)");
+      ARLO_CUDA(launch_layernorm(dt, b, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
+                                 c.ln_eps, rt->X, s),
+                "ln1 launch (CLS rows)");
+      ARLO_CUDA(tc_launch_gemm(bk.cls.f1, s), "ffn1 gemm launch (CLS rows)");
+      ARLO_CUDA(tc_launch_gemm(bk.cls.f2, s), "ffn2 gemm launch (CLS rows)");
+      ARLO_CUDA(launch_layernorm(dt, b, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
+                                 c.ln_eps, rt->X, s),
+                "ln2 launch (CLS rows)");
+      continue;
+    }
     if (dt == DT_BF16) {
       ARLO_CUDA(tc_launch_gemm(bk.plans[l].qkv, s), "qkv gemm launch");
     } else {
@@ -235,7 +258,8 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  c.ln_eps, rt->X, s),
                 "ln2 launch");
   }
-  ARLO_CUDA(launch_head(dt, b, L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
+  // the pooler reads position 0 of sequence i at row i*L of X, or row i after a CLS-only last layer
+  ARLO_CUDA(launch_head(dt, b, bk.cls_prune ? 1 : L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
                         (const float*)w->hd(3), rt->pooled, rt->logits, s),
             "head launch");
   return ARLO_OK;
@@ -274,6 +298,21 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
                         EPI_BIAS_RESID, 0);
     }
     if (!ok) return set_error(ARLO_ECUDA, "tensor-map encoding failed (cuTensorMapEncodeTiled unavailable?)");
+  }
+  bk.cls_prune = !bk.fused_ln && getenv("ARLO_NO_CLS_PRUNE") == nullptr;
+  if (bk.cls_prune) {
+    const int l = c.layers - 1, b = bk.b, L = rt->L;
+    // out-proj: A = O rows {i*L}, residual = X rows {i*L}, y -> Y[0:b]; LN1 -> X[0:b];
+    // FFN1: X[0:b] -> F[0:b]; FFN2: F[0:b], residual X[0:b] -> Y[0:b]; LN2 -> X[0:b]
+    const bool ok =
+        attn_plan(&bk.attn_cls, rt->dt, b, L, c.heads, rt->QKV, 1) &&
+        tc_plan_gemm_strided(&bk.cls.o, b, H, H, rt->O, L * H, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X,
+                             L * H, rt->Y, EPI_BIAS_RESID, 0) &&
+        tc_plan_gemm(&bk.cls.f1, b, F, H, rt->X, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, rt->F,
+                     EPI_BIAS_GELU, 0) &&
+        tc_plan_gemm(&bk.cls.f2, b, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
+                     EPI_BIAS_RESID, 0);
+    if (!ok) return set_error(ARLO_ECUDA, "CLS-row plan: tensor-map encoding failed");
   }
   return ARLO_OK;
 }

@@ -35,9 +35,10 @@ GEMM_SHAPES = [
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
 @pytest.mark.parametrize("epi", [0, 1, 2])
-@pytest.mark.parametrize("force", [0, 128, -128, -256, 192, -192])
+@pytest.mark.parametrize("force", [0, 128, -128, -256, 192, -192, 1016, 1032, 1064])
 def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
-    if N % abs(force or 64):
+    """force: BN single CTA, -BN CTA pair, 1000 + BN skinny (small-M) kernel, 0 = tile chooser."""
+    if N % (force - 1000 if force > 1000 else abs(force or 64)):
         pytest.skip("tile width does not divide N")
     A = rnd((M, K), 1)
     W = rnd((N, K), 2, 0.02)
@@ -57,13 +58,13 @@ def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
     np.testing.assert_allclose(got, ref, rtol=8e-3, atol=8e-3)
 
 
-@pytest.mark.parametrize("bn", [64, 128, 192, 256, -128, -192, -256])
+@pytest.mark.parametrize("bn", [64, 128, 192, 256, -128, -192, -256, 1016, 1032, 1064])
 def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
     """Row results do not depend on the tile width (cross-L invariance contract)."""
     M, N, K = 300, 768, 768
     A, W, b = bf16_dev(rnd((M, K), 5)), bf16_dev(rnd((N, K), 6, 0.02)), f32_dev(rnd((N,), 7, 0.02))
     outs = []
-    for force in (bn, 0):
+    for force in (bn, -256):
         o = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
         arlo_lib.op_gemm(arlo_lib.BF16, A, W, b, o, epi=0, force_bn=force)
         outs.append(o)

@@ -180,3 +180,20 @@ def test_enqueue_matches_infer(arlo_lib):
     np.testing.assert_array_equal(out.cpu().numpy(), a[:12])
     assert rt.kernel_count(12) in (3 + 5 * cfg.layers, 3 + 7 * cfg.layers)  # fused / unfused LayerNorm
     rt.close()
+
+
+@pytest.mark.parametrize("L,max_batch", [(64, 8), (256, 4), (512, 32)])
+def test_cls_only_last_layer_is_bitwise(arlo_lib, monkeypatch, L, max_batch):
+    """The CLS-only last layer (out-proj/LN/FFN on the b position-0 rows, row stride
+    L*H) gives bitwise the logits of the full static-shape last layer."""
+    cfg = wl.BERT_BASE
+    w, W = weights(arlo_lib, cfg, 0)
+    lengths = wl.sample_lengths(max_batch, seed=51, lo=0, hi=L)
+    lengths[0] = L
+    ids = wl.sample_token_ids(cfg, lengths, L, seed=52)
+    pruned = run(arlo_lib, W, L, max_batch, ids, lengths)
+    monkeypatch.setenv("ARLO_NO_CLS_PRUNE", "1")
+    full = run(arlo_lib, W, L, max_batch, ids, lengths)
+    np.testing.assert_array_equal(pruned, full)
+    ref = orc.forward_batch(cfg, w, ids, lengths)
+    assert np.max(np.abs(pruned - ref)) <= 2e-2

@@ -1,6 +1,6 @@
-"""Run forwards of one BERT-base runtime (for an ncu launch list / per-kernel breakdown).
+"""Run forwards of one BERT-base (or BERT-large: 4th arg "large") runtime (for an ncu launch list / per-kernel breakdown).
 
-    python tools/forward_breakdown.py L b [reps]
+    python tools/forward_breakdown.py L b [reps] [base|large]
     ncu --metrics gpu__time_duration.sum --cache-control none --clock-control none --csv \
         --log-file out.csv python tools/forward_breakdown.py 128 32
     python tools/forward_breakdown.py --summarize out.csv
@@ -43,7 +43,7 @@ def main():
     from paper_conf_icpp_tanlyl024_b200 import workload as wl
     L, b = int(sys.argv[1]), int(sys.argv[2])
     reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
-    cfg = wl.BERT_BASE
+    cfg = wl.BERT_LARGE if len(sys.argv) > 4 and sys.argv[4] == "large" else wl.BERT_BASE
     W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg), arlo.BF16), arlo.BF16)
     rt = arlo.Runtime(W, L, b)
     lens = np.full(b, L, np.int32)

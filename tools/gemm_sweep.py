@@ -1,7 +1,10 @@
 """Time the tcgen05 GEMM at several shapes / tile choices with CUDA events (warm L2).
 
-    python tools/gemm_sweep.py [force ...]     force: 0 auto, 64/128/256 single CTA, -128/-256 CTA pair
+    python tools/gemm_sweep.py [--epi E] [--set base|large|small|all] [force ...]
+        force: 0 auto, 64/128/192/256 single CTA, -128/-192/-256 CTA pair
+        epi:   0 bias, 1 bias+GELU, 2 bias+residual
 """
+import argparse
 import os
 import sys
 
@@ -10,9 +13,17 @@ import torch
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_icpp_tanlyl024_b200 import arlo  # noqa: E402
 
-SHAPES = [(4096, 2304, 768), (4096, 3072, 768), (4096, 768, 3072), (8192, 8192, 8192), (4096, 4096, 8192),
-          (16384, 3072, 768), (16384, 1024, 4096), (16384, 768, 3072), (8192, 2304, 768), (2048, 768, 768),
-          (64, 2304, 768), (128, 768, 3072)]
+SETS = {
+    "base": [(4096, 2304, 768), (4096, 3072, 768), (4096, 768, 3072), (4096, 768, 768),
+             (16384, 2304, 768), (16384, 3072, 768), (16384, 768, 3072), (16384, 768, 768)],
+    "large": [(32768, 3072, 1024), (32768, 4096, 1024), (32768, 1024, 4096), (32768, 1024, 1024),
+              (16384, 3072, 1024), (16384, 4096, 1024), (16384, 1024, 4096), (16384, 1024, 1024),
+              (8192, 8192, 8192)],
+    "small": [(64, 2304, 768), (64, 3072, 768), (64, 768, 3072), (64, 768, 768),
+              (128, 2304, 768), (128, 768, 3072), (512, 2304, 768), (512, 768, 3072),
+              (128, 3072, 1024), (128, 1024, 4096)],
+}
+SETS["all"] = SETS["base"] + SETS["large"] + SETS["small"]
 
 
 def time_op(fn, reps=20):
@@ -43,23 +54,31 @@ def time_op(fn, reps=20):
 
 
 def main():
-    forces = [int(x) for x in sys.argv[1:]] or [0, 256, 192, 128, -256, -192, -128]
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--epi", type=int, default=0)
+    ap.add_argument("--set", default="base")
+    ap.add_argument("--no-cublas", action="store_true")
+    ap.add_argument("forces", nargs="*", type=int)
+    a = ap.parse_args()
+    forces = a.forces or [0, 256, 192, 128, -256, -192, -128]
     dev = torch.device("cuda")
-    for (M, N, K) in SHAPES:
+    for (M, N, K) in SETS[a.set]:
         A = torch.randn(M, K, device=dev).to(torch.bfloat16)
         W = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
         b = torch.zeros(N, device=dev)
+        R = torch.randn(M, N, device=dev).to(torch.bfloat16) if a.epi == 2 else None
         out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-        line = f"{M:6d} {N:5d} {K:5d}:"
+        line = f"{M:6d} {N:5d} {K:5d} choice={arlo.gemm_tile_choice(M, N, K):5d}:"
         fl = 2.0 * M * N * K
         for f in forces:
-            if N % abs(f or 64):
+            if N % (f - 1000 if f > 1000 else abs(f or 64)):
                 line += f"  {f:5d}=   n/a  "
                 continue
-            t = time_op(lambda st: arlo.op_gemm(arlo.BF16, A, W, b, out, epi=0, force_bn=f, stream=st))
-            line += f"  {f:5d}={fl / t / 1e12:6.0f}TF"
-        t = time_op(lambda st: torch.matmul(A, W.t()))
-        line += f"  cublas={fl / t / 1e12:6.0f}TF"
+            t = time_op(lambda st: arlo.op_gemm(arlo.BF16, A, W, b, out, epi=a.epi, residual=R, force_bn=f, stream=st))
+            line += f"  {f:5d}={fl / t / 1e12:5.0f}TF/{t * 1e6:6.1f}us"
+        if not a.no_cublas:
+            t = time_op(lambda st: torch.matmul(A, W.t()))
+            line += f"  cublas={fl / t / 1e12:5.0f}TF/{t * 1e6:6.1f}us"
         print(line, flush=True)
 
 
