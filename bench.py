@@ -295,6 +295,7 @@ def main():
         result["e2e"] = e2e_res
         result["bert_large"] = bert_large_per_L(arlo, torch, dev, stream, local_rank)
         result["trace_replay"] = trace_replay(arlo, torch, runtimes, cfg, stream, result)
+        result["cluster_replay"] = cluster_replay(arlo, torch, W, runtimes, cfg, stream)
         if not args.no_cpu_baseline:
             result["cpu_baseline"] = cpu_baseline()
     if rank == 0:
@@ -318,6 +319,32 @@ def trace_replay(arlo, torch, runtimes, cfg, stream, result):
                                                               slo_ms=150.0, max_batch=MAX_BATCH, per_L_ms=per_L,
                                                               stream=stream)
     return out
+
+
+def cluster_replay(arlo, torch, W, runtimes, cfg, stream):
+    """BASELINE configs[3]: BERT-base polymorphing with 8 runtimes (L = 64..512 step 64) placed by
+    the ILP (arlo_allocate) on G = 1, 2, 4, 8 GPUs, requests routed by Algorithm 1, vs ST-512.
+    Instances are independent replicas, so the G-GPU cluster is simulated with G virtual device
+    clocks driven by real forwards on this GPU (replay.cluster_replay)."""
+    from paper_conf_icpp_tanlyl024_b200 import replay
+    rts = dict(runtimes)
+    extra = []
+    for L in wl.RUNTIME_LENGTHS:
+        if L not in rts:
+            rt = arlo.Runtime(W, L, MAX_BATCH)
+            rt.set_stream(stream)
+            rts[L] = rt
+            extra.append(rt)
+    t0 = time.time()
+    res = replay.cluster_replay(arlo, torch, rts, cfg, Gs=(1, 2, 4, 8), n_requests=6000, slo_ms=150.0,
+                                max_batch=MAX_BATCH, stream=stream)
+    res["wall_s"] = time.time() - t0
+    res["note"] = ("one runtime instance per GPU (PAPER.md:L155), G virtual device clocks advanced by real "
+                   "forwards on this B200 (replicas never communicate); saturation = all requests at t=0; "
+                   "latencies from a Poisson replay at 70% of the saturation rate")
+    for rt in extra:
+        rt.close()
+    return res
 
 
 def bert_large_per_L(arlo, torch, dev, stream, device_index):

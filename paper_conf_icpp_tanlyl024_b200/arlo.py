@@ -31,7 +31,7 @@ EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
 EXPORTED = [
     "arlo_last_error", "arlo_version", "arlo_weights_count", "arlo_weights_create", "arlo_weights_destroy",
     "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
-    "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_allocate",
+    "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
     "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
     "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
@@ -68,6 +68,7 @@ _sig("arlo_runtime_max_batch", _i32, _vp)
 _sig("arlo_infer", C.c_int, _vp, _vp, _vp, _vp)
 _sig("arlo_enqueue", C.c_int, _vp, _i32, _vp, _vp, _vp)
 _sig("arlo_runtime_kernel_count", _i32, _vp, _i32)
+_sig("arlo_runtime_bucket", _i32, _vp, _i32)
 _sig("arlo_allocate", C.c_int, _i32, _i32, _P(_f64), _P(_f64), _P(_f64), _i32, _P(_i32), _P(_f64))
 _sig("arlo_sched_create", C.c_int, _i32, _P(_i32), _P(_i32), _P(_f64), _f64, _f64, _i32, _P(_vp))
 _sig("arlo_sched_destroy", None, _vp)
@@ -170,6 +171,10 @@ class Runtime:
 
     def set_stream(self, stream):
         check(lib.arlo_runtime_set_stream(self.handle, _stream_ptr(stream)))
+
+    def bucket_of(self, n: int) -> int:
+        """Batch bucket (captured graph) that serves n requests."""
+        return check(lib.arlo_runtime_bucket(self.handle, n))
 
     def kernel_count(self, n: int) -> int:
         return check(lib.arlo_runtime_kernel_count(self.handle, n))

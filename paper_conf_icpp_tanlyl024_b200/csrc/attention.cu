@@ -42,8 +42,10 @@ struct AttnCfg {
   // softmax warp w: q-tile w/8, key half (w/4)%2 of every chunk, TMEM lane quarter w%4
   static constexpr int kSoftWarps = 8 * NQ;
   static constexpr int kProdWarp = kSoftWarps;
-  static constexpr int kMmaWarp = kSoftWarps + 1;  // MMA warp of q-tile qi: kMmaWarp + qi
-  static constexpr int kThreads = 32 * (kSoftWarps + 1 + NQ);
+  // MMA issuers of q-tile qi: warp kMmaWarp + 2 qi issues the S = Q K^T MMAs, warp
+  // kMmaWarp + 2 qi + 1 the O += P V MMAs (two independent issue chains)
+  static constexpr int kMmaWarp = kSoftWarps + 1;
+  static constexpr int kThreads = 32 * (kSoftWarps + 1 + 2 * NQ);
   static constexpr int kSmem = 1024 + kTileBytes * (NQ + 2 * kKSlots) + 256;
   // TMEM columns, q-tile qi: S slot sl (64 fp32) at qi*NS*64 + sl*64; O (64 fp32)
   // at kOCol + qi*64; P slot sl (64 bf16 packed in 32 columns) at kPCol + (qi*NS + sl)*32
@@ -185,49 +187,53 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     }
   } else if (warp >= kMmaWarp) {
     // ------------------------------------------------------------ MMA issuers
-    // One warp per q-tile (tcgen05.mma issue blocks the issuing thread for
-    // ~100 cycles per instruction while the tensor pipe is not streaming, so two
-    // issuers keep both q-tiles' chains moving).  In order per q-tile: S(c) as
-    // soon as its TMEM slot is free and its K tile has landed, then PV(c-1) once
-    // P(c-1) is written, so S(c) overlaps the softmax of chunk c-1.
-    const int qi = warp - kMmaWarp;
+    // Two issuing warps per q-tile.  A tcgen05.mma costs its issuing thread
+    // ~50-200 cycles at these shapes (M=128, N=64, K=16; tools/mma_bench.cu),
+    // so one thread issuing both S(c+1) and PV(c) (8 MMAs per 64-key chunk) was
+    // the per-chunk critical path; with S and PV on separate chains each chunk
+    // costs at most 4 MMA issues per chain.  S(c) is issued as soon as its TMEM
+    // slot is free and its K tile has landed; PV(c) once P(c) is written.
+    const int qi = (warp - kMmaWarp) >> 1;
+    const bool pv_role = ((warp - kMmaWarp) & 1) != 0;
     if (qi < nq) {
-      constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
-      constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
-      const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
-      auto issue_pv = [&](int c) {
-        const int t = c >> 1, sl = c % NS;
-        ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
-        ptx::mbar_wait(&bar_v[t], 0);
-        ptx::tc_fence_after();
-        const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
-        const uint32_t v_addr = ptx::smem_u32(sV + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
-#pragma unroll
-        for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
-          ptx::mma_bf16_ts_w(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
-                             idesc_pv, (c | ks) != 0);
-        ptx::mma_commit_w(&pv_done[qi * NS + sl]);
-        if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&v_free[t & 1]);  // V tile t done for this q-tile
-        if (qi == 0 && c < 14 && lane == 0) atrace<TRACE>(48 + c);  // PV(0, c) issued
-      };
+      if (pv_role) {
+        constexpr uint32_t idesc_pv = ptx::idesc_bf16_f32_bmn(AQ, D);
 #pragma unroll 1
-      for (int c = 0; c < n_ch; ++c) {
-        const int t = c >> 1, sl = c % NS;
-        if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
-        ptx::mbar_wait(&bar_k[t], 0);
-        ptx::tc_fence_after();
-        const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
+        for (int c = 0; c < n_ch; ++c) {
+          const int t = c >> 1, sl = c % NS;
+          ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
+          ptx::mbar_wait(&bar_v[t], 0);
+          ptx::tc_fence_after();
+          const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
+          const uint32_t v_addr = ptx::smem_u32(sV + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
-        for (int k = 0; k < D / 16; ++k)
-          ptx::mma_bf16_ss_w(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
-                             ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
-        ptx::mma_commit_w(&s_full[qi * NS + sl]);
-        // K tile t is released (for this q-tile) once the S MMAs of both its chunks complete
-        if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&k_free[t & 1]);
-        if (qi == 0 && c < 16 && lane == 0) atrace<TRACE>(32 + c);  // S(0, c) issued
-        if (c > 0) issue_pv(c - 1);
+          for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
+            ptx::mma_bf16_ts_w(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
+                               idesc_pv, (c | ks) != 0);
+          ptx::mma_commit_w(&pv_done[qi * NS + sl]);
+          if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&v_free[t & 1]);  // V tile t done for this q-tile
+          if (qi == 0 && c < 14 && lane == 0) atrace<TRACE>(48 + c);  // PV(0, c) issued
+        }
+      } else {
+        constexpr uint32_t idesc_s = ptx::idesc_bf16_f32(AQ, KC);
+        const uint32_t q_addr = ptx::smem_u32(sQ + qi * kTileBytes);
+#pragma unroll 1
+        for (int c = 0; c < n_ch; ++c) {
+          const int t = c >> 1, sl = c % NS;
+          if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
+          ptx::mbar_wait(&bar_k[t], 0);
+          ptx::tc_fence_after();
+          const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
+#pragma unroll
+          for (int k = 0; k < D / 16; ++k)
+            ptx::mma_bf16_ss_w(tmem + qi * NS * KC + sl * KC, ptx::desc_k_sw128(q_addr + k * 32),
+                               ptx::desc_k_sw128(k_addr + k * 32), idesc_s, k > 0);
+          ptx::mma_commit_w(&s_full[qi * NS + sl]);
+          // K tile t is released (for this q-tile) once the S MMAs of both its chunks complete
+          if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&k_free[t & 1]);
+          if (qi == 0 && c < 16 && lane == 0) atrace<TRACE>(32 + c);  // S(0, c) issued
+        }
       }
-      issue_pv(n_ch - 1);
     }
   } else {
     // ----------------------------------------------------------------- softmax

@@ -57,6 +57,11 @@ __device__ __forceinline__ float ex2_approx(float x) {
 }
 
 __device__ __forceinline__ float gelu_erf_fast(float z) {
+#if defined(ARLO_GELU_EXPERIMENT)  // A/B only: tanh-form GELU, 1 MUFU (NOT the erf form; reading S2)
+  float th;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(th) : "f"(0.7978845608f * fmaf(0.044715f * z, z * z, z)));
+  return 0.5f * z * (1.0f + th);
+#else
   const float az = fabsf(z);
   const float t = rcp_approx(fmaf(az, 0.3275911f * 0.70710678118654752f, 1.0f));
   // coefficients pre-multiplied by 0.5
@@ -67,6 +72,7 @@ __device__ __forceinline__ float gelu_erf_fast(float z) {
   q *= t;
   const float e = ex2_approx(z * z * (-0.5f * 1.4426950408889634f));  // exp(-z^2/2) = exp(-a^2)
   return fmaxf(z, 0.0f) - az * q * e;
+#endif
 }
 
 // Pack two floats into a bf16x2 word (RNE), low half = a.

@@ -44,10 +44,23 @@ template <> struct Vec<float> {
   }
 };
 
+// gamma / beta are weights, independent of the predecessor kernel: every CTA stages them in
+// shared memory BEFORE the PDL wait, so their L2 round trip overlaps the previous kernel's tail
+// instead of sitting between the row statistics and the normalisation.
+__device__ __forceinline__ void stage_affine(int H, const float* __restrict__ g, const float* __restrict__ b,
+                                             float* sg, float* sb) {
+  for (int i = threadIdx.x * 4; i < H; i += blockDim.x * 4) {
+    *reinterpret_cast<float4*>(sg + i) = __ldg(reinterpret_cast<const float4*>(g + i));
+    *reinterpret_cast<float4*>(sb + i) = __ldg(reinterpret_cast<const float4*>(b + i));
+  }
+  __syncthreads();
+}
+
 // Normalise the row held in v[MAXV][VN] (only vectors lane + 32 i < nvec valid) and store it.
+// g, b point to the shared-memory copies of gamma / beta.
 template <typename T, int MAXV>
 __device__ __forceinline__ void ln_finish(float (&v)[MAXV][Vec<T>::N], int nvec, int H, int lane,
-                                          const float* __restrict__ g, const float* __restrict__ b,
+                                          const float* g, const float* b,
                                           float eps, T* __restrict__ out_row) {
   constexpr int VN = Vec<T>::N;
   float s = 0.f;
@@ -80,8 +93,8 @@ __device__ __forceinline__ void ln_finish(float (&v)[MAXV][Vec<T>::N], int nvec,
       float gg[VN], bb[VN], o[VN];
 #pragma unroll
       for (int j = 0; j < VN; j += 4) {
-        float4 g4 = __ldg(reinterpret_cast<const float4*>(g + c0 + j));
-        float4 b4 = __ldg(reinterpret_cast<const float4*>(b + c0 + j));
+        const float4 g4 = *reinterpret_cast<const float4*>(g + c0 + j);
+        const float4 b4 = *reinterpret_cast<const float4*>(b + c0 + j);
         gg[j] = g4.x; gg[j + 1] = g4.y; gg[j + 2] = g4.z; gg[j + 3] = g4.w;
         bb[j] = b4.x; bb[j + 1] = b4.y; bb[j + 2] = b4.z; bb[j + 3] = b4.w;
       }
@@ -98,7 +111,10 @@ __global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* _
                                                         const float* __restrict__ b, float eps,
                                                         T* __restrict__ out) {
   constexpr int VN = Vec<T>::N;
-  pdl_begin();
+  extern __shared__ float s_aff[];  // [gamma H | beta H]
+  pdl_launch_dependents();
+  stage_affine(H, g, b, s_aff, s_aff + H);
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
   if (row >= M) return;
@@ -108,7 +124,7 @@ __global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* _
 #pragma unroll
   for (int i = 0; i < MAXV; ++i)
     if (lane + 32 * i < nvec) Vec<T>::load(src + (lane + 32 * i) * VN, v[i]);
-  ln_finish<T, MAXV>(v, nvec, H, lane, g, b, eps, out + (size_t)row * H);
+  ln_finish<T, MAXV>(v, nvec, H, lane, s_aff, s_aff + H, eps, out + (size_t)row * H);
 }
 
 template <typename T, int MAXV>
@@ -122,7 +138,10 @@ __global__ void __launch_bounds__(256) embed_ln_kernel(int B, int L, int H, int 
                                                        const float* __restrict__ b, float eps,
                                                        T* __restrict__ out, int32_t* err_flag) {
   constexpr int VN = Vec<T>::N;
-  pdl_begin();
+  extern __shared__ float s_aff[];  // [gamma H | beta H]
+  pdl_launch_dependents();
+  stage_affine(H, g, b, s_aff, s_aff + H);
+  pdl_wait();
   const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
   if (row >= B * L) return;
@@ -151,7 +170,7 @@ __global__ void __launch_bounds__(256) embed_ln_kernel(int B, int L, int H, int 
       for (int j = 0; j < VN; ++j) v[i][j] = a[j] + p[j] + c[j];
     }
   }
-  ln_finish<T, MAXV>(v, nvec, H, lane, g, b, eps, out + (size_t)row * H);
+  ln_finish<T, MAXV>(v, nvec, H, lane, s_aff, s_aff + H, eps, out + (size_t)row * H);
 }
 
 }  // namespace
@@ -183,10 +202,10 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
   const int maxv = round_maxv(H / vn);
   dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
   if (dt == DT_BF16) {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, 0, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, 8 * H, s,
         M, H, (const bf16*)in, g, b, eps, (bf16*)out));
   } else {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<float, MV>, grid, block, 0, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<float, MV>, grid, block, 8 * H, s,
         M, H, (const float*)in, g, b, eps, (float*)out));
   }
   return cudaGetLastError();
@@ -202,11 +221,11 @@ cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int3
   const int maxv = round_maxv(H / vn);
   dim3 grid((B * L + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
   if (dt == DT_BF16) {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<bf16, MV>, grid, block, 0, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<bf16, MV>, grid, block, 8 * H, s,
         B, L, H, vocab, ids, lengths, (const bf16*)word, (const bf16*)pos, (const bf16*)type, g, b,
         eps, (bf16*)out, err_flag));
   } else {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<float, MV>, grid, block, 0, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<float, MV>, grid, block, 8 * H, s,
         B, L, H, vocab, ids, lengths, (const float*)word, (const float*)pos, (const float*)type, g,
         b, eps, (float*)out, err_flag));
   }

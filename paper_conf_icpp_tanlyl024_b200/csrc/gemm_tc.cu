@@ -92,11 +92,16 @@ struct TcCfg {
 // the warp's last TMEM load has completed.
 constexpr int CW = 32;  // chunk width: TMEM load / staging tile / TMA box (columns)
 
+#ifndef ARLO_EPI_DIRECT
+#define ARLO_EPI_DIRECT 0  // 1: store rows straight from registers instead of smem staging + TMA (A/B)
+#endif
+
 template <int BN, int EPI, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int ldr, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
-                                              uint8_t* stg, int& sc, Release release) {
+                                              uint8_t* stg, int& sc, Release release, bf16* __restrict__ outp,
+                                              int N) {
   static_assert(BN % CW == 0, "tile width must be a multiple of 32");
   constexpr int NCH = BN / CW;                                 // chunks per row block
   constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;  // chunks per warp (max)
@@ -152,6 +157,20 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       pk[2 * j] = pack_bf16x2(v0, v1);
       pk[2 * j + 1] = pack_bf16x2(v2, v3);
     }
+    if (ARLO_EPI_DIRECT) {
+      if (row_ok) {
+        uint4* o4 = reinterpret_cast<uint4*>(outp + (size_t)row * N + n0 + c * CW);
+#pragma unroll
+        for (int j = 0; j < CW / 8; ++j) o4[j] = make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+      }
+      ptx::tmem_wait_ld();
+      if (k == (nc >= 2 ? nc - 2 : 0)) {
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) release();
+      }
+      continue;
+    }
     // staging buffer sc % kStgBufs was last used kStgBufs chunks ago: make sure its TMA store has read it
     uint8_t* buf = stg + (sc % kStgBufs) * kStgBytes;
     if (sc >= kStgBufs) {
@@ -185,7 +204,7 @@ template <int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-               const bf16* __restrict__ resid, int ldr) {
+               const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
   using C = TcCfg<BN, false>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -294,7 +313,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
       epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg,
-                             sc, [te]() { ptx::mbar_arrive(te); });
+                             sc, [te]() { ptx::mbar_arrive(te); }, outp, N);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -321,7 +340,7 @@ template <int BN, int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-                    const bf16* __restrict__ resid, int ldr) {
+                    const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
   using C = TcCfg<BN, true>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -429,7 +448,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
       epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg, sc,
-                             [te]() { ptx::mbar_arrive_cluster(te); });
+                             [te]() { ptx::mbar_arrive_cluster(te); }, outp, N);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -895,7 +914,7 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
     attr_set = true;
   }
   return launch_k(kern, dim3(p.grid), dim3(kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias,
-                  (const bf16*)p.resid, p.ldr);
+                  (const bf16*)p.resid, p.ldr, (bf16*)p.out);
 }
 
 template <int BN, bool PAIR>

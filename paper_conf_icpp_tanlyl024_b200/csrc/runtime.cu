@@ -428,6 +428,11 @@ extern "C" int arlo_runtime_set_stream(arlo_runtime* rt, void* stream) {
 extern "C" int32_t arlo_runtime_length(const arlo_runtime* rt) { return rt ? rt->L : ARLO_EINVAL; }
 extern "C" int32_t arlo_runtime_max_batch(const arlo_runtime* rt) { return rt ? rt->max_batch : ARLO_EINVAL; }
 
+extern "C" int32_t arlo_runtime_bucket(const arlo_runtime* rt, int32_t n) {
+  if (!rt || n < 1 || n > rt->max_batch) return ARLO_EINVAL;
+  return rt->buckets[bucket_index(rt, n)].b;
+}
+
 extern "C" int32_t arlo_runtime_kernel_count(const arlo_runtime* rt, int32_t n) {
   if (!rt) return ARLO_EINVAL;
   int bi = bucket_index(rt, n < 1 ? 1 : n);

@@ -102,3 +102,207 @@ def replay(arlo, torch, runtimes: dict, cfg, n_requests: int, rate: float, seed:
                                              "demoted": float((runtime_of[m] != k).mean())}
     sched.close()
     return summary
+
+
+# ----------------------------------------------------------------------------------------------
+# Cluster replay: G GPUs, runtime instances placed by the Runtime Scheduler (arlo_allocate,
+# PAPER.md:L181-203 §3.3), one instance per GPU (no co-location, L155), requests routed by the
+# Request Scheduler (Algorithm 1).  Instances are independent replicas (north_star: no
+# collective), so a G-GPU cluster is simulated exactly by G virtual device clocks: every batch is
+# executed for real on this process's GPU (service_fn) and its measured device time advances the
+# clock of the virtual GPU that owns the instance.  Discrete-event simulation: arrivals and batch
+# completions are processed in time order, so Algorithm 1 sees the outstanding counts it would
+# see online.
+
+
+def slo_capacity(lat_ms_row, slo_ms: float) -> float:
+    """M_i ("maximum capacity within SLO"): the most requests one instance can finish
+    inside one SLO window while each of its batches meets the SLO: max_b b * floor(SLO / lat(b))
+    over the profiled batch sizes (reading of an unstated definition)."""
+    best = 0.0
+    for b, ms in enumerate(lat_ms_row, start=1):
+        if ms <= slo_ms:
+            best = max(best, b * np.floor(slo_ms / ms))
+    return max(best, 1.0)
+
+
+def plan_cluster(arlo, G: int, Ls, lat_ms, shares, rate: float, slo_ms: float):
+    """Runtime Scheduler inputs and decision for G GPUs.  lat_ms[i][b-1]: profiled forward latency
+    of runtime i at batch b; shares[i]: fraction of requests whose ideal runtime is i; rate: offered
+    req/s.  Q_i = requests per SLO window in bin i; M_i = slo_capacity.  Returns (N, Q, M)."""
+    lat = np.asarray(lat_ms, np.float64)
+    Q = np.asarray(shares, np.float64) * rate * slo_ms / 1e3
+    M = np.array([slo_capacity(row, slo_ms) for row in lat])
+    N, _obj = arlo.allocate(G, Q, M, lat)
+    return list(N), Q, M
+
+
+def simulate_cluster(arrivals, lengths, Ls, n_inst, capacity, service_fn, max_batch: int,
+                     sched_factory, lam: float = 0.85, alpha: float = 0.9, peek: int = 6):
+    """Discrete-event replay of requests (arrivals [s], lengths) on the instances n_inst[i] of
+    runtimes Ls[i] (each instance = one GPU).  service_fn(L, idx) -> seconds for a batch of request
+    indices idx on runtime L.  sched_factory(max_len, n_inst, capacity, lam, alpha, peek) builds the
+    Request Scheduler (arlo.Scheduler, or a test double).  Returns (done_s, runtime_of, busy_s)."""
+    import heapq
+    deployed = [k for k in range(len(Ls)) if n_inst[k] > 0]
+    dLs = [Ls[k] for k in deployed]
+    sched = sched_factory(dLs, [n_inst[k] for k in deployed], [float(capacity[k]) for k in deployed],
+                          lam, alpha, peek)
+    n = len(arrivals)
+    queues = {(r, j): collections.deque() for r in range(len(dLs)) for j in range(n_inst[deployed[r]])}
+    busy_until = {key: None for key in queues}
+    done = np.zeros(n)
+    runtime_of = np.zeros(n, np.int32)
+    inst_of = np.zeros(n, np.int32)
+    busy_s = {key: 0.0 for key in queues}
+    # (time, kind, seq, payload); at equal times: 0 completion, 1 arrival, 2 start of an idle instance
+    # (deferred so a batch takes every request that has arrived by its start time)
+    events = []
+    seq = 0
+    for i in range(n):
+        heapq.heappush(events, (float(arrivals[i]), 1, seq, i))
+        seq += 1
+
+    def start(key, t):
+        nonlocal seq
+        q = queues[key]
+        batch = [q.popleft() for _ in range(min(max_batch, len(q)))]
+        dt = service_fn(dLs[key[0]], batch)
+        busy_s[key] += dt
+        busy_until[key] = t + dt
+        heapq.heappush(events, (t + dt, 0, seq, (key, batch)))
+        seq += 1
+
+    while events:
+        t, kind, _s, payload = heapq.heappop(events)
+        if kind == 1:
+            i = payload
+            r, j = sched.dispatch(int(lengths[i]))
+            runtime_of[i], inst_of[i] = deployed[r], j
+            queues[(r, j)].append(i)
+            if busy_until[(r, j)] is None:
+                busy_until[(r, j)] = t  # start pending
+                heapq.heappush(events, (t, 2, seq, (r, j)))
+                seq += 1
+        elif kind == 2:
+            start(payload, t)
+        else:
+            key, batch = payload
+            for i in batch:
+                done[i] = t
+                sched.complete(key[0], key[1])
+            busy_until[key] = None
+            if queues[key]:
+                start(key, t)
+    sched.close()
+    return done, runtime_of, inst_of, busy_s
+
+
+def summarize(arrivals, lengths, done, runtime_of, Ls, slo_ms: float):
+    lat_ms = (done - arrivals) * 1e3
+    span = float(done.max() - arrivals.min())
+    out = {"requests": int(len(arrivals)), "served_rate": float(len(arrivals) / span), "makespan_s": span,
+           "mean_ms": float(lat_ms.mean()), "p98_ms": float(np.percentile(lat_ms, 98)),
+           "p99_ms": float(np.percentile(lat_ms, 99)), "slo_violations": float((lat_ms > slo_ms).mean()),
+           "per_bucket": {}}
+    ideal = wl.ideal_runtime(lengths, Ls)
+    for k, L in enumerate(Ls):
+        m = ideal == k
+        if m.any():
+            out["per_bucket"][str(L)] = {"requests": int(m.sum()), "mean_ms": float(lat_ms[m].mean()),
+                                         "p99_ms": float(np.percentile(lat_ms[m], 99)),
+                                         "demoted": float((runtime_of[m] != k).mean())}
+    return out
+
+
+def profile_runtimes(torch, runtimes: dict, cfg, max_batch: int, stream, reps: int = 5):
+    """lat_ms[i][b-1], b = 1..max_batch: device time of one forward (a batch of b pads to the
+    runtime's bucket, so b is timed at every bucket size and assigned to the b it covers)."""
+    dev = torch.device("cuda")
+    table = []
+    for L in sorted(runtimes):
+        rt = runtimes[L]
+        row = [0.0] * max_batch
+        lens = np.full(max_batch, L, np.int32)
+        ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
+        ld = torch.from_numpy(lens).to(dev)
+        out = torch.empty((max_batch, cfg.num_labels), device=dev)
+        cache = {}
+        for b in range(1, max_batch + 1):
+            bucket = rt.bucket_of(b)
+            if bucket not in cache:
+                for _ in range(2):
+                    rt.enqueue(bucket, ids, ld, out)
+                ev = []
+                for _ in range(reps):
+                    a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                    a.record(stream)
+                    rt.enqueue(bucket, ids, ld, out)
+                    e.record(stream)
+                    ev.append((a, e))
+                torch.cuda.synchronize()
+                cache[bucket] = float(np.median([a.elapsed_time(e) for a, e in ev]))
+            row[b - 1] = cache[bucket]
+        table.append(row)
+    return table
+
+
+def cluster_replay(arlo, torch, runtimes: dict, cfg, Gs=(1, 2, 4, 8), n_requests: int = 8000,
+                   slo_ms: float = 150.0, max_batch: int = 32, stream=None, load: float = 0.7):
+    """Aggregate req/s and latency of Arlo (ILP placement + Algorithm 1 over len(runtimes) runtimes)
+    and of ST (every GPU an L = max runtime instance) on G = 1, 2, 4, 8 GPUs.
+    Saturation replay (all requests at t = 0) gives req/s; a Poisson replay at `load` x that
+    rate gives mean / p98 / p99 latency.  Service times are real forwards on this GPU."""
+    Ls = sorted(runtimes)
+    dev = torch.device("cuda")
+    lat = profile_runtimes(torch, runtimes, cfg, max_batch, stream)
+    lengths = wl.sample_lengths(n_requests, seed=wl.SEED_ARRIVALS + 1)
+    ids_all = wl.sample_token_ids(cfg, lengths, max(Ls), seed=wl.SEED_ARRIVALS + 2)
+    ideal = wl.ideal_runtime(lengths, Ls)
+    shares = [float((ideal == k).mean()) for k in range(len(Ls))]
+    caps = [slo_capacity(row, slo_ms) for row in lat]
+    bufs = {L: (torch.empty((max_batch, L), dtype=torch.int32, device=dev),
+                torch.empty((max_batch,), dtype=torch.int32, device=dev)) for L in Ls}
+    out = torch.empty((max_batch, cfg.num_labels), device=dev)
+
+    def service(L, batch):
+        n = len(batch)
+        ids_d, len_d = bufs[L]
+        ids_d[:n].copy_(torch.from_numpy(np.ascontiguousarray(ids_all[batch, :L])))
+        len_d[:n].copy_(torch.from_numpy(lengths[batch].astype(np.int32)))
+        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        runtimes[L].enqueue(n, ids_d, len_d, out)
+        e.record(stream)
+        e.synchronize()
+        return a.elapsed_time(e) / 1e3
+
+    def factory(max_len, n_inst, capacity, lam, alpha, peek):
+        return arlo.Scheduler(max_len, n_inst, capacity, lam, alpha, peek)
+
+    def run(n_inst, arrivals):
+        done, rof, _inst, busy = simulate_cluster(arrivals, lengths, Ls, n_inst, caps, service, max_batch, factory)
+        return summarize(arrivals, lengths, done, rof, Ls, slo_ms)
+
+    res = {"runtimes": Ls, "requests": n_requests, "slo_ms": slo_ms, "capacity_per_slo_window": caps,
+           "profile_ms": {str(L): {str(b): round(lat[k][b - 1], 4) for b in (1, 2, 4, 8, 16, 32) if b <= max_batch}
+                          for k, L in enumerate(Ls)}, "per_G": {}}
+    zero = np.zeros(n_requests)
+    for G in Gs:
+        st = [0] * (len(Ls) - 1) + [G]
+        st_sat = run(st, zero)
+        # plan Arlo at the load the ST deployment saturates at x 2 (re-planned below at its own rate)
+        N, Q, M = plan_cluster(arlo, G, Ls, lat, shares, 2.0 * st_sat["served_rate"], slo_ms)
+        arlo_sat = run(N, zero)
+        N, Q, M = plan_cluster(arlo, G, Ls, lat, shares, load * arlo_sat["served_rate"], slo_ms)
+        arlo_sat = run(N, zero)
+        rate = load * arlo_sat["served_rate"]
+        arr = wl.poisson_arrivals(n_requests, rate, seed=wl.SEED_ARRIVALS)
+        arlo_lat = run(N, arr)
+        st_lat = run(st, wl.poisson_arrivals(n_requests, load * st_sat["served_rate"], seed=wl.SEED_ARRIVALS))
+        res["per_G"][str(G)] = {
+            "arlo": {"instances": {str(L): int(N[k]) for k, L in enumerate(Ls)},
+                     "saturation_req_s": arlo_sat["served_rate"], "poisson": arlo_lat},
+            "st512": {"saturation_req_s": st_sat["served_rate"], "poisson": st_lat},
+            "speedup_saturation": arlo_sat["served_rate"] / st_sat["served_rate"]}
+    return res

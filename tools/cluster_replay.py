@@ -1,0 +1,35 @@
+"""Cluster replay only (BASELINE configs[3] / [4]): ILP-placed runtimes on G virtual GPUs.
+
+    python tools/cluster_replay.py [base|roberta] [n_requests]
+"""
+import json
+import os
+import sys
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_icpp_tanlyl024_b200 import arlo, replay  # noqa: E402
+from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
+
+
+def main():
+    model = sys.argv[1] if len(sys.argv) > 1 else "base"
+    n = int(sys.argv[2]) if len(sys.argv) > 2 else 6000
+    cfg = wl.ROBERTA_LARGE if model == "roberta" else wl.BERT_BASE
+    slo = 450.0 if model == "roberta" else 150.0  # PAPER.md:L297 (R uses the BERT-large SLO)
+    dev = torch.device("cuda")
+    s = torch.cuda.Stream()
+    W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg), arlo.BF16, dev), arlo.BF16)
+    rts = {}
+    for L in wl.RUNTIME_LENGTHS:
+        rts[L] = arlo.Runtime(W, L, 32)
+        rts[L].set_stream(s)
+    Gs = (8,) if model == "roberta" else (1, 2, 4, 8)
+    res = replay.cluster_replay(arlo, torch, rts, cfg, Gs=Gs, n_requests=n, slo_ms=slo, max_batch=32, stream=s)
+    res["model"] = cfg.name
+    print(json.dumps(res))
+
+
+if __name__ == "__main__":
+    main()
