@@ -291,6 +291,15 @@ def main():
     if rank == 0 and not args.no_extras:
         result["roofline"] = roofline_dominant(arlo, torch, dev, stream, step_times)
         result["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
+        result["per_L_latency_ms_restricted"] = per_L_table(runtimes, torch, dev, stream, cfg, restricted=True)
+        pl = result["per_L_latency_ms"]
+        result["paper_context"] = {
+            "note": "context only: RTX 3090, FP32 TensorRT static shape, batch 1 (BASELINE.md section 1)",
+            "bert_base_L512_b1_ms": {"paper_rtx3090": 4.86, "this_b200_bf16": pl["512"]["1"]["median"],
+                                     "source": "PAPER.md:L101 (Fig. 2a)"},
+            "latency_ratio_L512_over_L64_b1": {"paper_rtx3090": 4.22,
+                                               "this_b200_bf16": pl["512"]["1"]["median"] / pl["64"]["1"]["median"],
+                                               "source": "PAPER.md:L95"}}
         result["uniform_512"] = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
         result["e2e"] = e2e_res
         result["bert_large"] = bert_large_per_L(arlo, torch, dev, stream, local_rank)
@@ -366,7 +375,7 @@ def bert_large_per_L(arlo, torch, dev, stream, device_index):
         rt = arlo.Runtime(W, L, 64)
         rt.set_stream(stream)
         row = {}
-        for b in (1, 16, 64):
+        for b in (1, 4, 16, 32, 64):
             lens = np.full(b, L, np.int32)
             ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
             ld = torch.from_numpy(lens).to(dev)
@@ -443,13 +452,16 @@ def roofline_dominant(arlo, torch, dev, stream, step_times):
             "algorithmic_flops_per_launch": flops}
 
 
-def per_L_table(runtimes, torch, dev, stream, cfg):
-    """Offline-profiler table (A4): latency of one forward vs batch bucket for every runtime."""
+def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False):
+    """Offline-profiler table (A4): latency of one forward vs batch bucket for every runtime.
+    restricted=False: every request has length L (roofline mode, SURVEY 8(d)(i));
+    restricted=True: lengths drawn from the skewed distribution restricted to (L-64, L] (8(d)(ii)),
+    where attention skips the key chunks past each request's length."""
     table = {}
     for L, rt in runtimes.items():
         row = {}
-        for b in (1, 2, 4, 8, 16, 32):
-            lens = np.full(b, L, np.int32)
+        for b in ((1, 8, 32) if restricted else (1, 2, 4, 8, 16, 32)):
+            lens = (wl.sample_lengths(b, seed=7 + b, lo=L - 64, hi=L) if restricted else np.full(b, L)).astype(np.int32)
             ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
             ld = torch.from_numpy(lens).to(dev)
             out = torch.empty((b, cfg.num_labels), device=dev)
@@ -462,7 +474,10 @@ def per_L_table(runtimes, torch, dev, stream, cfg):
                 e.record(stream)
             torch.cuda.synchronize()
             ts = [a.elapsed_time(e) for a, e in ev]
-            row[str(b)] = {"median": float(np.median(ts)), "tflops": metrics.forward_flops(cfg, b, L) / (np.median(ts) / 1e3) / 1e12}
+            row[str(b)] = {"median": float(np.median(ts)),
+                           "tflops": metrics.forward_flops(cfg, b, L) / (np.median(ts) / 1e3) / 1e12}
+            if restricted:
+                row[str(b)]["mean_len"] = float(lens.mean())
         table[str(L)] = row
     return table
 

@@ -242,12 +242,23 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_begin();  // setup above overlapped the previous kernel's tail
-  if (threadIdx.x == 0) trace(0);
+  pdl_launch_dependents();  // setup above overlapped the previous kernel's tail
 
   if (warp == kProducerWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
+      // W never depends on the previous kernel: the first tile's first STAGES W
+      // tiles are requested before the PDL wait, its A tiles right after it
+      const int pre = blockIdx.x < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
+      {
+        const int n0 = (blockIdx.x / num_m) * BN;
+        for (int kb = 0; kb < pre; ++kb) {
+          ptx::mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
+          ptx::tma_load_2d(sB + kb * C::B_BYTES, &tmB, &full[kb], kb * BK, n0);
+        }
+      }
+      pdl_wait();
+      if (threadIdx.x == kProducerWarp * 32) trace(0);
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
@@ -255,16 +266,23 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
         trace(2 + 6 * it);
         for (int kb = 0; kb < kblocks; ++kb) {
-          ptx::mbar_wait(&empty[stage], phase ^ 1);
-          ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
-          ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
-          ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          if (it == 0 && kb < pre) {
+            ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
+          } else {
+            ptx::mbar_wait(&empty[stage], phase ^ 1);
+            ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+            ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
+            ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          }
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
     }
   } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------- MMA issuer
+    pdl_wait();
     if (lane == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
       int stage = 0;
@@ -300,6 +318,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     // --------------------------------------------------------------- epilogue
     // warp w may only touch TMEM lanes 32*(w%4)..+31 (rows of the tile); the
     // two warps sharing a quarter take one column half each.
+    pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
     uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0;
@@ -380,29 +399,51 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   ptx::cluster_sync();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_begin();  // setup above overlapped the previous kernel's tail
-  if (threadIdx.x == 0) trace(0);
+  pdl_launch_dependents();  // setup above overlapped the previous kernel's tail
 
   if (warp == kProducerWarp) {
     if (lane == 0) {
+      // W tiles of the first tile are requested before the PDL wait (see gemm_tc_kernel)
+      const int pre = pair < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
+      {
+        const int n0 = (pair / num_m) * BN + rank * C::B_ROWS;
+        for (int kb = 0; kb < pre; ++kb) {
+          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[kb], 2 * C::STAGE_BYTES);
+          ptx::tma_load_2d_pair(sB + kb * C::B_BYTES, &tmB, ptx::mapa_shared(&full[kb], 0), kb * BK, n0);
+        }
+      }
+      pdl_wait();
+      if (threadIdx.x == kProducerWarp * 32) trace(0);
       int stage = 0;
       uint32_t phase = 0;
       int it = 0;
       for (int tile = pair; tile < tiles; tile += npairs, ++it) {
         trace(2 + 6 * it);
+#if defined(ARLO_GEMM_SAME_TILE)  // bandwidth experiment only (wrong results): every pair loads tile 0
+        const int m0 = rank * BM;
+        const int n0 = rank * C::B_ROWS;
+#else
         const int m0 = (tile % num_m) * 2 * BM + rank * BM;
         const int n0 = (tile / num_m) * BN + rank * C::B_ROWS;
+#endif
         for (int kb = 0; kb < kblocks; ++kb) {
-          ptx::mbar_wait(&empty[stage], phase ^ 1);
-          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
           const uint32_t fb = ptx::mapa_shared(&full[stage], 0);
-          ptx::tma_load_2d_pair(sA + stage * C::A_BYTES, &tmA, fb, kb * BK, m0);
-          ptx::tma_load_2d_pair(sB + stage * C::B_BYTES, &tmB, fb, kb * BK, n0);
+          if (it == 0 && kb < pre) {
+            ptx::tma_load_2d_pair(sA + stage * C::A_BYTES, &tmA, fb, kb * BK, m0);
+          } else {
+            ptx::mbar_wait(&empty[stage], phase ^ 1);
+            if (rank == 0) ptx::mbar_arrive_expect_tx(&full[stage], 2 * C::STAGE_BYTES);
+            ptx::tma_load_2d_pair(sA + stage * C::A_BYTES, &tmA, fb, kb * BK, m0);
+            ptx::tma_load_2d_pair(sB + stage * C::B_BYTES, &tmB, fb, kb * BK, n0);
+          }
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
     }
   } else if (warp == kMmaWarp) {
+    pdl_wait();
     if (lane == 0 && rank == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(2 * BM, BN);
       int stage = 0;
@@ -435,6 +476,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       }
     }
   } else {
+    pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
     uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0;
