@@ -283,7 +283,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   } else if (warp == kMmaWarp) {
     // ------------------------------------------------------------- MMA issuer
     pdl_wait();
-    if (lane == 0) {
+    {  // converged warp, elected lane issues (see gemm_tc_pair_kernel)
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
       int stage = 0;
       uint32_t phase = 0;
@@ -293,24 +293,24 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
         ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
-        trace(3 + 6 * it);
+        if (lane == 0) trace(3 + 6 * it);
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < kblocks; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
-          if (kb == 0) trace(4 + 6 * it);
+          if (kb == 0 && lane == 0) trace(4 + 6 * it);
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
-            ptx::mma_bf16_ss(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
-                             ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
+            ptx::mma_bf16_ss_w(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
+                               ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
           }
-          ptx::mma_commit(&empty[stage]);
+          ptx::mma_commit_w(&empty[stage]);
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
-        ptx::mma_commit(&tfull[acc]);
-        trace(5 + 6 * it);
+        ptx::mma_commit_w(&tfull[acc]);
+        if (lane == 0) trace(5 + 6 * it);
         if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
       }
     }
@@ -444,7 +444,10 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     }
   } else if (warp == kMmaWarp) {
     pdl_wait();
-    if (lane == 0 && rank == 0) {
+    // the whole (converged) MMA warp runs the issue loop and one elected lane issues:
+    // a lone lane of a diverged warp pays ~1/3 more per tcgen05.mma (tools/mma_bench.cu),
+    // which measured 16.1 -> 12.3 us on the FFN2 mainloop at M = 4096
+    if (rank == 0) {
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(2 * BM, BN);
       int stage = 0;
       uint32_t phase = 0;
@@ -454,24 +457,24 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       for (int tile = pair; tile < tiles; tile += npairs, ++it) {
         ptx::mbar_wait(&tempty[acc], acc_phase ^ 1);
         ptx::tc_fence_after();
-        trace(3 + 6 * it);
+        if (lane == 0) trace(3 + 6 * it);
         const uint32_t d_tmem = tmem_base + acc * BN;
         for (int kb = 0; kb < kblocks; ++kb) {
           ptx::mbar_wait(&full[stage], phase);
           ptx::tc_fence_after();
-          if (kb == 0) trace(4 + 6 * it);
+          if (kb == 0 && lane == 0) trace(4 + 6 * it);
           const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k) {
-            ptx::mma_bf16_ss_pair(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
-                                  ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
+            ptx::mma_bf16_ss_pair_w(d_tmem, ptx::desc_k_sw128(a_addr + k * 32),
+                                    ptx::desc_k_sw128(b_addr + k * 32), idesc, (kb | k) != 0);
           }
-          ptx::mma_commit_pair(&empty[stage]);
+          ptx::mma_commit_pair_w(&empty[stage]);
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
-        ptx::mma_commit_pair(&tfull[acc]);
-        trace(5 + 6 * it);
+        ptx::mma_commit_pair_w(&tfull[acc]);
+        if (lane == 0) trace(5 + 6 * it);
         if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
       }
     }
@@ -589,25 +592,28 @@ gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
       }
     }
   } else if (warp == 5) {
+    // the whole (converged) warp runs the issue loop and one elected lane issues each
+    // MMA: ~1/3 cheaper per instruction than a lone lane of a diverged warp
+    // (tools/mma_bench.cu), which matters here because a BN = 16 MMA is only 8 tensor
+    // cycles and the K chain is issue-bound
     pdl_begin();
-    if (lane == 0) {
-      constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
-      int stage = 0;
-      uint32_t phase = 0;
-      for (int kb = 0; kb < kblocks; ++kb) {
-        ptx::mbar_wait(&full[stage], phase);
-        ptx::tc_fence_after();
-        const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
-        const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
+    constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
+    int stage = 0;
+    uint32_t phase = 0;
+#pragma unroll 1
+    for (int kb = 0; kb < kblocks; ++kb) {
+      ptx::mbar_wait(&full[stage], phase);
+      ptx::tc_fence_after();
+      const uint32_t a_addr = ptx::smem_u32(sA + stage * C::A_BYTES);
+      const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
-        for (int k = 0; k < BK / 16; ++k)
-          ptx::mma_bf16_ss(tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32), idesc,
+      for (int k = 0; k < BK / 16; ++k)
+        ptx::mma_bf16_ss_w(tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32), idesc,
                            (kb | k) != 0);
-        ptx::mma_commit(&empty[stage]);
-        if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
-      }
-      ptx::mma_commit(tfull);
+      ptx::mma_commit_w(&empty[stage]);
+      if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
     }
+    ptx::mma_commit_w(tfull);
   } else {
     pdl_begin();
     // epilogue: thread = row (TMEM lane), BN columns, straight 16-byte stores
@@ -875,7 +881,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else if (warp == kMmaWarp) {
-    if (lane == 0) {
+    {  // converged warp, elected lane issues
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
       int stage = 0;
       uint32_t phase = 0;
@@ -892,12 +898,12 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           const uint32_t b_addr = ptx::smem_u32(sB + stage * C::B_BYTES);
 #pragma unroll
           for (int k = 0; k < BK / 16; ++k)
-            ptx::mma_bf16_ss(d_tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32), idesc,
-                             (kb | k) != 0);
-          ptx::mma_commit(&empty[stage]);
+            ptx::mma_bf16_ss_w(d_tmem, ptx::desc_k_sw128(a_addr + k * 32), ptx::desc_k_sw128(b_addr + k * 32),
+                               idesc, (kb | k) != 0);
+          ptx::mma_commit_w(&empty[stage]);
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
-        ptx::mma_commit(&tfull[acc]);
+        ptx::mma_commit_w(&tfull[acc]);
         if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
       }
     }
