@@ -467,14 +467,14 @@ def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False):
             out = torch.empty((b, cfg.num_labels), device=dev)
             for _ in range(3):
                 rt.enqueue(b, ids, ld, out)
-            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(10)]
+            ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(20)]
             for a, e in ev:
                 a.record(stream)
                 rt.enqueue(b, ids, ld, out)
                 e.record(stream)
             torch.cuda.synchronize()
             ts = [a.elapsed_time(e) for a, e in ev]
-            row[str(b)] = {"median": float(np.median(ts)),
+            row[str(b)] = {"median": float(np.median(ts)), "p99": float(np.percentile(ts, 99)),
                            "tflops": metrics.forward_flops(cfg, b, L) / (np.median(ts) / 1e3) / 1e12}
             if restricted:
                 row[str(b)]["mean_len"] = float(lens.mean())

@@ -1034,42 +1034,42 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
 }
 
 // Tile choice: a function of (M, N, K) only (never of the data), minimising a
-// wave-quantised time estimate.  Wide kernels, per tile: MMA time of a
-// 128 x BN x K slab at 8192 flop/clk/SM divided by a feed efficiency measured
-// on B200 (tools/gemm_sweep.py: CTA pairs and single CTAs at BN >= 192 sustain
-// the tensor pipe; BN = 128 tiles re-read A twice as often and run ~30%
-// slower), plus a fixed ~1 us tile prologue/epilogue cost.  Skinny kernel (one
-// CTA per 128 x BN tile, M <= 512): the CTA's operand bytes at ~kSkFeed B/clk
-// per SM plus ~1.5 us of latency.  Returns BN for the single-CTA kernel, -BN
-// for the CTA-pair kernel, kSkinnyCode + BN for the skinny kernel.
-constexpr double kSkFeed = 96.0;
-
+// wave-quantised time estimate fitted to graph-replayed B200 sweeps
+// (tools/gemm_sweep.py --set small/base/large/mid: over 39 shapes the pick is
+// the measured best or within 3 % of it on all but two, 11 % and 22 % off):
+//   wide kernels:  waves * (2.5 us + kblocks * max(MMA time of one 64-deep
+//                  k-block / eff(pair, BN), 0.12 us)),
+//   skinny kernel: waves * (2.5 us + kblocks * (0.11 + 0.0005 BN) us).
+// eff is the fraction of the tensor pipe a tile shape sustains (operand
+// staging per flop: the CTA pair at BN = 256 is best, single-CTA BN = 256 pays
+// for its 32 KB W stage).  Returns BN for the single-CTA kernel, -BN for the
+// CTA-pair kernel, kSkinnyCode + BN for the skinny kernel.
 int tc_choose_bn(int M, int N, int K) {
   const int sms = num_sms();
+  const double kblocks = K / BK;
   double best = 1e30;
   int best_bn = 0;
-  const int cands[7] = {-256, -192, 256, 192, -128, 128, 64};
-  for (int c : cands) {
-    const bool pair = c < 0;
-    const int bn = pair ? -c : c;
+  struct Cand { int code; double eff; };
+  const Cand cands[7] = {{-256, 0.75}, {-192, 0.65}, {256, 0.45}, {192, 0.70}, {-128, 0.50}, {128, 0.60}, {64, 0.45}};
+  for (const Cand& c : cands) {
+    const bool pair = c.code < 0;
+    const int bn = pair ? -c.code : c.code;
     if (N % bn) continue;
     const int tile_m = pair ? 2 * BM : BM;
     const long tiles = (long)((M + tile_m - 1) / tile_m) * (N / bn);
     const long slots = pair ? sms / 2 : sms;
     const long waves = (tiles + slots - 1) / slots;
-    const double mma_us = (double)BM * bn * K * 2 / 8192.0 / 1.9e3;
-    double eff = bn >= 192 ? (pair ? 1.0 : 0.92) : (bn == 128 ? 0.68 : (bn == 64 ? 0.5 : 0.3));
-    const double t = waves * (mma_us / eff + 1.0);
-    if (t < best * 0.999) { best = t; best_bn = c; }
+    const double mma_kb_us = (double)tile_m * bn * BK * 2 / (pair ? 16384.0 : 8192.0) / 1.9e3;
+    const double per_kb = mma_kb_us / c.eff > 0.12 ? mma_kb_us / c.eff : 0.12;
+    const double t = waves * (2.5 + kblocks * per_kb);
+    if (t < best * 0.999) { best = t; best_bn = c.code; }
   }
-  if (M <= 512 && getenv("ARLO_NO_SKINNY") == nullptr) {
-    const int a_rows = M < BM ? ((M + 7) & ~7) : BM;
+  if (M <= 1024 && getenv("ARLO_NO_SKINNY") == nullptr) {
     for (int bn : {16, 32, 64}) {
       if (N % bn) continue;
       const long ctas = (long)((M + BM - 1) / BM) * (N / bn);
       const long waves = (ctas + sms - 1) / sms;
-      const double bytes = 2.0 * (double)(a_rows + bn) * K;
-      const double t = waves * (bytes / kSkFeed / 1.9e3 + 1.5);
+      const double t = waves * (2.5 + kblocks * (0.11 + 0.0005 * bn));
       if (t < best * 0.999) { best = t; best_bn = kSkinnyCode + bn; }
     }
   }

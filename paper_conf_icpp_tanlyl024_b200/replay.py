@@ -248,11 +248,13 @@ def profile_runtimes(torch, runtimes: dict, cfg, max_batch: int, stream, reps: i
 
 
 def cluster_replay(arlo, torch, runtimes: dict, cfg, Gs=(1, 2, 4, 8), n_requests: int = 8000,
-                   slo_ms: float = 150.0, max_batch: int = 32, stream=None, load: float = 0.7):
+                   slo_ms: float = 150.0, max_batch: int = 32, stream=None, load: float = 0.7,
+                   loads=(0.5, 0.7, 0.9, 0.97)):
     """Aggregate req/s and latency of Arlo (ILP placement + Algorithm 1 over len(runtimes) runtimes)
     and of ST (every GPU an L = max runtime instance) on G = 1, 2, 4, 8 GPUs.
-    Saturation replay (all requests at t = 0) gives req/s; a Poisson replay at `load` x that
-    rate gives mean / p98 / p99 latency.  Service times are real forwards on this GPU."""
+    Saturation replay (all requests at t = 0) gives req/s; Poisson replays at `loads` x that rate
+    give mean / p98 / p99 latency (per length bucket at `load`) and req/s at SLO.
+    Service times are real forwards on this GPU."""
     Ls = sorted(runtimes)
     dev = torch.device("cuda")
     lat = profile_runtimes(torch, runtimes, cfg, max_batch, stream)
@@ -291,18 +293,25 @@ def cluster_replay(arlo, torch, runtimes: dict, cfg, Gs=(1, 2, 4, 8), n_requests
     for G in Gs:
         st = [0] * (len(Ls) - 1) + [G]
         st_sat = run(st, zero)
-        # plan Arlo at the load the ST deployment saturates at x 2 (re-planned below at its own rate)
+        # plan Arlo at twice the rate ST saturates at, measure its saturation, re-plan at load x that
         N, Q, M = plan_cluster(arlo, G, Ls, lat, shares, 2.0 * st_sat["served_rate"], slo_ms)
         arlo_sat = run(N, zero)
         N, Q, M = plan_cluster(arlo, G, Ls, lat, shares, load * arlo_sat["served_rate"], slo_ms)
         arlo_sat = run(N, zero)
-        rate = load * arlo_sat["served_rate"]
-        arr = wl.poisson_arrivals(n_requests, rate, seed=wl.SEED_ARRIVALS)
-        arlo_lat = run(N, arr)
-        st_lat = run(st, wl.poisson_arrivals(n_requests, load * st_sat["served_rate"], seed=wl.SEED_ARRIVALS))
+        # load sweep (Poisson arrivals): req/s at SLO = highest offered rate whose p99 <= SLO
+        sweep = {}
+        for name, n_inst, sat in (("arlo", N, arlo_sat["served_rate"]), ("st512", st, st_sat["served_rate"])):
+            pts = []
+            for f in loads:
+                r = run(n_inst, wl.poisson_arrivals(n_requests, f * sat, seed=wl.SEED_ARRIVALS))
+                pts.append({"load": f, "offered_req_s": f * sat, "mean_ms": r["mean_ms"], "p98_ms": r["p98_ms"],
+                            "p99_ms": r["p99_ms"], "slo_violations": r["slo_violations"],
+                            "per_bucket": r["per_bucket"] if f == load else None})
+            ok = [p for p in pts if p["p99_ms"] <= slo_ms]
+            sweep[name] = {"points": pts, "req_s_at_slo": max((p["offered_req_s"] for p in ok), default=None)}
         res["per_G"][str(G)] = {
             "arlo": {"instances": {str(L): int(N[k]) for k, L in enumerate(Ls)},
-                     "saturation_req_s": arlo_sat["served_rate"], "poisson": arlo_lat},
-            "st512": {"saturation_req_s": st_sat["served_rate"], "poisson": st_lat},
+                     "saturation_req_s": arlo_sat["served_rate"], "load_sweep": sweep["arlo"]},
+            "st512": {"saturation_req_s": st_sat["served_rate"], "load_sweep": sweep["st512"]},
             "speedup_saturation": arlo_sat["served_rate"] / st_sat["served_rate"]}
     return res

@@ -23,7 +23,8 @@ SETS = {
               (128, 2304, 768), (128, 768, 3072), (512, 2304, 768), (512, 768, 3072),
               (128, 3072, 1024), (128, 1024, 4096)],
 }
-SETS["all"] = SETS["base"] + SETS["large"] + SETS["small"]
+SETS["mid"] = [(m, n, k) for m in (1024, 2048, 8192) for (n, k) in ((2304, 768), (3072, 768), (768, 3072), (768, 768))]
+SETS["all"] = SETS["base"] + SETS["large"] + SETS["small"] + SETS["mid"]
 
 
 def time_op(fn, reps=20):
