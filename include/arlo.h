@@ -196,6 +196,15 @@ void arlo_sched_destroy(arlo_sched* s);
  */
 int arlo_dispatch(arlo_sched* s, int32_t length, int32_t* runtime_out, int32_t* instance_out);
 
+/* Dispatch policy (the Table 4 ablation): ARLO_DISPATCH_RS =
+ * Algorithm 1 (default); ARLO_DISPATCH_ILB = Intra-group Load Balance: the
+ * runtime requiring the least padding, its least-loaded instance;
+ * ARLO_DISPATCH_IG = Inter-groups Greedy: the least busy head instance among
+ * ALL candidate runtimes (fewest outstanding requests, ties to the smaller
+ * max_length; peek is ignored).  Errors: EINVAL. */
+enum { ARLO_DISPATCH_RS = 0, ARLO_DISPATCH_ILB = 1, ARLO_DISPATCH_IG = 2 };
+int arlo_sched_set_policy(arlo_sched* s, int32_t policy);
+
 /* Replace lambda, alpha and peek of an existing scheduler (state is kept).
  * Errors: EINVAL (peek < 1). */
 int arlo_sched_set_params(arlo_sched* s, double lambda, double alpha, int32_t peek);

@@ -77,6 +77,34 @@ def dispatch(q: MultiLevelQueue, length: int, lam: float, alpha: float, peek: in
     return chosen, inst
 
 
+def dispatch_ilb(q: MultiLevelQueue, length: int):
+    """ILB, "Intra-group Load Balance" (Table 4 baseline): the runtime
+    requiring the least padding, i.e. the first candidate, and its least-loaded instance."""
+    Qe = candidate_runtimes(q, length)
+    if not Qe:
+        return None
+    chosen = Qe[0]
+    inst, _, _ = q.front(chosen)
+    q.outstanding[chosen][inst] += 1
+    return chosen, inst
+
+
+def dispatch_ig(q: MultiLevelQueue, length: int):
+    """IG, "Inter-groups Greedy": the least busy instance among all
+    candidate runtime queues.  Reading S20: least busy = fewest outstanding requests;
+    ties go to the smaller max_length (less padding), then the lower instance id."""
+    Qe = candidate_runtimes(q, length)
+    if not Qe:
+        return None
+    best = None
+    for i in Qe:                              # every candidate, ascending max_length
+        inst, N, _ = q.front(i)
+        if best is None or N < best[2]:
+            best = (i, inst, N)
+    q.outstanding[best[0]][best[1]] += 1
+    return best[0], best[1]
+
+
 def complete(q: MultiLevelQueue, runtime: int, instance: int):
     """A request finished: the instance's outstanding count drops by one."""
     q.outstanding[runtime][instance] -= 1

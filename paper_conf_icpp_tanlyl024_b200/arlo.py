@@ -26,13 +26,14 @@ lib = C.CDLL(LIB_PATH)
 
 OK, EINVAL, ETOOLONG, ENOMEM, ECUDA, EINFEASIBLE, ENOCAND, ENODEV = 0, -1, -2, -3, -4, -5, -6, -7
 BF16, FP32 = 0, 1
+DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
 
 EXPORTED = [
     "arlo_last_error", "arlo_version", "arlo_weights_count", "arlo_weights_create", "arlo_weights_destroy",
     "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
-    "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
+    "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_sched_set_policy", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
     "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
     "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
 ]
@@ -69,6 +70,7 @@ _sig("arlo_infer", C.c_int, _vp, _vp, _vp, _vp)
 _sig("arlo_enqueue", C.c_int, _vp, _i32, _vp, _vp, _vp)
 _sig("arlo_runtime_kernel_count", _i32, _vp, _i32)
 _sig("arlo_runtime_bucket", _i32, _vp, _i32)
+_sig("arlo_sched_set_policy", C.c_int, _vp, _i32)
 _sig("arlo_allocate", C.c_int, _i32, _i32, _P(_f64), _P(_f64), _P(_f64), _i32, _P(_i32), _P(_f64))
 _sig("arlo_sched_create", C.c_int, _i32, _P(_i32), _P(_i32), _P(_f64), _f64, _f64, _i32, _P(_vp))
 _sig("arlo_sched_destroy", None, _vp)
@@ -223,6 +225,10 @@ class Scheduler:
 
     def set_params(self, lam: float, alpha: float, peek: int):
         check(lib.arlo_sched_set_params(self.handle, lam, alpha, peek))
+
+    def set_policy(self, policy: int):
+        """DISPATCH_RS (Algorithm 1), DISPATCH_ILB or DISPATCH_IG (PAPER.md:L373 baselines)."""
+        check(lib.arlo_sched_set_policy(self.handle, policy))
 
     def dispatch(self, length: int):
         r, i = _i32(), _i32()

@@ -117,6 +117,7 @@ struct arlo_sched {
   std::vector<Level> levels;
   double lambda, alpha;
   int peek;
+  int policy = ARLO_DISPATCH_RS;
 };
 
 extern "C" {
@@ -192,6 +193,30 @@ int arlo_dispatch(arlo_sched* s, int32_t length, int32_t* runtime_out, int32_t* 
   for (int k = 0; k < K && nc < s->peek && nc < 64; ++k)
     if (s->levels[k].max_len >= length && !s->levels[k].heap.empty()) cand[nc++] = k;
   if (nc == 0) return set_error(ARLO_ENOCAND, "arlo_dispatch: no runtime with max_length >= %d", length);
+  if (s->policy == ARLO_DISPATCH_ILB || s->policy == ARLO_DISPATCH_IG) {
+    // baselines of PAPER.md:L373 (Table 4): ILB = ideal runtime (least padding), its
+    // least-loaded instance; IG = least busy instance over ALL candidate runtimes
+    // (reading S20: fewest outstanding requests, ties to the smaller max_length)
+    int q = -1;
+    if (s->policy == ARLO_DISPATCH_ILB) {
+      q = cand[0];
+    } else {
+      int best = 0x7fffffff;
+      for (int k = 0; k < K; ++k) {
+        const Level& l = s->levels[k];
+        if (l.max_len < length || l.heap.empty()) continue;
+        const int n = l.outstanding[l.heap[0]];
+        if (n < best) { best = n; q = k; }
+      }
+    }
+    Level& l = s->levels[q];
+    const int inst = l.heap[0];
+    l.outstanding[inst] += 1;
+    l.sift_down(0);
+    *runtime_out = q;
+    *instance_out = inst;
+    return ARLO_OK;
+  }
   double lam = s->lambda;
   int q = -1;
   for (int c = 0; c < nc; ++c) {  // line 6
@@ -211,6 +236,14 @@ int arlo_dispatch(arlo_sched* s, int32_t length, int32_t* runtime_out, int32_t* 
   l.sift_down(0);                               // line 22 UPDATE
   *runtime_out = q;
   *instance_out = inst;
+  return ARLO_OK;
+}
+
+int arlo_sched_set_policy(arlo_sched* s, int32_t policy) {
+  using namespace arlo;
+  if (!s || policy < ARLO_DISPATCH_RS || policy > ARLO_DISPATCH_IG)
+    return set_error(ARLO_EINVAL, "arlo_sched_set_policy: bad arguments");
+  s->policy = policy;
   return ARLO_OK;
 }
 

@@ -315,3 +315,60 @@ def cluster_replay(arlo, torch, runtimes: dict, cfg, Gs=(1, 2, 4, 8), n_requests
             "st512": {"saturation_req_s": st_sat["served_rate"], "load_sweep": sweep["st512"]},
             "speedup_saturation": arlo_sat["served_rate"] / st_sat["served_rate"]}
     return res
+
+
+def dispatch_ablation(arlo, torch, runtimes: dict, cfg, G: int = 8, n_requests: int = 6000, slo_ms: float = 150.0,
+                      max_batch: int = 32, stream=None, loads=(0.7, 0.9), bursty: bool = True):
+    """Table 4 of the paper: the Request Scheduler (RS, Algorithm 1) against the
+    ILB and IG dispatchers on the same ILP deployment of G GPUs, Twitter-Bursty-like (MMPP)
+    arrivals at `loads` x the RS saturation rate.  Mean / p98 / p99 latency per policy."""
+    Ls = sorted(runtimes)
+    dev = torch.device("cuda")
+    lat = profile_runtimes(torch, runtimes, cfg, max_batch, stream)
+    lengths = wl.sample_lengths(n_requests, seed=wl.SEED_ARRIVALS + 11)
+    ids_all = wl.sample_token_ids(cfg, lengths, max(Ls), seed=wl.SEED_ARRIVALS + 12)
+    ideal = wl.ideal_runtime(lengths, Ls)
+    shares = [float((ideal == k).mean()) for k in range(len(Ls))]
+    caps = [slo_capacity(row, slo_ms) for row in lat]
+    bufs = {L: (torch.empty((max_batch, L), dtype=torch.int32, device=dev),
+                torch.empty((max_batch,), dtype=torch.int32, device=dev)) for L in Ls}
+    out = torch.empty((max_batch, cfg.num_labels), device=dev)
+
+    def service(L, batch):
+        n = len(batch)
+        ids_d, len_d = bufs[L]
+        ids_d[:n].copy_(torch.from_numpy(np.ascontiguousarray(ids_all[batch, :L])))
+        len_d[:n].copy_(torch.from_numpy(lengths[batch].astype(np.int32)))
+        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        a.record(stream)
+        runtimes[L].enqueue(n, ids_d, len_d, out)
+        e.record(stream)
+        e.synchronize()
+        return a.elapsed_time(e) / 1e3
+
+    codes = {"rs": arlo.DISPATCH_RS, "ilb": arlo.DISPATCH_ILB, "ig": arlo.DISPATCH_IG}
+
+    def run(n_inst, arrivals, policy):
+        def factory(max_len, n, capacity, lam, alpha, peek):
+            s = arlo.Scheduler(max_len, n, capacity, lam, alpha, peek)
+            s.set_policy(codes[policy])
+            return s
+        done, rof, _inst, _busy = simulate_cluster(arrivals, lengths, Ls, n_inst, caps, service, max_batch, factory)
+        return summarize(arrivals, lengths, done, rof, Ls, slo_ms)
+
+    zero = np.zeros(n_requests)
+    N, _Q, _M = plan_cluster(arlo, G, Ls, lat, shares, 1e5, slo_ms)
+    sat = run(N, zero, "rs")["served_rate"]
+    N, _Q, _M = plan_cluster(arlo, G, Ls, lat, shares, 0.7 * sat, slo_ms)
+    sat = run(N, zero, "rs")["served_rate"]
+    arrivals_fn = wl.mmpp_arrivals if bursty else wl.poisson_arrivals
+    res = {"G": G, "instances": {str(L): int(N[k]) for k, L in enumerate(Ls)}, "rs_saturation_req_s": sat,
+           "arrivals": "MMPP (Twitter-Bursty-like)" if bursty else "Poisson", "points": []}
+    for f in loads:
+        arr = arrivals_fn(n_requests, f * sat, seed=wl.SEED_ARRIVALS)
+        row = {"load": f, "offered_req_s": f * sat}
+        for pol in ("rs", "ilb", "ig"):
+            r = run(N, arr, pol)
+            row[pol] = {k: r[k] for k in ("mean_ms", "p98_ms", "p99_ms", "slo_violations")}
+        res["points"].append(row)
+    return res

@@ -134,3 +134,49 @@ def test_allocate_paper_scale_8_runtimes_8_gpus(arlo_lib):
     assert N == ref[0] and abs(val - ref[1]) < 1e-9 * abs(ref[1])
     assert sum(N) == G and N[-1] >= 1
     assert dt < 0.5
+
+
+@pytest.mark.parametrize("policy", ["ilb", "ig", "rs"])
+def test_dispatch_policies_match_oracle(arlo_lib, policy):
+    """RS (Algorithm 1) and the ILB / IG baselines of PAPER.md:L373 through the ABI, against
+    the oracle on a random interleaving of arrivals and completions."""
+    rng = np.random.default_rng(17)
+    max_len = [64, 128, 192, 256, 512]
+    n_inst = [2, 3, 0, 1, 2]
+    cap = [6.0, 5.0, 4.0, 3.0, 2.0]
+    s = arlo_lib.Scheduler(max_len, n_inst, cap, 0.85, 0.9, 6)
+    code = {"rs": arlo_lib.DISPATCH_RS, "ilb": arlo_lib.DISPATCH_ILB, "ig": arlo_lib.DISPATCH_IG}[policy]
+    s.set_policy(code)
+    q = osch.MultiLevelQueue(max_len, n_inst, cap)
+    live = []
+    for step in range(600):
+        if live and rng.random() < 0.45:
+            r, i = live.pop(int(rng.integers(len(live))))
+            s.complete(r, i)
+            osch.complete(q, r, i)
+            continue
+        length = int(rng.integers(1, 513))
+        if policy == "rs":
+            want = osch.dispatch(q, length, 0.85, 0.9, 6)
+        elif policy == "ilb":
+            want = osch.dispatch_ilb(q, length)
+        else:
+            want = osch.dispatch_ig(q, length)
+        got = s.dispatch(length)
+        assert got == want, (step, length, got, want)
+        live.append(got)
+    s.close()
+
+
+def test_ilb_ig_hand_cases(arlo_lib):
+    """ILB keeps to the ideal runtime however loaded; IG takes the emptiest candidate."""
+    s = arlo_lib.Scheduler([128, 256, 512], [1, 1, 1], [2.0, 2.0, 2.0], 0.85, 0.9, 6)
+    s.set_policy(arlo_lib.DISPATCH_ILB)
+    assert [s.dispatch(100) for _ in range(3)] == [(0, 0)] * 3
+    s.set_policy(arlo_lib.DISPATCH_IG)
+    assert s.dispatch(100) == (1, 0)   # level 0 has 3 outstanding, levels 1 and 2 none -> smaller max_len
+    assert s.dispatch(100) == (2, 0)   # level 1 now 1, level 2 0
+    assert s.dispatch(300) == (2, 0)   # only level 2 can run a length-300 request
+    with pytest.raises(arlo_lib.ArloError):
+        s.set_policy(7)
+    s.close()

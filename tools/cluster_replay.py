@@ -1,6 +1,6 @@
 """Cluster replay only (BASELINE configs[3] / [4]): ILP-placed runtimes on G virtual GPUs.
 
-    python tools/cluster_replay.py [base|roberta] [n_requests]
+    python tools/cluster_replay.py [base|roberta|ablation] [n_requests]
 """
 import json
 import os
@@ -15,6 +15,9 @@ from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
 
 def main():
     model = sys.argv[1] if len(sys.argv) > 1 else "base"
+    ablation = model == "ablation"
+    if ablation:
+        model = "base"
     n = int(sys.argv[2]) if len(sys.argv) > 2 else 6000
     cfg = wl.ROBERTA_LARGE if model == "roberta" else wl.BERT_BASE
     slo = 450.0 if model == "roberta" else 150.0  # PAPER.md:L297 (R uses the BERT-large SLO)
@@ -25,6 +28,11 @@ def main():
     for L in wl.RUNTIME_LENGTHS:
         rts[L] = arlo.Runtime(W, L, 32)
         rts[L].set_stream(s)
+    if ablation:
+        res = replay.dispatch_ablation(arlo, torch, rts, cfg, G=8, n_requests=n, slo_ms=slo, max_batch=32, stream=s)
+        res["model"] = cfg.name
+        print(json.dumps(res))
+        return
     Gs = (8,) if model == "roberta" else (1, 2, 4, 8)
     res = replay.cluster_replay(arlo, torch, rts, cfg, Gs=Gs, n_requests=n, slo_ms=slo, max_batch=32, stream=s)
     res["model"] = cfg.name
