@@ -61,6 +61,22 @@ __device__ __forceinline__ float gelu_erf_fast(float z) {
   float th;
   asm("tanh.approx.f32 %0, %1;" : "=f"(th) : "f"(0.7978845608f * fmaf(0.044715f * z, z * z, z)));
   return 0.5f * z * (1.0f + th);
+#elif defined(ARLO_GELU_AS28)
+  // A&S 7.1.28: erf(a) = 1 - (1 + a1 a + ... + a6 a^6)^-16, |error| <= 3e-7; one MUFU (rcp)
+  const float az = fabsf(z);
+  const float a = az * 0.70710678118654752f;
+  float p = fmaf(a, 0.0000430638f, 0.0002765672f);
+  p = fmaf(a, p, 0.0001520143f);
+  p = fmaf(a, p, 0.0092705272f);
+  p = fmaf(a, p, 0.0422820123f);
+  p = fmaf(a, p, 0.0705230784f);
+  p = fmaf(a, p, 1.0f);
+  float r = rcp_approx(p);
+  r *= r;
+  r *= r;
+  r *= r;
+  r *= r;  // (1 + ...)^-16 = erfc(a)
+  return fmaf(-0.5f * az, r, fmaxf(z, 0.0f));
 #else
   const float az = fabsf(z);
   const float t = rcp_approx(fmaf(az, 0.3275911f * 0.70710678118654752f, 1.0f));

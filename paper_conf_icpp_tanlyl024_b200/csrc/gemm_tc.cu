@@ -1150,8 +1150,8 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   if (M <= 0 || K % 64 || K <= 0) return false;
   int bn = 0;
   if (N % 192 == 0 && N / 192 <= 8 && N > 256 && (192 / kEpiGroups) % 32 == 0) bn = 192;
-  if (N % 256 == 0 && N / 256 <= 8) bn = 256;
-  if (N == 128) bn = 128;
+  if (N % 256 == 0 && N / 256 <= 8 && (256 / kEpiGroups) % 32 == 0 && 256 % kEpiGroups == 0) bn = 256;
+  if (N == 128 && (128 / kEpiGroups) % 32 == 0 && 128 % kEpiGroups == 0) bn = 128;
   if (!bn) return false;
   const int nt = N / bn;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->epi = EPI_BIAS_RESID; p->ln = true;
@@ -1176,11 +1176,15 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
   }
   if (p.ln) {
     switch (p.BN) {
-      case 128: return launch_ln<128>(p, s);
-      case 192:
-        if constexpr ((192 / kEpiGroups) % 32 == 0) return launch_ln<192>(p, s);
+      case 128:
+        if constexpr ((128 / kEpiGroups) % 32 == 0 && 128 % kEpiGroups == 0) return launch_ln<128>(p, s);
         return cudaErrorInvalidValue;
-      case 256: return launch_ln<256>(p, s);
+      case 192:
+        if constexpr ((192 / kEpiGroups) % 32 == 0 && 192 % kEpiGroups == 0) return launch_ln<192>(p, s);
+        return cudaErrorInvalidValue;
+      case 256:
+        if constexpr ((256 / kEpiGroups) % 32 == 0 && 256 % kEpiGroups == 0) return launch_ln<256>(p, s);
+        return cudaErrorInvalidValue;
     }
     return cudaErrorInvalidValue;
   }
