@@ -91,6 +91,27 @@ __device__ __forceinline__ float gelu_erf_fast(float z) {
 #endif
 }
 
+// gelu_erf_fast on two values with the sm_100 paired fp32 instructions (FFMA2 / FMUL2):
+// the same A&S 7.1.26 evaluation, half the FMA-pipe issue slots.  Every GEMM
+// epilogue (single CTA, CTA pair, skinny) uses this one function, so a given
+// element is computed bitwise identically whatever tile produced it.  The
+// polynomial is negated (exact) so that the last step is one FFMA2:
+// GELU = max(z, 0) + (-0.5 |z| erfc(a)).
+__device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
+__device__ __forceinline__ float2 gelu2_erf_fast(float2 z) {
+  const float2 az = make_float2(fabsf(z.x), fabsf(z.y));
+  const float2 d = __ffma2_rn(az, f2(0.3275911f * 0.70710678118654752f), f2(1.0f));
+  const float2 t = make_float2(rcp_approx(d.x), rcp_approx(d.y));
+  float2 q = __ffma2_rn(t, f2(-0.5f * 1.061405429f), f2(-0.5f * -1.453152027f));
+  q = __ffma2_rn(t, q, f2(-0.5f * 1.421413741f));
+  q = __ffma2_rn(t, q, f2(-0.5f * -0.284496736f));
+  q = __ffma2_rn(t, q, f2(-0.5f * 0.254829592f));
+  const float2 s = __fmul2_rn(__fmul2_rn(z, z), f2(-0.5f * 1.4426950408889634f));
+  const float2 e = make_float2(ex2_approx(s.x), ex2_approx(s.y));  // exp(-z^2/2) = exp(-a^2)
+  const float2 h = __fmul2_rn(__fmul2_rn(q, t), az);                // -0.5 |z| erfc(a) / exp(-a^2)
+  return __ffma2_rn(h, e, make_float2(fmaxf(z.x, 0.0f), fmaxf(z.y, 0.0f)));
+}
+
 // Pack two floats into a bf16x2 word (RNE), low half = a.
 __device__ __forceinline__ uint32_t pack_bf16x2(float a, float b) {
   __nv_bfloat162 h = __floats2bfloat162_rn(a, b);

@@ -96,6 +96,41 @@ constexpr int CW = 32;  // chunk width: TMEM load / staging tile / TMA box (colu
 #define ARLO_EPI_DIRECT 0  // 1: store rows straight from registers instead of smem staging + TMA (A/B)
 #endif
 
+// Epilogue arithmetic of 4 consecutive columns of one row: acc + bias, then GELU or
+// + residual (two bf16x2 words ua, ub), RNE-packed to two bf16x2 words.  Paired fp32
+// instructions (FADD2 / FFMA2); shared by every GEMM kernel so the result of an element
+// does not depend on the tile shape that produced it.
+template <int EPI>
+__device__ __forceinline__ void epi_pack4(const uint32_t* r, float4 b4, uint32_t ua, uint32_t ub, uint32_t& p0,
+                                          uint32_t& p1) {
+#if defined(ARLO_EPI_SCALAR)  // A/B only: the previous scalar epilogue arithmetic
+  float v0 = __uint_as_float(r[0]) + b4.x, v1 = __uint_as_float(r[1]) + b4.y;
+  float v2 = __uint_as_float(r[2]) + b4.z, v3 = __uint_as_float(r[3]) + b4.w;
+  if (EPI == EPI_BIAS_GELU) {
+    v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
+  }
+  if (EPI == EPI_BIAS_RESID) {
+    const float2 fa = unpack_bf16x2(ua), fb = unpack_bf16x2(ub);
+    v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
+  }
+  p0 = pack_bf16x2(v0, v1);
+  p1 = pack_bf16x2(v2, v3);
+  return;
+#endif
+  float2 x0 = __fadd2_rn(make_float2(__uint_as_float(r[0]), __uint_as_float(r[1])), make_float2(b4.x, b4.y));
+  float2 x1 = __fadd2_rn(make_float2(__uint_as_float(r[2]), __uint_as_float(r[3])), make_float2(b4.z, b4.w));
+  if (EPI == EPI_BIAS_GELU) {
+    x0 = gelu2_erf_fast(x0);
+    x1 = gelu2_erf_fast(x1);
+  }
+  if (EPI == EPI_BIAS_RESID) {
+    x0 = __fadd2_rn(x0, unpack_bf16x2(ua));
+    x1 = __fadd2_rn(x1, unpack_bf16x2(ub));
+  }
+  p0 = pack_bf16x2(x0.x, x0.y);
+  p1 = pack_bf16x2(x1.x, x1.y);
+}
+
 template <int BN, int EPI, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int ldr, const float* __restrict__ bias,
@@ -142,20 +177,13 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
 #pragma unroll
     for (int j = 0; j < CW / 4; ++j) {
       const float4 b4 = __ldg(bias4 + j);
-      float v0 = __uint_as_float(r[cur][4 * j + 0]) + b4.x;
-      float v1 = __uint_as_float(r[cur][4 * j + 1]) + b4.y;
-      float v2 = __uint_as_float(r[cur][4 * j + 2]) + b4.z;
-      float v3 = __uint_as_float(r[cur][4 * j + 3]) + b4.w;
-      if (EPI == EPI_BIAS_GELU) {
-        v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
-      }
+      uint32_t ua = 0, ub = 0;
       if (EPI == EPI_BIAS_RESID) {
         const uint4 u = rv[cur][j >> 1];
-        const float2 fa = unpack_bf16x2((j & 1) ? u.z : u.x), fb = unpack_bf16x2((j & 1) ? u.w : u.y);
-        v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
+        ua = (j & 1) ? u.z : u.x;
+        ub = (j & 1) ? u.w : u.y;
       }
-      pk[2 * j] = pack_bf16x2(v0, v1);
-      pk[2 * j + 1] = pack_bf16x2(v2, v3);
+      epi_pack4<EPI>(&r[cur][4 * j], b4, ua, ub, pk[2 * j], pk[2 * j + 1]);
     }
     if (ARLO_EPI_DIRECT) {
       if (row_ok) {
@@ -493,7 +521,13 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
       epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg, sc,
-                             [te]() { ptx::mbar_arrive_cluster(te); }, outp, N);
+                             [te]() {
+#if defined(ARLO_ARRIVE_RELEASE_CLUSTER)  // A/B only: the previous fenced arrive
+                               ptx::mbar_arrive_cluster(te);
+#else
+                               ptx::mbar_arrive_remote(te);
+#endif
+                             }, outp, N);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -638,20 +672,13 @@ gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
 #pragma unroll
         for (int j = 0; j < 4; ++j) {
           const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + n0 + c0) + j);
-          float v0 = __uint_as_float(r[4 * j + 0]) + b4.x;
-          float v1 = __uint_as_float(r[4 * j + 1]) + b4.y;
-          float v2 = __uint_as_float(r[4 * j + 2]) + b4.z;
-          float v3 = __uint_as_float(r[4 * j + 3]) + b4.w;
-          if (EPI == EPI_BIAS_GELU) {
-            v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
-          }
+          uint32_t ua = 0, ub = 0;
           if (EPI == EPI_BIAS_RESID) {
             const uint4 u = rv[j >> 1];
-            const float2 fa = unpack_bf16x2((j & 1) ? u.z : u.x), fb = unpack_bf16x2((j & 1) ? u.w : u.y);
-            v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
+            ua = (j & 1) ? u.z : u.x;
+            ub = (j & 1) ? u.w : u.y;
           }
-          pk[2 * j] = pack_bf16x2(v0, v1);
-          pk[2 * j + 1] = pack_bf16x2(v2, v3);
+          epi_pack4<EPI>(&r[4 * j], b4, ua, ub, pk[2 * j], pk[2 * j + 1]);
         }
         uint4* o4 = reinterpret_cast<uint4*>(out + (size_t)row * N + n0 + c0);
         o4[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);

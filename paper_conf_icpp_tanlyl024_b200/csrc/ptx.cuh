@@ -281,6 +281,17 @@ __device__ __forceinline__ float ld_shared_cluster_f32(uint32_t cluster_addr) {
   return v;
 }
 
+// Arrive on an mbarrier of another CTA of the cluster with CTA-scope release (the CUTLASS
+// ClusterBarrier::arrive form): no fence.  Enough when the arrive only hands back a resource
+// whose last use is already complete (e.g. an accumulator whose tcgen05.ld's were waited on and
+// fenced with tcgen05.fence::before_thread_sync).  The .release.cluster form below compiles to
+// MEMBAR.ALL.CTA + MEMBAR.ALL.GPU before the arrive, which stalled the GEMM epilogue warps
+// (~16 % of warp samples in the FFN1 ncu capture).
+__device__ __forceinline__ void mbar_arrive_remote(uint32_t cluster_addr) {
+  asm volatile("mbarrier.arrive.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
+}
+
+// Cluster-scope release: orders this thread's prior DSMEM / shared writes before the arrive.
 __device__ __forceinline__ void mbar_arrive_cluster(uint32_t cluster_addr) {
   asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(cluster_addr) : "memory");
 }
