@@ -104,7 +104,10 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   constexpr int kSoftWarps = Cfg::kSoftWarps, kProdWarp = Cfg::kProdWarp, kMmaWarp = Cfg::kMmaWarp;
   constexpr int kAttnThreads = Cfg::kThreads;
   constexpr uint32_t kOCol = Cfg::kOCol, kPCol = Cfg::kPCol, kTmemCols = Cfg::kTmemCols;
-  pdl_begin();
+  // PDL: barrier init and the TMEM allocation below overlap the previous kernel's tail;
+  // nothing the previous kernels write (QKV) or read (O) is touched before pdl_wait().
+  // `lengths` is filled by the runtime's input copy, which precedes every kernel of the graph.
+  pdl_launch_dependents();
   const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
   const int len = __ldg(lengths + b);
@@ -112,6 +115,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   const int row_base = b * L;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (q0 >= len) {  // every q-tile wholly padded (or empty slot): zeros
+    pdl_wait();
     const int rows = min(NQ * AQ, L - q0);
     for (int i = threadIdx.x; i < rows * 8; i += kAttnThreads) {
       const int r = i >> 3, c = i & 7;
@@ -164,6 +168,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem = *tmem_slot;
+  pdl_wait();
   if (threadIdx.x == 0) atrace<TRACE>(0);
 
   if (warp == kProdWarp) {
