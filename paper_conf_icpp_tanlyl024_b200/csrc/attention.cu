@@ -265,18 +265,23 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
                            float (&ls)[2]) {
         constexpr bool MASK = decltype(mask_tag)::value;
         uint32_t pk[8];
+        float2 acc = make_float2(ls[0], ls[1]);
 #pragma unroll
         for (int e = 0; e < 16; e += 2) {
-          float p0 = ex2_approx(fmaf(__uint_as_float(v[e]), c2, -mc));
-          float p1 = ex2_approx(fmaf(__uint_as_float(v[e + 1]), c2, -mc));
+          // paired FFMA2 / FADD2: bitwise the scalar fmaf / += (even keys into ls[0], odd into ls[1])
+          const float2 x = __ffma2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])),
+                                      make_float2(c2, c2), make_float2(-mc, -mc));
+          float p0 = ex2_approx(x.x);
+          float p1 = ex2_approx(x.y);
           if (MASK) {
             if (key0 + e >= len) p0 = 0.f;
             if (key0 + e + 1 >= len) p1 = 0.f;
           }
-          ls[0] += p0;
-          ls[1] += p1;
+          acc = __fadd2_rn(acc, make_float2(p0, p1));
           pk[e >> 1] = pack_bf16x2(p0, p1);
         }
+        ls[0] = acc.x;
+        ls[1] = acc.y;
         ptx::tmem_st_32x32b_x8(t_p, pk);
       };
       // this warp's 32 keys of a chunk against max mc; returns the partial p sum

@@ -136,6 +136,20 @@ __device__ __forceinline__ void pdl_begin() {
   pdl_wait();
 }
 
+// 16-byte load of data a PREDECESSOR kernel produced (activations, residuals), for use
+// after pdl_wait().  A volatile asm load is kept after the volatile griddepcontrol.wait;
+// __ldg / const __restrict__ loads (ld.global.nc) are not: nvcc hoisted such loads above
+// the wait (SASS: LDG.CONSTANT before ACQBULK), which read the pooled features before the
+// pooler had written them.  Weights (never written by a kernel) keep __ldg.
+__device__ __forceinline__ uint4 ld_dep_v4(const void* p) {
+  uint4 v;
+  asm volatile("ld.global.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "l"(p)
+               : "memory");
+  return v;
+}
+
 bool pdl_enabled();  // false when ARLO_NO_PDL is set in the environment (A/B measurements)
 
 template <typename... KArgs, typename... Args>

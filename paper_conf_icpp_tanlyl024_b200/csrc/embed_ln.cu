@@ -21,8 +21,8 @@ constexpr int kRowsPerBlock = 8;  // 8 warps, 256 threads
 template <typename T> struct Vec;
 template <> struct Vec<bf16> {
   static constexpr int N = 8;  // 16 B
-  static __device__ __forceinline__ void load(const bf16* p, float* f) {
-    uint4 u = __ldg(reinterpret_cast<const uint4*>(p));
+  static __device__ __forceinline__ void load(const bf16* p, float* f, bool dep = false) {
+    uint4 u = dep ? ld_dep_v4(p) : __ldg(reinterpret_cast<const uint4*>(p));
     float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
     f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
   }
@@ -35,8 +35,14 @@ template <> struct Vec<bf16> {
 };
 template <> struct Vec<float> {
   static constexpr int N = 4;
-  static __device__ __forceinline__ void load(const float* p, float* f) {
-    float4 v = __ldg(reinterpret_cast<const float4*>(p));
+  static __device__ __forceinline__ void load(const float* p, float* f, bool dep = false) {
+    float4 v;
+    if (dep) {
+      const uint4 u = ld_dep_v4(p);
+      v = make_float4(__uint_as_float(u.x), __uint_as_float(u.y), __uint_as_float(u.z), __uint_as_float(u.w));
+    } else {
+      v = __ldg(reinterpret_cast<const float4*>(p));
+    }
     f[0] = v.x; f[1] = v.y; f[2] = v.z; f[3] = v.w;
   }
   static __device__ __forceinline__ void store(float* p, const float* f) {
@@ -123,7 +129,7 @@ __global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* _
   float v[MAXV][VN];
 #pragma unroll
   for (int i = 0; i < MAXV; ++i)
-    if (lane + 32 * i < nvec) Vec<T>::load(src + (lane + 32 * i) * VN, v[i]);
+    if (lane + 32 * i < nvec) Vec<T>::load(src + (lane + 32 * i) * VN, v[i], true);  // predecessor's output
   ln_finish<T, MAXV>(v, nvec, H, lane, s_aff, s_aff + H, eps, out + (size_t)row * H);
 }
 

@@ -176,7 +176,7 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   uint4 rv[2][RV];
   if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-    for (int j = 0; j < RV; ++j) rv[0][j] = __ldg(res4 + cg * RV + j);
+    for (int j = 0; j < RV; ++j) rv[0][j] = ld_dep_v4(res4 + cg * RV + j);
   }
   ptx::tmem_ld_32x32b_x32(t_row + cg * CW, r[0]);
   ptx::tmem_wait_ld();
@@ -189,7 +189,7 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       ptx::tmem_ld_32x32b_x32(t_row + (c + kEpiGroups) * CW, r[nxt]);
       if (EPI == EPI_BIAS_RESID && row_ok) {
 #pragma unroll
-        for (int j = 0; j < RV; ++j) rv[nxt][j] = __ldg(res4 + (c + kEpiGroups) * RV + j);
+        for (int j = 0; j < RV; ++j) rv[nxt][j] = ld_dep_v4(res4 + (c + kEpiGroups) * RV + j);
       }
     }
     const float4* bias4 = reinterpret_cast<const float4*>(bias + n0 + c * CW);
@@ -685,8 +685,8 @@ gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
         uint4 rv[2];
         if (EPI == EPI_BIAS_RESID) {
           const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0 + c0);
-          rv[0] = __ldg(res4);
-          rv[1] = __ldg(res4 + 1);
+          rv[0] = ld_dep_v4(res4);
+          rv[1] = ld_dep_v4(res4 + 1);
         }
         uint32_t pk[8];
 #pragma unroll
@@ -776,7 +776,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
     uint4 rv[4];
     if (row_ok) {
 #pragma unroll
-      for (int j = 0; j < 4; ++j) rv[j] = __ldg(res4 + c * 4 + j);
+      for (int j = 0; j < 4; ++j) rv[j] = ld_dep_v4(res4 + c * 4 + j);
     } else {
 #pragma unroll
       for (int j = 0; j < 4; ++j) rv[j] = make_uint4(0, 0, 0, 0);

@@ -35,34 +35,85 @@ template <> struct Ld8<float> {
   }
 };
 
+// 16-byte vectors of T: VN = 16 / sizeof(T) elements.
+template <typename T>
+__device__ __forceinline__ void unpack16(const uint4& u, float* f) {
+  if constexpr (sizeof(T) == 2) {
+    float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
+    f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
+  } else {
+    f[0] = __uint_as_float(u.x); f[1] = __uint_as_float(u.y); f[2] = __uint_as_float(u.z); f[3] = __uint_as_float(u.w);
+  }
+}
+
+constexpr int kMaxVecPerLane = 16;  // H * sizeof(T) / (16 B * 32 lanes) for H <= 2048 fp32
+
+// The warp's W_p row is loaded into registers BEFORE the PDL wait (weights never depend
+// on the previous kernel); the CLS rows are then staged with every 16-byte load of a thread
+// issued before any shared-memory store (one L2 round trip, not one per element).
 template <typename T>
 __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const T* __restrict__ x,
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
                                                      float* __restrict__ pooled) {
   extern __shared__ float xs[];  // [kRows][H]
-  pdl_begin();
-  const int b0 = blockIdx.y * kRows;
-  const int nb = min(kRows, B - b0);
-  for (int i = threadIdx.x; i < kRows * H; i += blockDim.x) {
-    const int r = i / H, k = i - r * H;
-    xs[i] = r < nb ? Elem<T>::to_f(x[(size_t)(b0 + r) * L * H + k]) : 0.f;  // position 0 of sequence b0+r
-  }
-  __syncthreads();
+  constexpr int VN = 16 / sizeof(T);
+  pdl_launch_dependents();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int j = blockIdx.x * kFeat + warp;
+  const int nvec = H / VN;  // 16-byte vectors per row
+  uint4 wv[kMaxVecPerLane];
+  if (j < H) {
+    const uint4* wr = reinterpret_cast<const uint4*>(w_p + (size_t)j * H);
+#pragma unroll
+    for (int i = 0; i < kMaxVecPerLane; ++i)
+      if (lane + 32 * i < nvec) wv[i] = __ldg(wr + lane + 32 * i);
+  }
+  pdl_wait();
+  const int b0 = blockIdx.y * kRows;
+  const int nb = min(kRows, B - b0);
+  {
+    constexpr int kPer = kRows * 2048 / (16 / 4) / 256;  // max vectors per thread (fp32, H = 2048)
+    uint4 u[kPer];
+#pragma unroll
+    for (int t = 0; t < kPer; ++t) {
+      const int i = threadIdx.x + 256 * t;
+      const int r = i / nvec, c = i - r * nvec;
+      if (r < nb) u[t] = ld_dep_v4(reinterpret_cast<const uint4*>(x + (size_t)(b0 + r) * L * H) + c);
+    }
+#pragma unroll
+    for (int t = 0; t < kPer; ++t) {
+      const int i = threadIdx.x + 256 * t;
+      const int r = i / nvec, c = i - r * nvec;
+      if (r < kRows) {
+        float f[VN];
+        if (r < nb) {
+          unpack16<T>(u[t], f);
+        } else {
+#pragma unroll
+          for (int e = 0; e < VN; ++e) f[e] = 0.f;
+        }
+#pragma unroll
+        for (int e = 0; e < VN; ++e) xs[r * H + c * VN + e] = f[e];
+      }
+    }
+  }
+  __syncthreads();
   if (j >= H) return;
-  constexpr int VN = Ld8<T>::N;
   float acc[kRows];
 #pragma unroll
   for (int r = 0; r < kRows; ++r) acc[r] = 0.f;
-  const T* wr = w_p + (size_t)j * H;
-  for (int k = lane * VN; k < H; k += 32 * VN) {
-    float wv[VN];
-    Ld8<T>::load(wr + k, wv);
 #pragma unroll
-    for (int r = 0; r < kRows; ++r) {
+  for (int i = 0; i < kMaxVecPerLane; ++i) {
+    const int v = lane + 32 * i;
+    if (v < nvec) {
+      float w[VN];
+      unpack16<T>(wv[i], w);
+      const int k = v * VN;
 #pragma unroll
-      for (int e = 0; e < VN; ++e) acc[r] = fmaf(wv[e], xs[r * H + k + e], acc[r]);
+      for (int r = 0; r < kRows; ++r) {
+#pragma unroll
+        for (int e = 0; e < VN; ++e) acc[r] = fmaf(w[e], xs[r * H + k + e], acc[r]);
+      }
     }
   }
 #pragma unroll
@@ -72,21 +123,48 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
   }
 }
 
+// One warp per (sequence, label): 16-byte loads of the W_c row (before the PDL wait) and of
+// the pooled row, fixed lane-strided order then a warp_sum, so logits do not depend on B.
 template <typename T>
 __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const float* __restrict__ pooled,
                                                         const T* __restrict__ w_c, const float* __restrict__ b_c,
                                                         float* __restrict__ logits) {
-  pdl_begin();
+  constexpr int VN = 16 / sizeof(T);
+  pdl_launch_dependents();
   const int b = blockIdx.x;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const float* p = pooled + (size_t)b * H;
+  const int nvec = H / VN;
   for (int c = warp; c < C; c += 2) {
-    const T* wr = w_c + (size_t)c * H;
+    uint4 wv[kMaxVecPerLane];
+    const uint4* wr = reinterpret_cast<const uint4*>(w_c + (size_t)c * H);
+#pragma unroll
+    for (int i = 0; i < kMaxVecPerLane; ++i)
+      if (lane + 32 * i < nvec) wv[i] = __ldg(wr + lane + 32 * i);
+    if (c == warp) pdl_wait();
+    const float* p = pooled + (size_t)b * H;
     float s = 0.f;
-    for (int k = lane; k < H; k += 32) s = fmaf(Elem<T>::to_f(wr[k]), p[k], s);
+#pragma unroll
+    for (int i = 0; i < kMaxVecPerLane; ++i) {
+      const int v = lane + 32 * i;
+      if (v < nvec) {
+        float w[VN];
+        unpack16<T>(wv[i], w);
+#pragma unroll
+        for (int e = 0; e < VN; e += 4) {
+          const uint4 qu = ld_dep_v4(p + v * VN + e);
+          const float4 q = make_float4(__uint_as_float(qu.x), __uint_as_float(qu.y), __uint_as_float(qu.z),
+                                       __uint_as_float(qu.w));
+          s = fmaf(w[e], q.x, s);
+          s = fmaf(w[e + 1], q.y, s);
+          s = fmaf(w[e + 2], q.z, s);
+          s = fmaf(w[e + 3], q.w, s);
+        }
+      }
+    }
     s = warp_sum(s);
     if (lane == 0) logits[(size_t)b * C + c] = s + b_c[c];
   }
+  if (warp >= C) pdl_wait();
 }
 
 template <typename T>
@@ -112,7 +190,7 @@ cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p,
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p,
                         const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
-  if (H > 2048) return cudaErrorInvalidValue;
+  if (H > 2048 || H % 8) return cudaErrorInvalidValue;
   return dt == DT_BF16 ? launch_t<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s)
                        : launch_t<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
 }

@@ -4,6 +4,7 @@
     python tools/profile_ops.py attn B L heads len  # masked attention, all lengths = len
     python tools/profile_ops.py ln M H              # LayerNorm
     python tools/profile_ops.py embed B L           # embedding + LN (BERT-base tables)
+    python tools/profile_ops.py head B L            # CLS pooler + classifier (BERT-base)
 """
 import os
 import sys
@@ -54,6 +55,16 @@ def main():
         out = torch.empty(B * L, H, device=dev, dtype=torch.bfloat16)
         for _ in range(reps):
             arlo.op_embed(arlo.BF16, ids, lens, word, pos, typ, g, bb, 1e-12, out)
+    elif op == "head":
+        B, L = a
+        H = 768
+        x = torch.randn(B * L, H, device=dev).to(torch.bfloat16)
+        wp = (0.02 * torch.randn(H, H, device=dev)).to(torch.bfloat16)
+        wc = (0.02 * torch.randn(2, H, device=dev)).to(torch.bfloat16)
+        bp, bc = torch.zeros(H, device=dev), torch.zeros(2, device=dev)
+        logits = torch.empty(B, 2, device=dev)
+        for _ in range(reps):
+            arlo.op_head(arlo.BF16, B, L, x, wp, bp, wc, bc, logits)
     torch.cuda.synchronize()
 
 
