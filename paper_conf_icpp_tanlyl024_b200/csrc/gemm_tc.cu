@@ -46,6 +46,19 @@ constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 stagi
 #endif
 constexpr int kStgBufs = ARLO_STG_BUFS;         // staging tiles per epilogue warp (TMA stores in flight)
 constexpr int kStagingBytes = kEpiWarps * kStgBufs * kStgBytes;
+
+// Warp-role layout of the persistent kernels for EW epilogue warps (EW / 4 column groups per
+// TMEM lane quarter), then the TMA producer and the MMA warp.  EW = 8 by default; the
+// GELU epilogue (two MUFU ops per element) runs with EW = 12 where it, not the mainloop,
+// paces the kernel (M <= 8192: FFN1 at M = 4096 918 -> 985 TF, at M = 8192 1093 -> 1168 TF,
+// gpurun_out/ab18; at M = 16384 and K = 1024 the 12-warp variant lost); the
+// bias / residual epilogues lose with 12 (fewer smem stages, more residual traffic in flight).
+template <int EW>
+struct Roles {
+  static_assert(EW % 4 == 0, "epilogue warps cover the four TMEM lane quarters");
+  static constexpr int kEpi = EW, kGroups = EW / 4, kProducer = EW, kMma = EW + 1, kThreads = 32 * (EW + 2);
+  static constexpr int kStaging = EW * kStgBufs * kStgBytes;
+};
 constexpr int kSmemBudget = 229376;            // 224 KB of the 227 KB opt-in maximum
 
 // Optional event trace (tools/gemm_trace.py): when g_trace != nullptr every CTA
@@ -88,8 +101,9 @@ constexpr int tmem_cols_for(int n) {
 // PAIR = false: one CTA computes a 128 x BN tile; PAIR = true: a CTA pair
 // (cluster of 2, cta_group::2) computes a 256 x BN tile, each CTA holding 128
 // rows of A, BN/2 rows of W and its 128 x BN half of the accumulator.
-template <int BN, bool PAIR, int RESERVE = 0>
+template <int BN, bool PAIR, int RESERVE = 0, int EW = kEpiWarps>
 struct TcCfg {
+  static constexpr int kStagingBytes = Roles<EW>::kStaging;
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
   static constexpr int B_BYTES = B_ROWS * BK * 2;
@@ -151,7 +165,7 @@ __device__ __forceinline__ void epi_pack4(const uint32_t* r, float4 b4, uint32_t
   p1 = pack_bf16x2(x1.x, x1.y);
 }
 
-template <int BN, int EPI, typename Release>
+template <int BN, int EPI, int kEpiGroups, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int ldr, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
@@ -248,12 +262,15 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   }
 }
 
-template <int BN, int EPI>
-__global__ void __launch_bounds__(kThreads, 1)
+template <int BN, int EPI, int EW>
+__global__ void __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
                const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
-  using C = TcCfg<BN, false>;
+  using C = TcCfg<BN, false, 0, EW>;
+  using R = Roles<EW>;
+  constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
+  constexpr int kStagingBytes = R::kStaging;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -379,8 +396,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg,
-                             sc, [te]() { ptx::mbar_arrive(te); }, outp, N);
+      epilogue_tile<BN, EPI, kEpiGroups>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid,
+                                         &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -403,12 +420,15 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 // tfull barriers (multicast); both CTAs' epilogue warps arrive on the
 // leader's tempty barrier.  Halves the L2->SM operand traffic per FLOP and
 // deepens the smem pipeline relative to the single-CTA kernel.
-template <int BN, int EPI>
-__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads, 1)
+template <int BN, int EPI, int EW>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
                     const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
-  using C = TcCfg<BN, true>;
+  using C = TcCfg<BN, true, 0, EW>;
+  using R = Roles<EW>;
+  constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
+  constexpr int kStagingBytes = R::kStaging;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -540,7 +560,8 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
-      epilogue_tile<BN, EPI>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid, &tmC, stg, sc,
+      epilogue_tile<BN, EPI, kEpiGroups>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid,
+                                         &tmC, stg, sc,
                              [te]() {
 #if defined(ARLO_ARRIVE_RELEASE_CLUSTER)  // A/B only: the previous fenced arrive
                                ptx::mbar_arrive_cluster(te);
@@ -998,18 +1019,26 @@ EncodeTiledFn get_encode_fn() {
   return fn;
 }
 
-template <int BN, int EPI, bool PAIR>
-cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
-  using C = TcCfg<BN, PAIR>;
-  auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI> : gemm_tc_kernel<BN, EPI>;
+template <int BN, int EPI, bool PAIR, int EW>
+cudaError_t launch_cfg_ew(const TcGemmPlan& p, cudaStream_t s) {
+  using C = TcCfg<BN, PAIR, 0, EW>;
+  auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI, EW> : gemm_tc_kernel<BN, EPI, EW>;
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  return launch_k(kern, dim3(p.grid), dim3(kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K, p.bias,
-                  (const bf16*)p.resid, p.ldr, (bf16*)p.out);
+  return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K,
+                  p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out);
+}
+
+template <int BN, int EPI, bool PAIR>
+cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
+  if constexpr (EPI == EPI_BIAS_GELU) {
+    if (p.ew == 12) return launch_cfg_ew<BN, EPI, PAIR, 12>(p, s);
+  }
+  return launch_cfg_ew<BN, EPI, PAIR, kEpiWarps>(p, s);
 }
 
 template <int BN, bool PAIR>
@@ -1097,7 +1126,8 @@ int tc_choose_bn(int M, int N, int K) {
   double best = 1e30;
   int best_bn = 0;
   struct Cand { int code; double eff; };
-  const Cand cands[7] = {{-256, 0.75}, {-192, 0.65}, {256, 0.45}, {192, 0.70}, {-128, 0.50}, {128, 0.60}, {64, 0.45}};
+  const Cand cands[8] = {{-256, 0.75}, {-192, 0.65}, {256, 0.45}, {192, 0.70}, {-128, 0.50}, {128, 0.60}, {96, 0.55},
+                         {64, 0.45}};
   for (const Cand& c : cands) {
     const bool pair = c.code < 0;
     const int bn = pair ? -c.code : c.code;
@@ -1135,7 +1165,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   if (choice > kSkinnyCode) {
     const int bn = choice - kSkinnyCode;
     if ((bn != 16 && bn != 32 && bn != 64) || N % bn) return false;
-    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->epi = epi; p->ln = false;
+    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->epi = epi; p->ln = false; p->ew = 4;
     p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
     p->a_rows = M < BM ? ((M + 7) & ~7) : BM;
     p->grid = (N / bn) * ((M + BM - 1) / BM);
@@ -1145,7 +1175,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   }
   const bool pair = choice < 0;
   const int bn = pair ? -choice : choice;
-  if (bn != 64 && bn != 128 && bn != 192 && bn != 256) return false;
+  if (bn != 64 && bn != 96 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn < 128) return false;
   if (N % bn) return false;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->epi = epi; p->ln = false;
@@ -1154,6 +1184,10 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
   const int slots = pair ? num_sms() / 2 : num_sms();
   p->grid = (tiles < slots ? tiles : slots) * (pair ? 2 : 1);
+#ifndef ARLO_GELU_EW12_MAX_M
+#define ARLO_GELU_EW12_MAX_M 8192  // A/B hook: 0 keeps 8 epilogue warps everywhere
+#endif
+  p->ew = (epi == EPI_BIAS_GELU && M <= ARLO_GELU_EW12_MAX_M) ? 12 : kEpiWarps;
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128, (uint64_t)lda)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
@@ -1202,6 +1236,7 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   if (!bn) return false;
   const int nt = N / bn;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->ew = kEpiWarps;
   p->bias = bias; p->resid = resid; p->ldr = N; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
   const int num_m = (M + BM - 1) / BM;
   const int clusters = num_sms() / nt;
@@ -1245,6 +1280,7 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
   }
   switch (p.BN) {
     case 64: return launch_bn<64, false>(p, s);
+    case 96: return launch_bn<96, false>(p, s);
     case 128: return launch_bn<128, false>(p, s);
     case 192: return launch_bn<192, false>(p, s);
     case 256: return launch_bn<256, false>(p, s);

@@ -18,23 +18,6 @@ namespace {
 constexpr int kRows = 8;   // sequences per CTA
 constexpr int kFeat = 8;   // output features per CTA (one per warp)
 
-template <typename T> struct Ld8;
-template <> struct Ld8<bf16> {
-  static constexpr int N = 8;
-  static __device__ __forceinline__ void load(const bf16* p, float* f) {
-    const uint4 u = __ldg(reinterpret_cast<const uint4*>(p));
-    float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
-    f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
-  }
-};
-template <> struct Ld8<float> {
-  static constexpr int N = 4;
-  static __device__ __forceinline__ void load(const float* p, float* f) {
-    const float4 u = __ldg(reinterpret_cast<const float4*>(p));
-    f[0] = u.x; f[1] = u.y; f[2] = u.z; f[3] = u.w;
-  }
-};
-
 // 16-byte vectors of T: VN = 16 / sizeof(T) elements.
 template <typename T>
 __device__ __forceinline__ void unpack16(const uint4& u, float* f) {
@@ -46,12 +29,15 @@ __device__ __forceinline__ void unpack16(const uint4& u, float* f) {
   }
 }
 
-constexpr int kMaxVecPerLane = 16;  // H * sizeof(T) / (16 B * 32 lanes) for H <= 2048 fp32
+// MAXV = 16-byte vectors per lane of one H-row, ceil(H * sizeof(T) / 512): a warp's W row and
+// (kRows * 32 == 256 threads) a thread's share of the kRows staged CLS rows both take MAXV
+// registers of 16 B, so the register count follows H (173 registers at a fixed 16 limited the
+// pooler to one CTA per SM: 31 us at B = 32).
 
 // The warp's W_p row is loaded into registers BEFORE the PDL wait (weights never depend
 // on the previous kernel); the CLS rows are then staged with every 16-byte load of a thread
 // issued before any shared-memory store (one L2 round trip, not one per element).
-template <typename T>
+template <typename T, int MAXV>
 __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const T* __restrict__ x,
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
                                                      float* __restrict__ pooled) {
@@ -61,18 +47,19 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int j = blockIdx.x * kFeat + warp;
   const int nvec = H / VN;  // 16-byte vectors per row
-  uint4 wv[kMaxVecPerLane];
+  uint4 wv[MAXV];
   if (j < H) {
     const uint4* wr = reinterpret_cast<const uint4*>(w_p + (size_t)j * H);
 #pragma unroll
-    for (int i = 0; i < kMaxVecPerLane; ++i)
+    for (int i = 0; i < MAXV; ++i)
       if (lane + 32 * i < nvec) wv[i] = __ldg(wr + lane + 32 * i);
   }
   pdl_wait();
   const int b0 = blockIdx.y * kRows;
   const int nb = min(kRows, B - b0);
   {
-    constexpr int kPer = kRows * 2048 / (16 / 4) / 256;  // max vectors per thread (fp32, H = 2048)
+    constexpr int kPer = MAXV;  // kRows * nvec / 256 <= MAXV vectors per thread
+    static_assert(kRows * 32 == 256, "one staged vector per thread per 32 of a row");
     uint4 u[kPer];
 #pragma unroll
     for (int t = 0; t < kPer; ++t) {
@@ -103,7 +90,7 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
 #pragma unroll
   for (int r = 0; r < kRows; ++r) acc[r] = 0.f;
 #pragma unroll
-  for (int i = 0; i < kMaxVecPerLane; ++i) {
+  for (int i = 0; i < MAXV; ++i) {
     const int v = lane + 32 * i;
     if (v < nvec) {
       float w[VN];
@@ -125,7 +112,7 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
 
 // One warp per (sequence, label): 16-byte loads of the W_c row (before the PDL wait) and of
 // the pooled row, fixed lane-strided order then a warp_sum, so logits do not depend on B.
-template <typename T>
+template <typename T, int MAXV>
 __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const float* __restrict__ pooled,
                                                         const T* __restrict__ w_c, const float* __restrict__ b_c,
                                                         float* __restrict__ logits) {
@@ -135,16 +122,16 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int nvec = H / VN;
   for (int c = warp; c < C; c += 2) {
-    uint4 wv[kMaxVecPerLane];
+    uint4 wv[MAXV];
     const uint4* wr = reinterpret_cast<const uint4*>(w_c + (size_t)c * H);
 #pragma unroll
-    for (int i = 0; i < kMaxVecPerLane; ++i)
+    for (int i = 0; i < MAXV; ++i)
       if (lane + 32 * i < nvec) wv[i] = __ldg(wr + lane + 32 * i);
     if (c == warp) pdl_wait();
     const float* p = pooled + (size_t)b * H;
     float s = 0.f;
 #pragma unroll
-    for (int i = 0; i < kMaxVecPerLane; ++i) {
+    for (int i = 0; i < MAXV; ++i) {
       const int v = lane + 32 * i;
       if (v < nvec) {
         float w[VN];
@@ -167,22 +154,41 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
   if (warp >= C) pdl_wait();
 }
 
-template <typename T>
+template <typename T, int MAXV>
 cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
                      const float* b_c, float* pooled, float* logits, cudaStream_t s) {
   const size_t smem = (size_t)kRows * H * sizeof(float);
   static bool attr = false;
   if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(pooler_kernel<T>, cudaFuncAttributeMaxDynamicSharedMemorySize, 8 * 2048 * 4);
+    cudaError_t e = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                         kRows * 2048 * 4);
+    if (e != cudaSuccess) return e;
+    e = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                             cudaSharedmemCarveoutMaxShared);
     if (e != cudaSuccess) return e;
     attr = true;
   }
   dim3 grid((H + kFeat - 1) / kFeat, (B + kRows - 1) / kRows);
-  cudaError_t e = launch_k(pooler_kernel<T>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p, b_p,
-                           pooled);
+  cudaError_t e = launch_k(pooler_kernel<T, MAXV>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p,
+                           b_p, pooled);
   if (e != cudaSuccess) return e;
-  return launch_k(classifier_kernel<T>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c, b_c,
-                  logits);
+  return launch_k(classifier_kernel<T, MAXV>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c,
+                  b_c, logits);
+}
+
+template <typename T>
+cudaError_t launch_dt(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
+                      const float* b_c, float* pooled, float* logits, cudaStream_t s) {
+  const int maxv = (H * (int)sizeof(T) + 511) / 512;
+  switch (maxv) {
+    case 1: return launch_t<T, 1>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 2: return launch_t<T, 2>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 3: return launch_t<T, 3>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 4: return launch_t<T, 4>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 5: case 6: return launch_t<T, 6>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 7: case 8: return launch_t<T, 8>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    default: return launch_t<T, 16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+  }
 }
 
 }  // namespace
@@ -191,8 +197,8 @@ cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, con
                         const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s) {
   if (B <= 0) return cudaSuccess;
   if (H > 2048 || H % 8) return cudaErrorInvalidValue;
-  return dt == DT_BF16 ? launch_t<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s)
-                       : launch_t<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+  return dt == DT_BF16 ? launch_dt<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s)
+                       : launch_dt<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
 }
 
 }  // namespace arlo

@@ -33,6 +33,7 @@ struct TcGemmPlan {
   CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN (BN/2 for a pair)}, 128B swizzle
   CUtensorMap tmC;  // output      [M, N] bf16, box {32, 32}, 64B swizzle (epilogue TMA stores)
   int M, N, K, BN, epi, grid;
+  int ew;       // epilogue warps of the persistent kernels (8, or 12 for GELU at M <= 8192)
   bool pair;    // CTA-pair (cta_group::2) kernel, 256-row tiles
   bool skinny;  // small-M kernel: one CTA per 128 x BN tile (BN 16/32/64), direct stores
   int a_rows;   // skinny: A box rows (min(128, M rounded up to 8))

@@ -35,7 +35,7 @@ GEMM_SHAPES = [
 
 @pytest.mark.parametrize("M,N,K", GEMM_SHAPES)
 @pytest.mark.parametrize("epi", [0, 1, 2])
-@pytest.mark.parametrize("force", [0, 128, -128, -256, 192, -192, 1016, 1032, 1064])
+@pytest.mark.parametrize("force", [0, 96, 128, -128, -256, 192, -192, 1016, 1032, 1064])
 def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
     """force: BN single CTA, -BN CTA pair, 1000 + BN skinny (small-M) kernel, 0 = tile chooser."""
     if N % (force - 1000 if force > 1000 else abs(force or 64)):
@@ -58,21 +58,25 @@ def test_gemm_tcgen05_bf16(arlo_lib, M, N, K, epi, force):
     np.testing.assert_allclose(got, ref, rtol=8e-3, atol=8e-3)
 
 
-@pytest.mark.parametrize("bn", [64, 128, 192, 256, -128, -192, -256, 1016, 1032, 1064])
-def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn):
-    """Row results do not depend on the tile width (cross-L invariance contract)."""
+@pytest.mark.parametrize("epi", [0, 1, 2])
+@pytest.mark.parametrize("bn", [64, 96, 128, 192, 256, -128, -192, -256, 1016, 1032, 1064])
+def test_gemm_tile_widths_agree_bitwise(arlo_lib, bn, epi):
+    """Row results do not depend on the tile width, the epilogue warp count (12 for GELU at
+    M <= 8192, 8 otherwise) or M (cross-L invariance contract), for every epilogue."""
     M, N, K = 300, 768, 768
     A, W, b = bf16_dev(rnd((M, K), 5)), bf16_dev(rnd((N, K), 6, 0.02)), f32_dev(rnd((N,), 7, 0.02))
+    R = bf16_dev(rnd((M, N), 8))
     outs = []
     for force in (bn, -256):
         o = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
-        arlo_lib.op_gemm(arlo_lib.BF16, A, W, b, o, epi=0, force_bn=force)
+        arlo_lib.op_gemm(arlo_lib.BF16, A, W, b, o, epi=epi, residual=R if epi == 2 else None, force_bn=force)
         outs.append(o)
     torch.cuda.synchronize()
     assert torch.equal(outs[0], outs[1])
     # and a row does not depend on M (prefix of rows)
     o2 = torch.empty((77, N), device="cuda", dtype=torch.bfloat16)
-    arlo_lib.op_gemm(arlo_lib.BF16, A[:77].contiguous(), W, b, o2, epi=0, force_bn=64)
+    arlo_lib.op_gemm(arlo_lib.BF16, A[:77].contiguous(), W, b, o2, epi=epi,
+                     residual=R[:77].contiguous() if epi == 2 else None, force_bn=64)
     torch.cuda.synchronize()
     assert torch.equal(o2, outs[0][:77])
 

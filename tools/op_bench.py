@@ -14,6 +14,15 @@ from tools.gemm_sweep import time_op  # noqa: E402
 
 def main():
     dev = torch.device("cuda")
+    H = 768
+    wp = (0.02 * torch.randn(H, H, device=dev)).to(torch.bfloat16)
+    wc = (0.02 * torch.randn(2, H, device=dev)).to(torch.bfloat16)
+    bp, bc = torch.zeros(H, device=dev), torch.zeros(2, device=dev)
+    for B in (1, 8, 32):
+        x = torch.randn(B * 128, H, device=dev).to(torch.bfloat16)
+        logits = torch.empty(B, 2, device=dev)
+        t = time_op(lambda st: arlo.op_head(arlo.BF16, B, 128, x, wp, bp, wc, bc, logits, stream=st))
+        print(f"head (pooler + classifier) B={B:3d} H={H}: {t * 1e6:7.2f} us", flush=True)
     for (M, H) in ((64, 768), (4096, 768), (16384, 768), (32768, 1024)):
         x = torch.randn(M, H, device=dev).to(torch.bfloat16)
         g, bb = torch.ones(H, device=dev), torch.zeros(H, device=dev)
