@@ -41,7 +41,10 @@ template <typename T, int MAXV>
 __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const T* __restrict__ x,
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
                                                      float* __restrict__ pooled) {
-  extern __shared__ float xs[];  // [kRows][H]
+  // [kRows][nvec] raw 16-byte vectors of T: lane-consecutive vectors are bank-conflict free
+  // (fp32 staging with 8 floats per lane put lanes 4 apart on the same banks: 8-way STS,
+  // 2x LDS.128 wavefronts; the pooler was shared-memory bound at 22 us for b = 32)
+  extern __shared__ uint4 xs[];
   constexpr int VN = 16 / sizeof(T);
   pdl_launch_dependents();
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -71,17 +74,7 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
     for (int t = 0; t < kPer; ++t) {
       const int i = threadIdx.x + 256 * t;
       const int r = i / nvec, c = i - r * nvec;
-      if (r < kRows) {
-        float f[VN];
-        if (r < nb) {
-          unpack16<T>(u[t], f);
-        } else {
-#pragma unroll
-          for (int e = 0; e < VN; ++e) f[e] = 0.f;
-        }
-#pragma unroll
-        for (int e = 0; e < VN; ++e) xs[r * H + c * VN + e] = f[e];
-      }
+      if (r < kRows) xs[r * nvec + c] = r < nb ? u[t] : make_uint4(0, 0, 0, 0);
     }
   }
   __syncthreads();
@@ -95,11 +88,12 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
     if (v < nvec) {
       float w[VN];
       unpack16<T>(wv[i], w);
-      const int k = v * VN;
 #pragma unroll
       for (int r = 0; r < kRows; ++r) {
+        float xv[VN];
+        unpack16<T>(xs[r * nvec + v], xv);
 #pragma unroll
-        for (int e = 0; e < VN; ++e) acc[r] = fmaf(w[e], xs[r * H + k + e], acc[r]);
+        for (int e = 0; e < VN; ++e) acc[r] = fmaf(w[e], xv[e], acc[r]);
       }
     }
   }
@@ -157,7 +151,7 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
 template <typename T, int MAXV>
 cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
                      const float* b_c, float* pooled, float* logits, cudaStream_t s) {
-  const size_t smem = (size_t)kRows * H * sizeof(float);
+  const size_t smem = (size_t)kRows * H * sizeof(T);
   static bool attr = false;
   if (!attr) {
     cudaError_t e = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributeMaxDynamicSharedMemorySize,

@@ -21,3 +21,4 @@ full attn_l128 attn_tc python tools/profile_ops.py attn 32 128 12 128
 full attn_l512 attn_tc python tools/profile_ops.py attn 64 512 16 512
 full layernorm layernorm python tools/profile_ops.py ln 4096 768
 full embed embed_ln python tools/profile_ops.py embed 32 128
+full pooler pooler python tools/profile_ops.py head 32 128
