@@ -51,10 +51,16 @@ struct AttnCfg {
   // at kOCol + qi*64; P slot sl (64 bf16 packed in 32 columns) at kPCol + (qi*NS + sl)*32
   static constexpr uint32_t kOCol = NQ * NS * KC;
   static constexpr uint32_t kPCol = kOCol + NQ * D;
-  static constexpr uint32_t kUsedCols = NQ * (NS * KC + D + NS * KC / 2);
+  // ALIAS (NS == 1): a warp writes its 32 keys of P (16 packed columns) over the first 16
+  // columns of its own 32 S columns, after its S values are in registers.  TMEM per q-tile
+  // is then 64 (S/P) + 64 (O) columns: 128 per CTA, so three CTAs share an SM (the b = 32,
+  // L <= 128 grids of 384 CTAs run in one wave instead of 1.3).  The next S MMA into the
+  // slot waits for the PV MMA that read P from it.
+  static constexpr bool ALIAS = NS == 1;
+  static constexpr uint32_t kUsedCols = ALIAS ? NQ * (NS * KC + D) : NQ * (NS * KC + D + NS * KC / 2);
   static constexpr uint32_t kTmemCols = kUsedCols <= 128 ? 128 : kUsedCols <= 256 ? 256 : 512;
   static_assert(kUsedCols <= 512, "attention TMEM");
-  static constexpr int kMinBlocks = 512 / kTmemCols < 2 ? 1 : 2;
+  static constexpr int kMinBlocks = ALIAS ? 3 : 512 / kTmemCols < 2 ? 1 : 2;
   static_assert(kSmem * kMinBlocks <= 232448, "attention smem");
 };
 
@@ -209,11 +215,14 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::mbar_wait(&p_full[qi * NS + sl], (c / NS) & 1);
           ptx::mbar_wait(&bar_v[t], 0);
           ptx::tc_fence_after();
-          const uint32_t p_tmem = tmem + kPCol + (qi * NS + sl) * (KC / 2);
+          // P of keys [16 ks, 16 ks + 16): half ks / 2, 8 packed columns per K = 16 step
+          const uint32_t p_tmem = Cfg::ALIAS ? tmem + (qi * NS + sl) * KC : tmem + kPCol + (qi * NS + sl) * (KC / 2);
           const uint32_t v_addr = ptx::smem_u32(sV + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
 #pragma unroll
           for (int ks = 0; ks < KC / 16; ++ks)  // 16 keys = 8 packed P columns per step
-            ptx::mma_bf16_ts_w(tmem + kOCol + qi * D, p_tmem + ks * 8, ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
+            ptx::mma_bf16_ts_w(tmem + kOCol + qi * D,
+                               p_tmem + (Cfg::ALIAS ? (ks >> 1) * (KC / 2) + (ks & 1) * 8 : ks * 8),
+                               ptx::desc_mn_sw128(v_addr + ks * 2048, 0),
                                idesc_pv, (c | ks) != 0);
           ptx::mma_commit_w(&pv_done[qi * NS + sl]);
           if ((c & 1) || c == n_ch - 1) ptx::mma_commit_w(&v_free[t & 1]);  // V tile t done for this q-tile
@@ -226,6 +235,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         for (int c = 0; c < n_ch; ++c) {
           const int t = c >> 1, sl = c % NS;
           if (c >= NS) ptx::mbar_wait(&s_free[qi * NS + sl], ((c - NS) / NS) & 1);
+          if (Cfg::ALIAS && c >= NS) ptx::mbar_wait(&pv_done[qi * NS + sl], ((c - NS) / NS) & 1);
           ptx::mbar_wait(&bar_k[t], 0);
           ptx::tc_fence_after();
           const uint32_t k_addr = ptx::smem_u32(sK + (t & 1) * kTileBytes + (c & 1) * (KC * 128));
@@ -331,43 +341,125 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::tc_fence_after();
         }
         float ls;
-        if (c == 0) {
-          // first chunk: row max from a first pass over S, shared by the pair
-          xs[par * AQ + r] = half_max(full, t_chunk, key0);
-          pair_sync();
-          m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
-          ls = exp_any(full, t_chunk, m * c2, key0, t_p);
-        } else {
-          // single streaming pass against the (possibly stale) running max.  A row
-          // whose p sum passes 2^8 in either half (necessary if any p > 2^8;
-          // impossible while every p <= 4) is redone by both halves against the
-          // new row max, O and l rescaled.
-          ls = exp_any(full, t_chunk, m * c2, key0, t_p);
-          xs[par * AQ + r] = ls;
-          pair_sync();
-          const bool need = ls > 256.0f || xp[par * AQ + r] > 256.0f;  // same in both warps
-          if (__any_sync(0xffffffffu, need)) {
-            xmax[qi][hf][r] = half_max(full, t_chunk, key0);
-            pair_sync();
-            const float cmax = fmaxf(m, fmaxf(xmax[qi][0][r], xmax[qi][1][r]));
-            float alpha = 1.f;
-            if (need) {
-              alpha = ex2_approx((m - cmax) * c2);
-              l *= alpha;
-              m = cmax;
-            }
-            // O holds PV_0..c-1 (warp-collective TMEM traffic: every row takes part)
-            ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);
-            ptx::tc_fence_after();
-            uint32_t ov[32];
-            ptx::tmem_ld_32x32b_x32(t_o, ov);
+        if constexpr (Cfg::ALIAS) {
+          // one TMEM read of the warp's 32 S values; max, exp and (rare) redo from registers;
+          // P stored last, over the first 16 of these S columns
+          // (S stays intact in TMEM until P is stored at the end, so the rare redo re-reads it:
+          // va / vb are not live across the pair barrier, which keeps the kernel under the
+          // 56-register budget of three 352-thread CTAs per SM)
+          uint32_t va[16], vb[16], pk[16];
+          auto load_s = [&]() {
+            ptx::tmem_ld_32x32b_x16(t_chunk, va);
+            ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);
             ptx::tmem_wait_ld();
+          };
+          auto reg_max = [&]() {
+            float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
-            for (int e = 0; e < 32; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
-            ptx::tmem_st_32x32b_x16(t_o, *reinterpret_cast<uint32_t(*)[16]>(&ov[0]));
-            ptx::tmem_st_32x32b_x16(t_o + 16, *reinterpret_cast<uint32_t(*)[16]>(&ov[16]));
-            ptx::tmem_wait_st();
+            for (int e = 0; e < 16; ++e) {
+              if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+              if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
+            }
+            return fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+          };
+          auto reg_exp = [&](float mc) {
+            float2 acc = make_float2(0.f, 0.f);
+#pragma unroll
+            for (int e = 0; e < 32; e += 2) {
+              const uint32_t* v = e < 16 ? va : vb;
+              const int ee = e & 15;
+              const float2 x = __ffma2_rn(make_float2(__uint_as_float(v[ee]), __uint_as_float(v[ee + 1])),
+                                          make_float2(c2, c2), make_float2(-mc, -mc));
+              float p0 = ex2_approx(x.x);
+              float p1 = ex2_approx(x.y);
+              if (!full) {
+                if (key0 + e >= len) p0 = 0.f;
+                if (key0 + e + 1 >= len) p1 = 0.f;
+              }
+              acc = __fadd2_rn(acc, make_float2(p0, p1));
+              pk[e >> 1] = pack_bf16x2(p0, p1);
+            }
+            return acc.x + acc.y;
+          };
+          load_s();
+          if (c == 0) {
+            xs[par * AQ + r] = reg_max();
+            pair_sync();
+            m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
+            ls = reg_exp(m * c2);
+          } else {
+            ls = reg_exp(m * c2);
+            xs[par * AQ + r] = ls;
+            pair_sync();
+            const bool need = ls > 256.0f || xp[par * AQ + r] > 256.0f;  // same in both warps
+            if (__any_sync(0xffffffffu, need)) {
+              load_s();
+              xmax[qi][hf][r] = reg_max();
+              pair_sync();
+              const float cmax = fmaxf(m, fmaxf(xmax[qi][0][r], xmax[qi][1][r]));
+              float alpha = 1.f;
+              if (need) {
+                alpha = ex2_approx((m - cmax) * c2);
+                l *= alpha;
+                m = cmax;
+              }
+              // O holds PV_0..c-1 (complete: S(c) was issued after PV(c-1) finished); rescaled
+              // 16 columns at a time, then S re-read (register budget)
+#pragma unroll
+              for (int h2 = 0; h2 < 2; ++h2) {
+                uint32_t ov[16];
+                ptx::tmem_ld_32x32b_x16(t_o + 16 * h2, ov);
+                ptx::tmem_wait_ld();
+#pragma unroll
+                for (int e = 0; e < 16; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
+                ptx::tmem_st_32x32b_x16(t_o + 16 * h2, ov);
+              }
+              ptx::tmem_wait_st();
+              load_s();
+              ls = reg_exp(m * c2);
+            }
+          }
+          ptx::tmem_st_32x32b_x8(t_chunk, *reinterpret_cast<uint32_t(*)[8]>(&pk[0]));
+          ptx::tmem_st_32x32b_x8(t_chunk + 8, *reinterpret_cast<uint32_t(*)[8]>(&pk[8]));
+        } else {
+          if (c == 0) {
+            // first chunk: row max from a first pass over S, shared by the pair
+            xs[par * AQ + r] = half_max(full, t_chunk, key0);
+            pair_sync();
+            m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
             ls = exp_any(full, t_chunk, m * c2, key0, t_p);
+          } else {
+            // single streaming pass against the (possibly stale) running max.  A row
+            // whose p sum passes 2^8 in either half (necessary if any p > 2^8;
+            // impossible while every p <= 4) is redone by both halves against the
+            // new row max, O and l rescaled.
+            ls = exp_any(full, t_chunk, m * c2, key0, t_p);
+            xs[par * AQ + r] = ls;
+            pair_sync();
+            const bool need = ls > 256.0f || xp[par * AQ + r] > 256.0f;  // same in both warps
+            if (__any_sync(0xffffffffu, need)) {
+              xmax[qi][hf][r] = half_max(full, t_chunk, key0);
+              pair_sync();
+              const float cmax = fmaxf(m, fmaxf(xmax[qi][0][r], xmax[qi][1][r]));
+              float alpha = 1.f;
+              if (need) {
+                alpha = ex2_approx((m - cmax) * c2);
+                l *= alpha;
+                m = cmax;
+              }
+              // O holds PV_0..c-1 (warp-collective TMEM traffic: every row takes part)
+              ptx::mbar_wait(&pv_done[qi * NS + ((c - 1) % NS)], ((c - 1) / NS) & 1);
+              ptx::tc_fence_after();
+              uint32_t ov[32];
+              ptx::tmem_ld_32x32b_x32(t_o, ov);
+              ptx::tmem_wait_ld();
+#pragma unroll
+              for (int e = 0; e < 32; ++e) ov[e] = __float_as_uint(__uint_as_float(ov[e]) * alpha);
+              ptx::tmem_st_32x32b_x16(t_o, *reinterpret_cast<uint32_t(*)[16]>(&ov[0]));
+              ptx::tmem_st_32x32b_x16(t_o + 16, *reinterpret_cast<uint32_t(*)[16]>(&ov[16]));
+              ptx::tmem_wait_st();
+              ls = exp_any(full, t_chunk, m * c2, key0, t_p);
+            }
           }
         }
         if (warp == 0 && lane == 0) atrace<TRACE>(4 + 3 * (c & 7));
@@ -498,7 +590,15 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
   if (p.dt == DT_BF16) {
     // one 128-query tile per CTA, two CTAs per SM (TMEM 256 columns, ~83 KB smem
     // each): one CTA's prologue/epilogue overlaps the other's exp stream
+#if defined(ARLO_ATTN_L128_ALIAS)
+    // A/B only: P aliased over S (128 TMEM columns), three CTAs per SM.  Correct (tests green)
+    // but not faster: at b = 32, 12 heads the 384 CTAs run in one wave (span 8.5 vs 9.5 us in
+    // isolation), yet each CTA serialises S(c+1) behind PV(c) and three CTAs share the MUFU /
+    // TMEM-read budget: 10.6 vs 10.1 us graph-replayed (gpurun_out/ab22)
+    if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
+#else
     if (p.L <= 128) return attn_launch_cfg<1, 1, 2>(p, lengths, o, s);
+#endif
     if (p.L <= 256) return attn_launch_cfg<1, 2, 2>(p, lengths, o, s);
     return attn_launch_cfg<1, 4, 2>(p, lengths, o, s);
   } else {
