@@ -422,12 +422,39 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::tmem_st_32x32b_x8(t_chunk, *reinterpret_cast<uint32_t(*)[8]>(&pk[0]));
           ptx::tmem_st_32x32b_x8(t_chunk + 8, *reinterpret_cast<uint32_t(*)[8]>(&pk[8]));
         } else {
+#if defined(ARLO_ATTN_C0_TWOPASS)  // A/B only: the previous max pass + exp pass over S
           if (c == 0) {
-            // first chunk: row max from a first pass over S, shared by the pair
             xs[par * AQ + r] = half_max(full, t_chunk, key0);
             pair_sync();
             m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
             ls = exp_any(full, t_chunk, m * c2, key0, t_p);
+          } else
+#endif
+          if (c == 0) {
+            // first chunk: row max shared by the pair, then exp, from ONE TMEM read of S
+            // (values kept in registers across the pair barrier; bitwise the two-pass result)
+            uint32_t va[16], vb[16];
+            ptx::tmem_ld_32x32b_x16(t_chunk, va);
+            ptx::tmem_ld_32x32b_x16(t_chunk + 16, vb);
+            ptx::tmem_wait_ld();
+            float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
+#pragma unroll
+            for (int e = 0; e < 16; ++e) {
+              if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+              if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
+            }
+            xs[par * AQ + r] = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
+            pair_sync();
+            m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
+            float l2[2] = {0.f, 0.f};
+            if (full) {
+              exp_piece(std::false_type{}, va, key0, m * c2, t_p, l2);
+              exp_piece(std::false_type{}, vb, key0 + 16, m * c2, t_p + 8, l2);
+            } else {
+              exp_piece(std::true_type{}, va, key0, m * c2, t_p, l2);
+              exp_piece(std::true_type{}, vb, key0 + 16, m * c2, t_p + 8, l2);
+            }
+            ls = l2[0] + l2[1];
           } else {
             // single streaming pass against the (possibly stale) running max.  A row
             // whose p sum passes 2^8 in either half (necessary if any p > 2^8;

@@ -16,7 +16,11 @@ namespace arlo {
 
 namespace {
 
-constexpr int kRowsPerBlock = 8;  // 8 warps, 256 threads
+#ifndef ARLO_LN_ROWS
+#define ARLO_LN_ROWS 16  // rows (warps) per CTA: 16 -> 4.08 us at M=4096 vs 4.40 (8), 4.10 (32); gpurun_out/ab23
+#endif
+constexpr int kRowsPerBlock = ARLO_LN_ROWS;  // one warp per row
+constexpr int kLnThreads = 32 * kRowsPerBlock;
 
 template <typename T> struct Vec;
 template <> struct Vec<bf16> {
@@ -112,7 +116,7 @@ __device__ __forceinline__ void ln_finish(float (&v)[MAXV][Vec<T>::N], int nvec,
 }
 
 template <typename T, int MAXV>
-__global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* __restrict__ in,
+__global__ void __launch_bounds__(kLnThreads) layernorm_kernel(int M, int H, const T* __restrict__ in,
                                                         const float* __restrict__ g,
                                                         const float* __restrict__ b, float eps,
                                                         T* __restrict__ out) {
@@ -134,7 +138,7 @@ __global__ void __launch_bounds__(256) layernorm_kernel(int M, int H, const T* _
 }
 
 template <typename T, int MAXV>
-__global__ void __launch_bounds__(256) embed_ln_kernel(int B, int L, int H, int vocab,
+__global__ void __launch_bounds__(kLnThreads) embed_ln_kernel(int B, int L, int H, int vocab,
                                                        const int32_t* __restrict__ ids,
                                                        const int32_t* __restrict__ lengths,
                                                        const T* __restrict__ word,
@@ -206,7 +210,7 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
   const int vn = dt == DT_BF16 ? 8 : 4;
   if (H % vn) return cudaErrorInvalidValue;
   const int maxv = round_maxv(H / vn);
-  dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
+  dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(kLnThreads);
   if (dt == DT_BF16) {
     ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, 8 * H, s,
         M, H, (const bf16*)in, g, b, eps, (bf16*)out));
@@ -225,7 +229,7 @@ cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int3
   const int vn = dt == DT_BF16 ? 8 : 4;
   if (H % vn) return cudaErrorInvalidValue;
   const int maxv = round_maxv(H / vn);
-  dim3 grid((B * L + kRowsPerBlock - 1) / kRowsPerBlock), block(256);
+  dim3 grid((B * L + kRowsPerBlock - 1) / kRowsPerBlock), block(kLnThreads);
   if (dt == DT_BF16) {
     ARLO_MAXV_SWITCH(maxv, return launch_k(embed_ln_kernel<bf16, MV>, grid, block, 8 * H, s,
         B, L, H, vocab, ids, lengths, (const bf16*)word, (const bf16*)pos, (const bf16*)type, g, b,
