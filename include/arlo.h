@@ -168,6 +168,21 @@ int32_t arlo_runtime_kernel_count(const arlo_runtime* rt, int32_t n);
 int arlo_allocate(int32_t G, int32_t I, const double* Q, const double* M, const double* lat,
                   int32_t nb, int32_t* N_out, double* objective_out);
 
+/*
+ * Instance replacement (§4): "each time Runtime Scheduler resolves
+ * a new allocation, it makes a replacement plan that replaces the minimum number
+ * of current runtime instances".  cur[g] = runtime index of GPU g's instance
+ * (-1 = none), g < G; N_new[I] = the new allocation (sum <= G).  Writes next[G]
+ * (-1 where sum N_new < G) and, if non-NULL, *n_replaced = #{g : next[g] != cur[g]},
+ * which is minimal: GPU g keeps cur[g] while that runtime still needs instances
+ * (lowest GPU indices first); the missing runtimes, in ascending order, go first
+ * to GPUs freed from an oversubscribed runtime, then to idle GPUs.  On B200 a replacement swaps which pre-captured CUDA graphs a
+ * GPU replays (the paper's "hot instances pre-loaded in GPU RAM").  Errors:
+ * EINVAL (G < 1, I < 1, N_new[i] < 0, sum N_new > G, cur[g] out of range).
+ */
+int arlo_replace_plan(int32_t G, int32_t I, const int32_t* cur, const int32_t* N_new, int32_t* next,
+                      int32_t* n_replaced);
+
 /* ------------------------------------------- Request Scheduler (host, C++) */
 typedef struct arlo_sched arlo_sched;
 

@@ -15,6 +15,10 @@ product path's ``arlo_allocate`` / ``arlo_dispatch`` live in C++ under
   outstanding load at the head.
 * ``allocate`` — the Runtime Scheduler program, Eqs. 1-7 (PAPER.md:L181-203
   §3.3), solved by enumerating every composition N_1 + ... + N_I = G.
+* ``replace_plan`` — instance replacement (§4): "a replacement
+  plan that replaces the minimum number of current runtime instances", as its
+  definition: every assignment of the new allocation to the GPUs, the one that
+  changes the fewest GPUs (ties: lexicographically smallest), by brute force.
 
 Readings: S13 both sums of Eqs. 1-2 run over i = 1..I; S14 Eq. 3
 keeps the printed floor; S15 L_i(B) is the profiled batch->latency table,
@@ -168,4 +172,20 @@ def allocate(G: int, Q, M, lat):
             continue
         if best is None or val < best[1]:
             best = (N, val)
+    return best
+
+
+def replace_plan(cur, N_new):
+    """among all per-GPU assignments `nxt` (runtime index or -1) with
+    #{g : nxt[g] == i} == N_new[i] for every i, the one minimising #{g : nxt[g] != cur[g]}.
+    Brute force (tiny G only).  Returns (nxt tuple, n_replaced)."""
+    G, I = len(cur), len(N_new)
+    spare = G - sum(N_new)
+    assert spare >= 0
+    pool = [i for i in range(I) for _ in range(N_new[i])] + [-1] * spare
+    best = None
+    for nxt in sorted(set(itertools.permutations(pool))):
+        changed = sum(1 for g in range(G) if nxt[g] != cur[g])
+        if best is None or changed < best[1]:
+            best = (nxt, changed)
     return best

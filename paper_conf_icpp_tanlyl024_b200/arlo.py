@@ -30,6 +30,7 @@ DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
 
 EXPORTED = [
+    "arlo_replace_plan",
     "arlo_last_error", "arlo_version", "arlo_weights_count", "arlo_weights_create", "arlo_weights_destroy",
     "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
@@ -72,6 +73,7 @@ _sig("arlo_runtime_kernel_count", _i32, _vp, _i32)
 _sig("arlo_runtime_bucket", _i32, _vp, _i32)
 _sig("arlo_sched_set_policy", C.c_int, _vp, _i32)
 _sig("arlo_allocate", C.c_int, _i32, _i32, _P(_f64), _P(_f64), _P(_f64), _i32, _P(_i32), _P(_f64))
+_sig("arlo_replace_plan", C.c_int, _i32, _i32, _P(_i32), _P(_i32), _P(_i32), _P(_i32))
 _sig("arlo_sched_create", C.c_int, _i32, _P(_i32), _P(_i32), _P(_f64), _f64, _f64, _i32, _P(_vp))
 _sig("arlo_sched_destroy", None, _vp)
 _sig("arlo_sched_set_params", C.c_int, _vp, _f64, _f64, _i32)
@@ -209,6 +211,18 @@ def allocate(G: int, Q, M, lat):
     check(lib.arlo_allocate(G, I, Q.ctypes.data_as(_P(_f64)), M.ctypes.data_as(_P(_f64)),
                             lat.ctypes.data_as(_P(_f64)), nb, N, C.byref(obj)))
     return tuple(int(v) for v in N), obj.value
+
+
+def replace_plan(cur, N_new):
+    """arlo_replace_plan: minimum-replacement plan from per-GPU runtime indices
+    cur (-1 = none) to the allocation N_new. Returns (next list, n_replaced)."""
+    G, I = len(cur), len(N_new)
+    c = (_i32 * G)(*cur)
+    nn = (_i32 * I)(*N_new)
+    nxt = (_i32 * G)()
+    rep = _i32()
+    check(lib.arlo_replace_plan(G, I, c, nn, nxt, C.byref(rep)))
+    return [int(v) for v in nxt], int(rep.value)
 
 
 class Scheduler:

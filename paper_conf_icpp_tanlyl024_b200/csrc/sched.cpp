@@ -268,6 +268,53 @@ int arlo_complete(arlo_sched* s, int32_t runtime, int32_t instance) {
   return ARLO_OK;
 }
 
+// Instance replacement plan (§4): after a new allocation N_new, replace the
+// minimum number of current runtime instances.  GPU g keeps its runtime cur[g] while fewer than
+// N_new[cur[g]] GPUs (lowest indices first) have claimed it; the runtimes still missing go, in
+// ascending runtime order, first to the GPUs freed from an oversubscribed runtime, then to idle
+// ones.  GPUs kept = sum_i min(count_i(cur), N_new[i]) + min(#idle, #spare), the most any plan can
+// keep (a matching of equal labels), so the number replaced is minimal.  Deterministic, O(G + I).
+int arlo_replace_plan(int32_t G, int32_t I, const int32_t* cur, const int32_t* N_new, int32_t* next,
+                      int32_t* n_replaced) {
+  using namespace arlo;
+  if (G < 1 || I < 1 || !cur || !N_new || !next)
+    return set_error(ARLO_EINVAL, "arlo_replace_plan: need G >= 1, I >= 1 and non-null arrays");
+  long total = 0;
+  for (int i = 0; i < I; ++i) {
+    if (N_new[i] < 0) return set_error(ARLO_EINVAL, "arlo_replace_plan: N_new[%d] < 0", i);
+    total += N_new[i];
+  }
+  if (total > G) return set_error(ARLO_EINVAL, "arlo_replace_plan: sum N_new = %ld > G = %d", total, G);
+  std::vector<int32_t> kept(I, 0);
+  for (int g = 0; g < G; ++g) {
+    const int32_t r = cur[g];
+    if (r < -1 || r >= I) return set_error(ARLO_EINVAL, "arlo_replace_plan: cur[%d] = %d out of range", g, r);
+    if (r >= 0 && kept[r] < N_new[r]) {
+      next[g] = r;
+      ++kept[r];
+    } else {
+      next[g] = -1;
+    }
+  }
+  // missing runtimes go first to GPUs freed from an oversubscribed runtime (they change in any
+  // case), then to idle GPUs (cur = -1), each group by ascending GPU index; an idle GPU left
+  // without a runtime stays idle (unchanged)
+  int i = 0;
+  for (int pass = 0; pass < 2; ++pass) {
+    for (int g = 0; g < G; ++g) {
+      if (next[g] >= 0 || (pass == 0) != (cur[g] >= 0)) continue;
+      while (i < I && kept[i] >= N_new[i]) ++i;
+      if (i == I) break;
+      next[g] = i;
+      ++kept[i];
+    }
+  }
+  int32_t replaced = 0;
+  for (int g = 0; g < G; ++g) replaced += next[g] != cur[g];
+  if (n_replaced) *n_replaced = replaced;
+  return ARLO_OK;
+}
+
 int32_t arlo_sched_outstanding(const arlo_sched* s, int32_t runtime, int32_t instance) {
   if (!s || runtime < 0 || runtime >= (int)s->levels.size()) return ARLO_EINVAL;
   const Level& l = s->levels[runtime];

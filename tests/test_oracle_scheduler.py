@@ -3,6 +3,7 @@ and hand-derived cases of Algorithm 1 and of the program Eqs. 1-7."""
 import json
 import os
 
+import numpy as np
 import pytest
 
 from oracle import scheduler as osch
@@ -109,3 +110,34 @@ def test_compositions_count():
         comps = list(osch.compositions(G, I))
         assert len(comps) == comb(G + I - 1, I - 1) == len(set(comps))
         assert all(sum(c) == G and len(c) == I for c in comps)
+
+
+# ------------------------------------------------------------------ instance replacement (L272)
+@pytest.mark.parametrize("cur,N_new,expected", [
+    ((0, 0, 1, 2), (1, 2, 1), 1),        # GPU 1 leaves runtime 0 (oversubscribed) for runtime 1
+    ((0, 1, 1, 2), (1, 2, 1), 0),        # allocation unchanged
+    ((-1, -1, -1), (2, 1), 3),           # cold start: every GPU loads an instance
+    ((2, 2, 2, 2), (1, 1, 1, 1), 3),     # one GPU keeps runtime 2, three are replaced
+    ((0, 1, 2), (0, 0, 2), 2),           # runtimes 0, 1 dropped; GPU 2 keeps runtime 2
+    ((0, 1, -1), (1, 1, 0), 0),          # a spare GPU stays spare
+])
+def test_replace_plan_hand_cases(cur, N_new, expected):
+    nxt, changed = osch.replace_plan(list(cur), list(N_new))
+    assert changed == expected
+    assert all(nxt.count(i) == n for i, n in enumerate(N_new))
+
+
+def test_replace_plan_matches_matching_bound():
+    """The minimum number of changed GPUs equals G minus the largest number of GPUs that can keep
+    their state: sum_i min(c_i, N_i) over runtimes plus min(c_-1, spare) idle GPUs (a bipartite
+    matching of equal labels), on random tiny cases."""
+    rng = np.random.default_rng(7)
+    for _ in range(200):
+        G, I = int(rng.integers(1, 6)), int(rng.integers(1, 4))
+        cur = [int(v) for v in rng.integers(-1, I, size=G)]
+        cuts = np.sort(rng.integers(0, G + 1, size=I))
+        N_new = [int(v) for v in np.diff(np.concatenate([[0], cuts]))]
+        spare = G - sum(N_new)
+        keep = sum(min(cur.count(i), N_new[i]) for i in range(I)) + min(cur.count(-1), spare)
+        _nxt, changed = osch.replace_plan(cur, N_new)
+        assert changed == G - keep

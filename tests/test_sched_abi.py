@@ -180,3 +180,32 @@ def test_ilb_ig_hand_cases(arlo_lib):
     with pytest.raises(arlo_lib.ArloError):
         s.set_policy(7)
     s.close()
+
+
+# ------------------------------------------------------------------ instance replacement (L272)
+def test_replace_plan_against_oracle(arlo_lib):
+    """arlo_replace_plan: the replaced count is the oracle's minimum; the plan realises N_new and
+    only moves a GPU whose runtime is oversubscribed in the new allocation (or that had none)."""
+    rng = np.random.default_rng(11)
+    for _ in range(300):
+        G, I = int(rng.integers(1, 6)), int(rng.integers(1, 4))
+        cur = [int(v) for v in rng.integers(-1, I, size=G)]
+        cuts = np.sort(rng.integers(0, G + 1, size=I))
+        N_new = [int(v) for v in np.diff(np.concatenate([[0], cuts]))]
+        nxt, rep = arlo_lib.replace_plan(cur, N_new)
+        _o, rep_o = osch.replace_plan(cur, N_new)
+        assert rep == rep_o
+        assert rep == sum(1 for g in range(G) if nxt[g] != cur[g])
+        assert all(nxt.count(i) == n for i, n in enumerate(N_new))
+        for g in range(G):
+            if nxt[g] != cur[g] and cur[g] >= 0:
+                assert cur.count(cur[g]) > N_new[cur[g]]
+
+
+def test_replace_plan_errors(arlo_lib):
+    with pytest.raises(RuntimeError):
+        arlo_lib.replace_plan([0, 1], [2, 1])       # sum N_new > G
+    with pytest.raises(RuntimeError):
+        arlo_lib.replace_plan([0, 5], [1, 1])       # cur out of range
+    with pytest.raises(RuntimeError):
+        arlo_lib.replace_plan([0, 1], [-1, 1])      # negative N_new
