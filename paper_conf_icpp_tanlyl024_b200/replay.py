@@ -372,3 +372,100 @@ def dispatch_ablation(arlo, torch, runtimes: dict, cfg, G: int = 8, n_requests: 
             row[pol] = {k: r[k] for k in ("mean_ms", "p98_ms", "p99_ms", "slo_violations")}
         res["points"].append(row)
     return res
+
+
+def realloc_replay(arlo, torch, runtimes: dict, cfg, G: int = 8, window_requests: int = 3000,
+                   scales=(1.0, 1.0, 1.6, 1.6, 2.2, 2.2, 1.3, 1.3), slo_ms: float = 150.0, max_batch: int = 32,
+                   stream=None, load: float = 0.9):
+    """Periodic re-allocation + instance replacement.
+    The length distribution drifts window by window (workload.drifting_lengths, `scales`); each
+    window is one Runtime Scheduler period.  "static": the allocation planned on window 0 is kept.
+    "periodic": at the start of window w the allocation is re-solved (arlo_allocate) on the bucket
+    shares OBSERVED in window w-1 and deployed with the minimum-replacement plan
+    (arlo_replace_plan); on B200 a replacement only switches which pre-captured graphs a GPU
+    replays (every GPU holds all runtimes' graphs, the paper's "hot instances pre-loaded in GPU
+    RAM").  Each length level lasts two windows, so the lagged re-plan catches up in the second.
+    Poisson arrivals at `load` x the saturation rate of the window-0 plan on the HEAVIEST window
+    (so the static plan runs near saturation there); windows are
+    simulated one after another (instances drain at the boundary).  Service times are real
+    forwards on this GPU.  Returns per-window latency / SLO violations for both policies and the
+    replacements made."""
+    Ls = sorted(runtimes)
+    dev = torch.device("cuda")
+    lat = profile_runtimes(torch, runtimes, cfg, max_batch, stream)
+    caps = [slo_capacity(row, slo_ms) for row in lat]
+    bufs = {L: (torch.empty((max_batch, L), dtype=torch.int32, device=dev),
+                torch.empty((max_batch,), dtype=torch.int32, device=dev)) for L in Ls}
+    out = torch.empty((max_batch, cfg.num_labels), device=dev)
+    windows = []
+    for w, sc in enumerate(scales):
+        lens = wl.drifting_lengths(window_requests, sc, seed=wl.SEED_ARRIVALS + 100 + w)
+        ids = wl.sample_token_ids(cfg, lens, max(Ls), seed=wl.SEED_ARRIVALS + 200 + w)
+        windows.append((lens, ids))
+
+    def shares_of(lens):
+        ideal = wl.ideal_runtime(lens, Ls)
+        return [float((ideal == k).mean()) for k in range(len(Ls))]
+
+    def factory(max_len, n_inst, capacity, lam, alpha, peek):
+        return arlo.Scheduler(max_len, n_inst, capacity, lam, alpha, peek)
+
+    def run_window(w, n_inst, arrivals):
+        lens, ids = windows[w]
+
+        def service(L, batch):
+            n = len(batch)
+            ids_d, len_d = bufs[L]
+            ids_d[:n].copy_(torch.from_numpy(np.ascontiguousarray(ids[batch, :L])))
+            len_d[:n].copy_(torch.from_numpy(lens[batch].astype(np.int32)))
+            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            runtimes[L].enqueue(n, ids_d, len_d, out)
+            e.record(stream)
+            e.synchronize()
+            return a.elapsed_time(e) / 1e3
+
+        done, rof, _inst, _busy = simulate_cluster(arrivals, lens, Ls, n_inst, caps, service, max_batch, factory)
+        return summarize(arrivals, lens, done, rof, Ls, slo_ms)
+
+    # offered rate: `load` x the saturation rate of the window-0 plan on window 0
+    sh0 = shares_of(windows[0][0])
+
+    def feasible_plan(shares, r):  # Eq. 3 lower bounds can exceed G at a too-high offered rate
+        while True:
+            try:
+                return plan_cluster(arlo, G, Ls, lat, shares, r, slo_ms)[0], r
+            except arlo.ArloError:
+                r *= 0.8
+
+    heavy = int(np.argmax(scales))
+    N0, r0 = feasible_plan(sh0, 1e5)
+    sat = run_window(heavy, N0, np.zeros(window_requests))["served_rate"]
+    N0, rate = feasible_plan(sh0, load * sat)
+    sat = run_window(heavy, N0, np.zeros(window_requests))["served_rate"]
+    rate = load * sat
+    res = {"runtimes": Ls, "G": G, "window_requests": window_requests, "scales": list(scales), "slo_ms": slo_ms,
+           "offered_req_s": rate, "windows": []}
+    gpus = [k for k, n in enumerate(N0) for _ in range(n)] + [-1] * (G - sum(N0))  # runtime index per GPU
+    N_cur = list(N0)
+    for w in range(len(scales)):
+        arrivals = wl.poisson_arrivals(window_requests, rate, seed=wl.SEED_ARRIVALS + 300 + w)
+        n_rep = 0
+        if w > 0:  # re-plan on the previous window's observed shares, minimum replacement
+            N_new, _r = feasible_plan(shares_of(windows[w - 1][0]), rate)
+            gpus, n_rep = arlo.replace_plan(gpus, list(N_new))
+            N_cur = [gpus.count(k) for k in range(len(Ls))]
+        st = run_window(w, list(N0), arrivals)
+        pe = run_window(w, N_cur, arrivals)
+        res["windows"].append({
+            "scale": scales[w], "mean_len": float(windows[w][0].mean()),
+            "static": {"instances": {str(L): int(N0[k]) for k, L in enumerate(Ls)}, "mean_ms": st["mean_ms"],
+                       "p99_ms": st["p99_ms"], "slo_violations": st["slo_violations"]},
+            "periodic": {"instances": {str(L): int(N_cur[k]) for k, L in enumerate(Ls)}, "replaced": n_rep,
+                         "mean_ms": pe["mean_ms"], "p99_ms": pe["p99_ms"], "slo_violations": pe["slo_violations"]}})
+    for pol in ("static", "periodic"):
+        res[pol + "_overall_slo_violations"] = float(np.mean([w_[pol]["slo_violations"] for w_ in res["windows"]]))
+        res[pol + "_worst_p99_ms"] = float(max(w_[pol]["p99_ms"] for w_ in res["windows"]))
+        res[pol + "_mean_ms"] = float(np.mean([w_[pol]["mean_ms"] for w_ in res["windows"]]))
+    res["replacements_total"] = int(sum(w_["periodic"]["replaced"] for w_ in res["windows"]))
+    return res

@@ -179,6 +179,16 @@ def sample_lengths(n: int, seed: int = SEED_LENGTHS, lo: int = 0, hi: int = 512)
     return lens
 
 
+def drifting_lengths(n: int, scale: float, seed: int = SEED_LENGTHS) -> np.ndarray:
+    """Lengths of one re-allocation window whose distribution has drifted: the base skewed lengths
+    multiplied by `scale` (re-rounded, clamped to [2, 512]).  A synthetic stand-in for the
+    coarse-time-scale shifts of the length distribution the Runtime Scheduler tracks
+    (§1, "every 10 minutes"; period 120 s, L299).  Generator only: no method
+    arithmetic."""
+    base = sample_lengths(n, seed=seed)
+    return np.clip(np.rint(base * scale), 2, 512).astype(np.int32)
+
+
 def sample_token_ids(cfg: ModelConfig, lengths: np.ndarray, L: int, seed: int = SEED_TOKENS) -> np.ndarray:
     """[b, L] int32 ids: CLS, uniform body, SEP, zero padding (reading S12)."""
     rng = np.random.default_rng(seed)

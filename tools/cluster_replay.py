@@ -1,6 +1,6 @@
 """Cluster replay only (BASELINE configs[3] / [4]): ILP-placed runtimes on G virtual GPUs.
 
-    python tools/cluster_replay.py [base|roberta|ablation] [n_requests]
+    python tools/cluster_replay.py [base|roberta|ablation|realloc] [n_requests] [G (realloc)] [load (realloc)]
 """
 import json
 import os
@@ -16,7 +16,8 @@ from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
 def main():
     model = sys.argv[1] if len(sys.argv) > 1 else "base"
     ablation = model == "ablation"
-    if ablation:
+    realloc = model == "realloc"
+    if ablation or realloc:
         model = "base"
     n = int(sys.argv[2]) if len(sys.argv) > 2 else 6000
     cfg = wl.ROBERTA_LARGE if model == "roberta" else wl.BERT_BASE
@@ -28,6 +29,14 @@ def main():
     for L in wl.RUNTIME_LENGTHS:
         rts[L] = arlo.Runtime(W, L, 32)
         rts[L].set_stream(s)
+    if realloc:
+        G = int(sys.argv[3]) if len(sys.argv) > 3 else 8
+        load = float(sys.argv[4]) if len(sys.argv) > 4 else 0.9
+        res = replay.realloc_replay(arlo, torch, rts, cfg, G=G, window_requests=n // 2, slo_ms=slo, max_batch=32,
+                                    stream=s, load=load)
+        res["model"] = cfg.name
+        print(json.dumps(res))
+        return
     if ablation:
         res = replay.dispatch_ablation(arlo, torch, rts, cfg, G=8, n_requests=n, slo_ms=slo, max_batch=32, stream=s)
         res["model"] = cfg.name
