@@ -165,12 +165,26 @@ __device__ __forceinline__ void epi_pack4(const uint32_t* r, float4 b4, uint32_t
   p1 = pack_bf16x2(x1.x, x1.y);
 }
 
+// Residual of this warp's first chunk of a tile (row row0 + lane, columns n0 + 32 cg ...): the
+// residual never depends on the MMA, so the epilogue warps load it BEFORE waiting for the
+// accumulator, taking its L2 latency off the exposed epilogue of one-round GEMMs.
+template <int BN, int EPI>
+__device__ __forceinline__ void prefetch_first_resid(uint4 (&rv)[CW / 8], const bf16* resid, int row0, int lane,
+                                                     int n0, int cg, int M, int ldr) {
+  if (EPI != EPI_BIAS_RESID || cg * CW >= BN) return;  // (a warp without chunks loads nothing)
+  const int row = row0 + lane;
+  if (row >= M) return;
+  const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0) + cg * (CW / 8);
+#pragma unroll
+  for (int j = 0; j < CW / 8; ++j) rv[j] = ld_dep_v4(res4 + j);
+}
+
 template <int BN, int EPI, int kEpiGroups, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int ldr, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
                                               uint8_t* stg, int& sc, Release release, bf16* __restrict__ outp,
-                                              int N) {
+                                              int N, const uint4* rv_first) {
   static_assert(BN % CW == 0, "tile width must be a multiple of 32");
   constexpr int NCH = BN / CW;                                 // chunks per row block
   constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;  // chunks per warp (max)
@@ -188,9 +202,9 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   }
   uint32_t r[2][CW];
   uint4 rv[2][RV];
-  if (EPI == EPI_BIAS_RESID && row_ok) {
+  if (EPI == EPI_BIAS_RESID && row_ok) {  // prefetched by the caller before the accumulator wait
 #pragma unroll
-    for (int j = 0; j < RV; ++j) rv[0][j] = ld_dep_v4(res4 + cg * RV + j);
+    for (int j = 0; j < RV; ++j) rv[0][j] = rv_first[j];
   }
   ptx::tmem_ld_32x32b_x32(t_row + cg * CW, r[0]);
   ptx::tmem_wait_ld();
@@ -392,12 +406,14 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     int it = 0;
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
       const int m0 = tile_m(tile, num_m, num_n) * BM, n0 = tile_n(tile, num_m, num_n) * BN;
+      uint4 rv0[CW / 8];
+      prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
       epilogue_tile<BN, EPI, kEpiGroups>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid,
-                                         &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N);
+                                         &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N, rv0);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -556,6 +572,8 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     int it = 0;
     for (int tile = pair; tile < tiles; tile += npairs, ++it) {
       const int m0 = tile_m(tile, num_m, num_n) * 2 * BM + rank * BM, n0 = tile_n(tile, num_m, num_n) * BN;
+      uint4 rv0[CW / 8];
+      prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
       ptx::mbar_wait(&tfull[acc], acc_phase);
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
@@ -568,7 +586,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
 #else
                                ptx::mbar_arrive_remote(te);
 #endif
-                             }, outp, N);
+                             }, outp, N, rv0);
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
