@@ -374,6 +374,23 @@ def dispatch_ablation(arlo, torch, runtimes: dict, cfg, G: int = 8, n_requests: 
     return res
 
 
+def periodic_plans(arlo, N0, window_shares, plan_fn):
+    """Deployments of the periodic policy: window 0 runs N0; at the start of
+    window w >= 1 the allocation plan_fn(shares observed in window w-1) is deployed on the GPUs
+    with the minimum-replacement plan (arlo_replace_plan).  Returns [(N per runtime, replaced)]
+    per window.  Host logic only (tests run it on the CPU)."""
+    I = len(N0)
+    G = int(sum(N0))
+    gpus = [k for k, n in enumerate(N0) for _ in range(n)]  # runtime index per GPU
+    out = [(list(N0), 0)]
+    for w in range(1, len(window_shares)):
+        N_new = list(plan_fn(window_shares[w - 1]))
+        assert sum(N_new) <= G
+        gpus, n_rep = arlo.replace_plan(gpus, N_new)
+        out.append(([gpus.count(k) for k in range(I)], n_rep))
+    return out
+
+
 def realloc_replay(arlo, torch, runtimes: dict, cfg, G: int = 8, window_requests: int = 3000,
                    scales=(1.0, 1.0, 1.6, 1.6, 2.2, 2.2, 1.3, 1.3), slo_ms: float = 150.0, max_batch: int = 32,
                    stream=None, load: float = 0.9):
@@ -446,15 +463,11 @@ def realloc_replay(arlo, torch, runtimes: dict, cfg, G: int = 8, window_requests
     rate = load * sat
     res = {"runtimes": Ls, "G": G, "window_requests": window_requests, "scales": list(scales), "slo_ms": slo_ms,
            "offered_req_s": rate, "windows": []}
-    gpus = [k for k, n in enumerate(N0) for _ in range(n)] + [-1] * (G - sum(N0))  # runtime index per GPU
-    N_cur = list(N0)
+    plans = periodic_plans(arlo, N0, [shares_of(lens) for lens, _ids in windows],
+                           lambda sh: feasible_plan(sh, rate)[0])
     for w in range(len(scales)):
         arrivals = wl.poisson_arrivals(window_requests, rate, seed=wl.SEED_ARRIVALS + 300 + w)
-        n_rep = 0
-        if w > 0:  # re-plan on the previous window's observed shares, minimum replacement
-            N_new, _r = feasible_plan(shares_of(windows[w - 1][0]), rate)
-            gpus, n_rep = arlo.replace_plan(gpus, list(N_new))
-            N_cur = [gpus.count(k) for k in range(len(Ls))]
+        N_cur, n_rep = plans[w]
         st = run_window(w, list(N0), arrivals)
         pe = run_window(w, N_cur, arrivals)
         res["windows"].append({

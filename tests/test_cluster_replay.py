@@ -66,3 +66,27 @@ def test_plan_cluster_satisfies_eqs_2_and_7(arlo_lib):
         N, Q, M = replay.plan_cluster(arlo_lib, G, Ls, lat, shares, 20000.0 * G, 150.0)
         assert sum(N) == G and N[-1] >= 1  # Eq. 2, Eq. 7
         assert all(n >= np.floor(q / m) for n, q, m in zip(N, Q, M))  # Eq. 3
+
+
+def test_periodic_plans_track_the_drift_with_minimum_replacement(arlo_lib):
+    """SURVEY NEXT-3 host logic: each window deploys the allocation planned on the previous window's
+    shares, reached from the current deployment by the minimum number of replaced
+    instances (L272): |N_new - N_cur|_1 / 2 when every GPU is used."""
+    Ls = [64, 128, 256, 512]
+    lat = np.array([[0.2 + 0.01 * b * k for b in range(1, 33)] for k in range(1, 5)])
+    shares = [[0.7, 0.2, 0.05, 0.05], [0.7, 0.2, 0.05, 0.05], [0.1, 0.2, 0.3, 0.4], [0.1, 0.2, 0.3, 0.4]]
+    G, rate, slo = 8, 2e5, 150.0
+
+    def plan(sh):
+        return replay.plan_cluster(arlo_lib, G, Ls, lat, sh, rate, slo)[0]
+
+    N0 = plan(shares[0])
+    plans = replay.periodic_plans(arlo_lib, N0, shares, plan)
+    assert plans[0] == (list(N0), 0)
+    for w in range(1, len(shares)):
+        N_w, rep = plans[w]
+        assert N_w == list(plan(shares[w - 1]))
+        prev = plans[w - 1][0]
+        assert rep == sum(abs(a - b) for a, b in zip(N_w, prev)) // 2
+        assert sum(N_w) == G and N_w[-1] >= 1          # Eqs. 2 and 7 hold after the replacement
+    assert plans[2][0] != plans[1][0]                   # the drift changed the deployment
