@@ -146,6 +146,13 @@ int32_t arlo_runtime_bucket(const arlo_runtime* rt, int32_t n);
 /* Number of kernels one forward at bucket b launches (graph node count). */
 int32_t arlo_runtime_kernel_count(const arlo_runtime* rt, int32_t n);
 
+/* Tile codes of the four GEMMs (QKV, out-proj, FFN1, FFN2; 0 = not a tensor-core GEMM, e.g.
+ * fp32 check mode) captured in the graph serving n requests.  Codes: BN single CTA, -BN CTA
+ * pair, 1000 + BN skinny.  bf16 runtimes pick them at create time by timing every valid tile on
+ * the device (ARLO_NO_AUTOTUNE=1: the analytic chooser); results are bitwise independent of the
+ * tile.  Writes codes[4].  Errors: EINVAL. */
+int arlo_runtime_gemm_tiles(const arlo_runtime* rt, int32_t n, int32_t* codes);
+
 /* ------------------------------------------- Runtime Scheduler (host, C++) */
 /*
  * Allocation program of PAPER.md:L181-203 (§3.3, Eqs. 1-7):

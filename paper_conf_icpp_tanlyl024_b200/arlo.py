@@ -30,7 +30,7 @@ DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
 
 EXPORTED = [
-    "arlo_replace_plan",
+    "arlo_replace_plan", "arlo_runtime_gemm_tiles",
     "arlo_last_error", "arlo_version", "arlo_weights_count", "arlo_weights_create", "arlo_weights_destroy",
     "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
@@ -71,6 +71,7 @@ _sig("arlo_infer", C.c_int, _vp, _vp, _vp, _vp)
 _sig("arlo_enqueue", C.c_int, _vp, _i32, _vp, _vp, _vp)
 _sig("arlo_runtime_kernel_count", _i32, _vp, _i32)
 _sig("arlo_runtime_bucket", _i32, _vp, _i32)
+_sig("arlo_runtime_gemm_tiles", C.c_int, _vp, _i32, _P(_i32))
 _sig("arlo_sched_set_policy", C.c_int, _vp, _i32)
 _sig("arlo_allocate", C.c_int, _i32, _i32, _P(_f64), _P(_f64), _P(_f64), _i32, _P(_i32), _P(_f64))
 _sig("arlo_replace_plan", C.c_int, _i32, _i32, _P(_i32), _P(_i32), _P(_i32), _P(_i32))
@@ -182,6 +183,12 @@ class Runtime:
 
     def kernel_count(self, n: int) -> int:
         return check(lib.arlo_runtime_kernel_count(self.handle, n))
+
+    def gemm_tiles(self, n: int):
+        """Tile codes (QKV, out-proj, FFN1, FFN2) of the graph serving n requests."""
+        codes = (_i32 * 4)()
+        check(lib.arlo_runtime_gemm_tiles(self.handle, n, codes))
+        return [int(v) for v in codes]
 
     def infer(self, token_ids, lengths, logits):
         """Synchronous; each argument a torch tensor (host or device) or numpy array."""

@@ -160,6 +160,7 @@ struct Bucket {
   int b = 0;
   std::vector<LayerPlans> plans;  // bf16 only
   bool fused_ln = false;          // o / f2 plans carry residual + LayerNorm (no separate LN kernels)
+  int tiles[4] = {0, 0, 0, 0};    // measured tile codes of the qkv, o, f1, f2 GEMMs (pick_tile)
   AttnPlan attn;
   // CLS-only last layer (bf16): only position 0 of each sequence feeds the pooler
   // (reading S8), so after the last layer's QKV projection and the attention of
@@ -265,6 +266,45 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
   return ARLO_OK;
 }
 
+// Build-time tile selection ("tactics", as a TensorRT engine build times its kernels): for one
+// GEMM shape of the runtime, time every valid tile code on the runtime's stream (layer-0 buffers,
+// 1 warm-up + 3 timed launches each) and keep the fastest; the analytic chooser's pick is one of
+// the candidates and wins ties.  Every tile code computes each output element with the same K
+// chain, so the choice changes time only, never a bit of the result (tile-width bitwise tests).
+// ARLO_NO_AUTOTUNE=1 keeps the analytic chooser.
+template <typename PlanFn>
+static int pick_tile(int M, int N, int K, cudaStream_t s, PlanFn plan) {
+  const int base = tc_choose_bn(M, N, K);
+  if (getenv("ARLO_NO_AUTOTUNE") != nullptr) return base;
+  std::vector<int> cands = {base};
+  for (int code : {-256, -192, -128, 256, 192, 128, 96, 64})
+    if (code != base && N % (code < 0 ? -code : code) == 0) cands.push_back(code);
+  if (M <= 1024)
+    for (int bn : {16, 32, 64})
+      if (kSkinnyCode + bn != base && N % bn == 0) cands.push_back(kSkinnyCode + bn);
+  cudaEvent_t e0, e1;
+  if (cudaEventCreate(&e0) != cudaSuccess) return base;
+  if (cudaEventCreate(&e1) != cudaSuccess) { cudaEventDestroy(e0); return base; }
+  int best = base;
+  float best_ms = 1e30f;
+  for (int code : cands) {
+    TcGemmPlan p;
+    if (!plan(&p, code)) continue;
+    if (tc_launch_gemm(p, s) != cudaSuccess) { cudaGetLastError(); continue; }
+    cudaEventRecord(e0, s);
+    bool ok = true;
+    for (int r = 0; r < 3 && ok; ++r) ok = tc_launch_gemm(p, s) == cudaSuccess;
+    cudaEventRecord(e1, s);
+    if (!ok || cudaEventSynchronize(e1) != cudaSuccess) { cudaGetLastError(); continue; }
+    float ms = 0.f;
+    cudaEventElapsedTime(&ms, e0, e1);
+    if (ms < best_ms * 0.98f) { best_ms = ms; best = code; }  // a candidate must beat the incumbent by 2 %
+  }
+  cudaEventDestroy(e0);
+  cudaEventDestroy(e1);
+  return best;
+}
+
 static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
   const arlo_weights* w = rt->w;
   const arlo_model_config& c = w->cfg;
@@ -278,12 +318,28 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
   bk.fused_ln = getenv("ARLO_FUSED_LN") != nullptr &&
                 tc_plan_gemm_ln(&probe, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X,
                                 (const float*)w->lt(0, LN1_G), (const float*)w->lt(0, LN1_B), c.ln_eps, rt->X);
+  // one tile code per GEMM shape of this bucket, measured on layer 0's buffers
+  cudaStream_t ts = rt->own_stream;
+  const int t_qkv = pick_tile(M, 3 * H, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, 3 * H, H, rt->X, w->lt(0, LW_QKV), (const float*)w->lt(0, LB_QKV), nullptr, rt->QKV,
+                        EPI_BIAS, code); });
+  const int t_f1 = pick_tile(M, F, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, F, H, rt->X, w->lt(0, LW_1), (const float*)w->lt(0, LB_1), nullptr, rt->F,
+                        EPI_BIAS_GELU, code); });
+  const int t_o = bk.fused_ln ? 0 : pick_tile(M, H, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X, rt->Y,
+                        EPI_BIAS_RESID, code); });
+  const int t_f2 = bk.fused_ln ? 0 : pick_tile(M, H, F, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, H, F, rt->F, w->lt(0, LW_2), (const float*)w->lt(0, LB_2), rt->X, rt->Y,
+                        EPI_BIAS_RESID, code); });
+  if (cudaStreamSynchronize(ts) != cudaSuccess) return set_error(ARLO_ECUDA, "tile selection failed");
+  bk.tiles[0] = t_qkv; bk.tiles[1] = t_o; bk.tiles[2] = t_f1; bk.tiles[3] = t_f2;
   for (int l = 0; l < c.layers; ++l) {
     LayerPlans& p = bk.plans[l];
     bool ok = tc_plan_gemm(&p.qkv, M, 3 * H, H, rt->X, w->lt(l, LW_QKV), (const float*)w->lt(l, LB_QKV), nullptr,
-                           rt->QKV, EPI_BIAS, 0) &&
+                           rt->QKV, EPI_BIAS, t_qkv) &&
               tc_plan_gemm(&p.f1, M, F, H, rt->X, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, rt->F,
-                           EPI_BIAS_GELU, 0);
+                           EPI_BIAS_GELU, t_f1);
     if (bk.fused_ln) {
       ok = ok &&
            tc_plan_gemm_ln(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X,
@@ -293,9 +349,9 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
     } else {
       ok = ok &&
            tc_plan_gemm(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y,
-                        EPI_BIAS_RESID, 0) &&
+                        EPI_BIAS_RESID, t_o) &&
            tc_plan_gemm(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, rt->Y,
-                        EPI_BIAS_RESID, 0);
+                        EPI_BIAS_RESID, t_f2);
     }
     if (!ok) return set_error(ARLO_ECUDA, "tensor-map encoding failed (cuTensorMapEncodeTiled unavailable?)");
   }
@@ -325,6 +381,14 @@ static void destroy_runtime(arlo_runtime* rt) {
   if (rt->h_stage) cudaFreeHost(rt->h_stage);
   if (rt->own_stream) cudaStreamDestroy(rt->own_stream);
   delete rt;
+}
+
+extern "C" int arlo_runtime_gemm_tiles(const arlo_runtime* rt, int32_t n, int32_t* codes) {
+  if (!rt || !codes) return set_error(ARLO_EINVAL, "arlo_runtime_gemm_tiles: null argument");
+  const int k = bucket_index(rt, n);
+  if (k < 0) return set_error(ARLO_EINVAL, "arlo_runtime_gemm_tiles: n = %d exceeds max_batch", n);
+  for (int i = 0; i < 4; ++i) codes[i] = rt->buckets[k].tiles[i];
+  return ARLO_OK;
 }
 
 extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out) {

@@ -197,3 +197,24 @@ def test_cls_only_last_layer_is_bitwise(arlo_lib, monkeypatch, L, max_batch):
     np.testing.assert_array_equal(pruned, full)
     ref = orc.forward_batch(cfg, w, ids, lengths)
     assert np.max(np.abs(pruned - ref)) <= 2e-2
+
+
+@pytest.mark.gpu
+def test_autotuned_tiles_are_bitwise_the_analytic_choice(arlo_lib, monkeypatch):
+    """Build-time tile selection (pick_tile) changes only which tile codes the graphs use: the
+    logits of an autotuned runtime equal those of one built with the analytic chooser bit for bit,
+    and every selected code is a valid tile code."""
+    cfg = wl.BERT_BASE
+    w, W = weights(arlo_lib, cfg, 0)
+    L, mb = 128, 32
+    lengths = wl.sample_lengths(mb, seed=21, lo=0, hi=L)
+    ids = wl.sample_token_ids(cfg, lengths, L, seed=22)
+    rt = arlo_lib.Runtime(W, L, mb)
+    tiles = {n: rt.gemm_tiles(n) for n in (1, 8, 32)}
+    rt.close()
+    valid = {-256, -192, -128, 256, 192, 128, 96, 64, 1016, 1032, 1064}
+    assert all(c in valid for codes in tiles.values() for c in codes), tiles
+    out_tuned = run(arlo_lib, W, L, mb, ids, lengths)
+    monkeypatch.setenv("ARLO_NO_AUTOTUNE", "1")
+    out_plain = run(arlo_lib, W, L, mb, ids, lengths)
+    assert np.array_equal(out_tuned, out_plain)
