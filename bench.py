@@ -290,6 +290,9 @@ def main():
 
     if rank == 0 and not args.no_extras:
         result["roofline"] = roofline_dominant(arlo, torch, dev, stream, step_times)
+        result["gemm_tiles"] = {"note": "QKV, out-proj, FFN1, FFN2 tile codes per batch bucket, timed on the device at "
+                                        "runtime creation (BN single CTA, -BN CTA pair, 1000+BN skinny)",
+                                **{str(L): {str(n): rt.gemm_tiles(n) for n in (1, 8, 16, 32)} for L, rt in runtimes.items()}}
         result["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
         result["per_L_latency_ms_restricted"] = per_L_table(runtimes, torch, dev, stream, cfg, restricted=True)
         pl = result["per_L_latency_ms"]
