@@ -223,6 +223,12 @@ def main():
     if world > 1:
         dist.barrier()
 
+    # ncu launch lists (tools/profile_round.sh): with ARLO_PROFILE_TIMED=1 and
+    # `ncu --profile-from-start off` only the timed steps are captured, not runtime creation
+    # (its build-time tile timing launches every tile variant) or warm-up
+    profile_timed = os.environ.get("ARLO_PROFILE_TIMED") == "1"
+    if profile_timed:
+        torch.cuda.cudart().cudaProfilerStart()
     sampler = ClockSampler(local_rank)
     sampler.start()
     time.sleep(0.3)
@@ -246,6 +252,8 @@ def main():
     if world > 1:
         dist.barrier()
     clocks = sampler.stop()
+    if profile_timed:
+        torch.cuda.cudart().cudaProfilerStop()
     step_times = [a.elapsed_time(b) for a, b in step_ms]
     total_ms = float(sum(step_times))
     # per-bucket latency: a request's latency = its forward's duration (all arrive at step start,

@@ -5,7 +5,7 @@ set -x
 mkdir -p gpurun_out/prof
 python __graft_entry__.py > /dev/null
 timeout 900 python bench.py > gpurun_out/prof/bench.json 2> gpurun_out/prof/bench.err
-timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv \
+ARLO_PROFILE_TIMED=1 timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv \
     --log-file gpurun_out/prof/launches.csv python bench.py --steps 2 --warmup 1 --no-extras --no-cpu-baseline \
     > gpurun_out/prof/bench_under_ncu.log 2>&1
 python tools/forward_breakdown.py --summarize gpurun_out/prof/launches.csv > gpurun_out/prof/launches_summary.txt 2>&1
