@@ -59,3 +59,12 @@ def test_arrivals():
     assert abs(len(t) / t[-1] - 1000) < 30
     t2 = wl.mmpp_arrivals(20000, 1000.0)
     assert np.all(np.diff(t2) >= 0) and 700 < len(t2) / t2[-1] < 1300
+
+
+def test_drifting_lengths_scale_and_range():
+    """Re-allocation windows (replay.realloc_replay): the base skewed lengths scaled, clamped to [2, 512]."""
+    base = wl.sample_lengths(5000, seed=4)
+    d = wl.drifting_lengths(5000, 1.6, seed=4)
+    assert d.min() >= 2 and d.max() <= 512
+    assert np.array_equal(wl.drifting_lengths(5000, 1.0, seed=4), base)
+    assert 1.4 < d.mean() / base.mean() < 1.65  # clamping at 512 trims the scaled tail
