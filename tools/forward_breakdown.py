@@ -24,7 +24,8 @@ def summarize(path):
             continue
         name = r[ki].split("(")[0].replace("arlo::<unnamed>::", "").replace("void ", "")[:44]
         v = float(r[vi].replace(",", ""))
-        v *= {"nsecond": 1e-3, "usecond": 1.0, "msecond": 1e3}.get(r[ui], 1.0)
+        v *= {"nsecond": 1e-3, "ns": 1e-3, "usecond": 1.0, "us": 1.0,
+              "msecond": 1e3, "ms": 1e3}.get(r[ui], 1.0)
         agg[name][0] += 1
         agg[name][1] += v
     tot = sum(v[1] for v in agg.values())
