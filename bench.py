@@ -9,7 +9,10 @@ with idle instances) and each runtime runs ceil(n_L / 32) static-shape
 forwards (embedding -> 12 x {QKV, masked attention, out-proj, LN, FFN1, FFN2,
 LN} -> pooler/classifier).  value = requests / second over the timed steps.
 
-Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl arlo|reference]
+Usage:  python bench.py [--gpus N] [--steps K] [--warmup W] [--impl arlo|reference] [--full]
+The last stdout line is one compact JSON object (the headline: value, per-bucket latency,
+roofline, cpu_baseline, e2e, clocks); the per-L tables, the ST-512 baseline, the BERT-large
+table, the GEMM roofline table and the oracle-timing details go to --extras-out.
 Under torchrun each rank serves its own R requests per step on its own GPU
 (independent replicas, no data-path collective; weak scaling); timing is
 the max over ranks.  `--impl reference` times the fp64 CPU oracle on the
@@ -37,6 +40,7 @@ from paper_conf_icpp_tanlyl024_b200 import workload as wl  # noqa: E402
 RUNTIME_LS = (64, 128, 256, 512)
 MAX_BATCH = 32
 METRIC = "BERT-base req/s & mean/p99 latency per length bucket; tensor-pipe util"
+WORKLOAD = "bert-base polymorphed runtimes L{64,128,256,512}, batch buckets <=32 (BASELINE configs[1])"
 
 
 def parse():
@@ -48,6 +52,11 @@ def parse():
     p.add_argument("--requests", type=int, default=512, help="requests per step per GPU")
     p.add_argument("--no-cpu-baseline", action="store_true")
     p.add_argument("--no-extras", action="store_true", help="skip per-L table / ST-512 / e2e (profiling runs)")
+    p.add_argument("--full", action="store_true", help="also run the trace replay and the cluster replay")
+    p.add_argument("--extras-out", default=os.path.join(ROOT, "gpurun_out", "bench_extras.json"),
+                   help="where the per-L tables, ST-512, BERT-large and oracle-timing details are written")
+    p.add_argument("--cpu-trace-requests", type=int, default=64, help="oracle trace-sample size (cpu_baseline)")
+    p.add_argument("--ref-requests", type=int, default=4, help="--impl reference: requests per step")
     return p.parse_args()
 
 
@@ -111,14 +120,30 @@ class ClockSampler:
                 "sm_max_mhz": max(mx) if mx else None, "reasons": reasons, "samples": len(self.rows)}
 
 
-# ------------------------------------------------------------------------- reference arm
-def run_reference(args, rank):
-    """The oracle, as it stands, timed on this host's cores on bounded samples of the workload."""
-    from oracle import encoder as orc
+# ------------------------------------------------------------------------- oracle timing
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except OSError:
+        pass
+    import platform
+    return platform.processor() or "unknown"
+
+
+def blas_threads() -> int:
     import threadpoolctl
+    return max((d.get("num_threads", 1) for d in threadpoolctl.threadpool_info()), default=1)
+
+
+def run_reference(args, rank):
+    """The oracle, as it stands, timed on this host's cores on bounded samples of the workload
+    (each step: the first `--ref-requests` requests of that step's skewed draw, real prefixes)."""
+    from oracle import encoder as orc
     cfg = wl.BERT_BASE
     w = wl.make_weights(cfg)
-    per_step = 4
+    per_step = args.ref_requests
     times, n_req = [], 0
     for step in range(args.warmup + args.steps):
         lengths = make_step_requests(step, rank, args.requests, cfg)[:per_step]
@@ -131,35 +156,78 @@ def run_reference(args, rank):
             times.append(dt)
             n_req += len(lengths)
     total = sum(times)
-    threads = max((d.get("num_threads", 1) for d in threadpoolctl.threadpool_info()), default=1)
     value = n_req / total
-    sample = f"{per_step} requests/step of the skewed length distribution (real prefixes, fp64 numpy)"
+    sample = (f"{per_step} requests/step of the skewed length distribution (real prefixes, fp64 numpy), "
+              f"{os.cpu_count()} host cores ({cpu_model()})")
     return {"metric": METRIC, "value": value, "unit": "req/s", "impl": "reference", "n_gpus": args.gpus,
             "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total / len(times),
             "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "f64",
-            "data": "synthetic", "config": {"workload": "bert-base polymorphed L{64,128,256,512} b<=32",
-                                            "sample": sample},
-            "cpu_baseline": {"value": value, "unit": "req/s", "cores": threads, "kind": "oracle", "sample": sample},
+            "data": "synthetic", "config": {"workload": WORKLOAD, "sample": sample},
+            "cpu_baseline": {"value": value, "unit": "req/s", "cores": blas_threads(), "kind": "oracle",
+                             "sample": sample},
             "e2e": {"value": value, "unit": "req/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
 
 
-def cpu_baseline(seconds=15.0):
-    from oracle import encoder as orc
+def cpu_baseline(trace_requests=64, one_thread_requests=8):
+    """Oracle timing plan: the oracle as it stands on this host's cores, on
+    bounded samples: (i) the tiny config (configs[0], L=32 b=4); (ii) a per-L subsample (BERT-base
+    b=2 per L, BERT-large b=1 per L, every request of length L); (iii) a subsample of the skewed
+    trace (the compact line's value, req/s); (iv) the same trace requests with BLAS limited to one
+    thread."""
     import threadpoolctl
+    from oracle import encoder as orc
+    out = {"kind": "oracle", "unit": "req/s", "cores": blas_threads(), "host_cpus": os.cpu_count(),
+           "cpu_model": cpu_model()}
+    # (i) tiny
+    cfg = wl.TINY
+    w = wl.make_weights(cfg)
+    lens = np.array([32, 17, 1, 2], np.int32)
+    ids = wl.sample_token_ids(cfg, lens, 32)
+    t0 = time.perf_counter()
+    orc.forward_batch(cfg, w, ids, lens)
+    out["tiny_L32_b4_ms"] = 1e3 * (time.perf_counter() - t0)
+    # (ii) per-L subsample
+    per_L = {}
+    for cfg, Ls, b in ((wl.BERT_BASE, (64, 128, 256, 512), 2), (wl.BERT_LARGE, (128, 256, 512), 1)):
+        w = wl.make_weights(cfg)
+        row = {}
+        for L in Ls:
+            lens = np.full(b, L, np.int32)
+            ids = wl.sample_token_ids(cfg, lens, L, seed=5)
+            t0 = time.perf_counter()
+            orc.forward_batch(cfg, w, ids, lens)
+            row[str(L)] = 1e3 * (time.perf_counter() - t0) / b
+        per_L[cfg.name] = row
+    out["per_L_ms_per_request"] = per_L
+    # (iii) trace subsample
     cfg = wl.BERT_BASE
     w = wl.make_weights(cfg)
-    lengths = wl.sample_lengths(256, seed=wl.SEED_LENGTHS + 999)
+    lengths = wl.sample_lengths(trace_requests, seed=wl.SEED_LENGTHS + 999)
     ids = wl.sample_token_ids(cfg, lengths, 512, seed=wl.SEED_TOKENS + 999)
     t0 = time.perf_counter()
-    n = 0
-    while n < len(lengths) and (time.perf_counter() - t0 < seconds or n < 4):
-        orc.forward_request(cfg, w, ids[n, :lengths[n]])
-        n += 1
+    for i in range(trace_requests):
+        orc.forward_request(cfg, w, ids[i, :lengths[i]])
     dt = time.perf_counter() - t0
-    threads = max((d.get("num_threads", 1) for d in threadpoolctl.threadpool_info()), default=1)
-    return {"value": n / dt, "unit": "req/s", "cores": threads, "kind": "oracle",
-            "sample": f"{n} requests of the skewed distribution (mean len {lengths[:n].mean():.1f}), "
-                      f"real prefixes, numpy fp64, {dt:.1f} s, {os.cpu_count()} host cores"}
+    out["value"] = trace_requests / dt
+    out["sample"] = (f"{trace_requests} requests of the skewed trace (mean len {lengths.mean():.1f}), real prefixes, "
+                     f"numpy fp64 on {os.cpu_count()} host cores, {dt:.1f} s")
+    # (iv) one BLAS thread, first requests of the same sample
+    with threadpoolctl.threadpool_limits(1):
+        t0 = time.perf_counter()
+        for i in range(one_thread_requests):
+            orc.forward_request(cfg, w, ids[i, :lengths[i]])
+        dt1 = time.perf_counter() - t0
+    out["one_thread_value"] = one_thread_requests / dt1
+    out["one_thread_sample"] = f"first {one_thread_requests} requests of the same sample, 1 BLAS thread"
+    return out
+
+
+def load_peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json"))), "MEASURED_PEAKS.json"
+    except Exception:
+        return {"bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0, "hbm_gbs": 6650.0}, \
+            "fallback (B200_PROFILING.md)"
 
 
 # ------------------------------------------------------------------------- main arm
@@ -272,66 +340,86 @@ def main():
         e2e_res = e2e(runtimes, torch, stream, steps[args.warmup:], R, cfg, flush)
 
     result = None
+    extras = {}
     if rank == 0:
-        result = {"metric": METRIC, "value": value, "unit": "req/s", "n_gpus": world, "steps": args.steps,
-                  "warmup": args.warmup, "ms_per_step": t_max / args.steps, "higher_is_better": True,
+        rnd = lambda x, k=4: None if x is None else float(f"{x:.{k}g}")  # noqa: E731
+        result = {"metric": METRIC, "value": rnd(value, 6), "unit": "req/s", "n_gpus": world, "steps": args.steps,
+                  "warmup": args.warmup, "ms_per_step": rnd(t_max / args.steps, 5), "higher_is_better": True,
                   "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
-                  "config": {"workload": "bert-base polymorphed runtimes L{64,128,256,512}, batch buckets <=32 "
-                                         "(BASELINE configs[1])",
-                             "requests_per_step_per_gpu": R, "lengths": "LogNormal(ln21,0.6)<=125 x512/125",
-                             "weights": "random N(0,0.02) seed 0", "l2": "flushed (512 MB write) between steps",
-                             "parallelism": f"replicas x{world}"},
+                  "config": {"workload": WORKLOAD, "requests_per_step_per_gpu": R,
+                             "lengths": "LogNormal(ln21,0.6)<=125 x512/125", "weights": "random N(0,0.02) seed 0",
+                             "l2": "flushed (512 MB write) between steps", "parallelism": f"replicas x{world}"},
                   "latency_ms_per_bucket": {
-                      str(L): {"requests": len(lat[L]),
-                               "forward_mean": float(np.mean(lat[L])) if lat[L] else None,
-                               "forward_p99": float(np.percentile(lat[L], 99)) if lat[L] else None,
-                               "completion_mean": float(np.mean(done[L])) if done[L] else None,
-                               "completion_p99": float(np.percentile(done[L], 99)) if done[L] else None}
+                      str(L): {"n": len(lat[L]),
+                               "mean": rnd(np.mean(lat[L])) if lat[L] else None,
+                               "p99": rnd(np.percentile(lat[L], 99)) if lat[L] else None,
+                               "completion_mean": rnd(np.mean(done[L])) if done[L] else None,
+                               "completion_p99": rnd(np.percentile(done[L], 99)) if done[L] else None}
                       for L in RUNTIME_LS},
                   "gpu_launches": int(launches), "clocks": clocks}
         pad_tokens = sum(L * n for (_, fwd) in steps[args.warmup:] for (L, n, *_r) in fwd)
         real_tokens = sum(int(x.sum()) for (x, _) in steps[args.warmup:])
         static_flops = sum(metrics.forward_flops(cfg, n, L) for (_, fwd) in steps[args.warmup:] for (L, n, *_r) in fwd)
-        result["padding_efficiency"] = real_tokens / pad_tokens
-        result["static_tflops"] = static_flops / (total_ms / 1e3) / 1e12
-        result["useful_tflops"] = sum(metrics.useful_flops(cfg, x) for (x, _) in steps[args.warmup:]) / (total_ms / 1e3) / 1e12
+        result["padding_efficiency"] = rnd(real_tokens / pad_tokens)
+        result["static_tflops"] = rnd(static_flops / (total_ms / 1e3) / 1e12)
+        result["useful_tflops"] = rnd(sum(metrics.useful_flops(cfg, x) for (x, _) in steps[args.warmup:])
+                                      / (total_ms / 1e3) / 1e12)
 
     if rank == 0 and not args.no_extras:
-        result["roofline"] = roofline_dominant(arlo, torch, dev, stream, step_times)
-        result["gemm_tiles"] = {"note": "QKV, out-proj, FFN1, FFN2 tile codes per batch bucket, timed on the device at "
-                                        "runtime creation (BN single CTA, -BN CTA pair, 1000+BN skinny)",
-                                **{str(L): {str(n): rt.gemm_tiles(n) for n in (1, 8, 16, 32)} for L, rt in runtimes.items()}}
-        result["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
-        result["per_L_latency_ms_restricted"] = per_L_table(runtimes, torch, dev, stream, cfg, restricted=True)
-        pl = result["per_L_latency_ms"]
-        result["paper_context"] = {
+        roof, gemm_table = roofline_dominant(arlo, torch, dev, stream, runtimes[128], flush)
+        result["roofline"] = roof
+        extras["gemm_roofline_L128_b32"] = gemm_table
+        extras["gemm_tiles"] = {"note": "QKV, out-proj, FFN1, FFN2 tile codes per batch bucket, timed on the device "
+                                        "at runtime creation (BN single CTA, -BN CTA pair, 1000+BN skinny)",
+                                **{str(L): {str(n): rt.gemm_tiles(n) for n in (1, 8, 16, 32)}
+                                   for L, rt in runtimes.items()}}
+        extras["per_L_latency_ms"] = per_L_table(runtimes, torch, dev, stream, cfg)
+        extras["per_L_latency_ms_restricted"] = per_L_table(runtimes, torch, dev, stream, cfg, restricted=True)
+        pl = extras["per_L_latency_ms"]
+        result["per_L_b1_ms"] = {L: rnd(pl[L]["1"]["median"]) for L in pl}
+        extras["paper_context"] = {
             "note": "context only: RTX 3090, FP32 TensorRT static shape, batch 1 (BASELINE.md section 1)",
             "bert_base_L512_b1_ms": {"paper_rtx3090": 4.86, "this_b200_bf16": pl["512"]["1"]["median"],
                                      "source": "PAPER.md:L101 (Fig. 2a)"},
             "latency_ratio_L512_over_L64_b1": {"paper_rtx3090": 4.22,
                                                "this_b200_bf16": pl["512"]["1"]["median"] / pl["64"]["1"]["median"],
                                                "source": "PAPER.md:L95"}}
-        result["uniform_512"] = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
+        st512 = uniform_512(runtimes, torch, dev, stream, steps[args.warmup:], flush, R, cfg)
+        extras["uniform_512"] = st512
+        result["uniform_512_req_s"] = rnd(st512["value"], 5)
         result["e2e"] = e2e_res
-        result["bert_large"] = bert_large_per_L(arlo, torch, dev, stream, local_rank)
-        result["trace_replay"] = trace_replay(arlo, torch, runtimes, cfg, stream, result)
-        result["cluster_replay"] = cluster_replay(arlo, torch, W, runtimes, cfg, stream)
+        bl = bert_large_per_L(arlo, torch, dev, stream, local_rank, flush)
+        extras["bert_large"] = bl
+        result["bert_large_frac_of_burst"] = {f"L{L}_b{b}": rnd(bl["per_L"][str(L)][str(b)]["frac_of_peak"], 3)
+                                              for L in (256, 512) for b in (32, 64)}
+        if args.full:
+            extras["trace_replay"] = trace_replay(arlo, torch, runtimes, cfg, stream, result, pl)
+            extras["cluster_replay"] = cluster_replay(arlo, torch, W, runtimes, cfg, stream)
         if not args.no_cpu_baseline:
-            result["cpu_baseline"] = cpu_baseline()
+            cb = cpu_baseline(args.cpu_trace_requests)
+            extras["cpu_baseline"] = cb
+            result["cpu_baseline"] = {k: (rnd(v) if isinstance(v, float) else v) for k, v in cb.items()
+                                      if k in ("value", "unit", "cores", "kind", "sample", "cpu_model", "host_cpus",
+                                               "one_thread_value")}
+        result["extras_file"] = os.path.relpath(args.extras_out, ROOT)
+        extras["headline"] = result
+        os.makedirs(os.path.dirname(os.path.abspath(args.extras_out)), exist_ok=True)
+        with open(args.extras_out, "w") as f:
+            json.dump(extras, f, indent=1)
     if rank == 0:
-        print(json.dumps(result), flush=True)
+        print(json.dumps(result, separators=(",", ":")), flush=True)
     for rt in runtimes.values():
         rt.close()
     if world > 1:
         dist.destroy_process_group()
 
 
-def trace_replay(arlo, torch, runtimes, cfg, stream, result):
+def trace_replay(arlo, torch, runtimes, cfg, stream, result, per_L_ms):
     """Mean / p98 / p99 latency per length bucket under Poisson and MMPP arrivals at
     70% of the measured saturation throughput, requests dispatched by Algorithm 1
     (replay.py); SLO 150 ms for BERT-base."""
     from paper_conf_icpp_tanlyl024_b200 import replay
-    per_L = {int(L): {int(b): v["median"] for b, v in row.items()} for L, row in result["per_L_latency_ms"].items()}
+    per_L = {int(L): {int(b): v["median"] for b, v in row.items()} for L, row in per_L_ms.items()}
     rate = 0.7 * result["value"] / max(1, result["n_gpus"])
     out = {}
     for bursty in (False, True):
@@ -367,100 +455,111 @@ def cluster_replay(arlo, torch, W, runtimes, cfg, stream):
     return res
 
 
-def bert_large_per_L(arlo, torch, dev, stream, device_index):
+def bert_large_per_L(arlo, torch, dev, stream, device_index, flush, reps=20):
     """north_star target: per-L bf16 BERT-large forward at L >= 256 as a fraction of
     the B200 tensor peak (BASELINE configs[2]: L in {128,256,512}, batch up to 64).
-    One forward per (L, b) replayed back to back from the runtime's CUDA graph."""
+    Per (L, b): 3 warm-up forwards, then `reps` timed forwards (CUDA events around each,
+    L2 flushed before each, outside the events), median reported, with the SM clocks
+    sampled by nvidia-smi during the row."""
     cfg = wl.BERT_LARGE
     W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg, seed=wl.SEED_WEIGHTS), arlo.BF16, dev),
                      arlo.BF16, device_index)
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
-    peak = peaks.get("bf16_tflops", 1590.0)
-    peak_sus = peaks.get("bf16_tflops_sustained", 1400.0)
+    peaks, src = load_peaks()
+    peak, peak_sus = peaks["bf16_tflops"], peaks["bf16_tflops_sustained"]
     out = {}
     for L in (128, 256, 512):
         rt = arlo.Runtime(W, L, 64)
         rt.set_stream(stream)
         row = {}
-        for b in (1, 4, 16, 32, 64):
+        for b in (1, 16, 32, 64):
             lens = np.full(b, L, np.int32)
             ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
             ld = torch.from_numpy(lens).to(dev)
             o = torch.empty((b, cfg.num_labels), device=dev)
             for _ in range(3):
                 rt.enqueue(b, ids, ld, o)
-            reps = 5
-            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-            a.record(stream)
-            for _ in range(reps):
-                rt.enqueue(b, ids, ld, o)
-            e.record(stream)
             torch.cuda.synchronize()
-            ms = a.elapsed_time(e) / reps
+            sampler = ClockSampler(device_index)
+            sampler.start()
+            ev = []
+            for _ in range(reps):
+                flush.zero_()
+                a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                a.record(stream)
+                rt.enqueue(b, ids, ld, o)
+                e.record(stream)
+                ev.append((a, e))
+            torch.cuda.synchronize()
+            clk = sampler.stop()
+            ts = sorted(a.elapsed_time(e) for a, e in ev)
+            ms = float(np.median(ts))
             tf = metrics.forward_flops(cfg, b, L) / (ms / 1e3) / 1e12
-            row[str(b)] = {"ms": ms, "static_tflops": tf, "frac_of_peak": tf / peak,
-                           "frac_of_sustained_peak": tf / peak_sus}
+            row[str(b)] = {"ms": ms, "min_ms": ts[0], "max_ms": ts[-1], "static_tflops": tf,
+                           "frac_of_peak": tf / peak, "frac_of_sustained_peak": tf / peak_sus,
+                           "sm_mhz": clk.get("sm_mhz"), "clock_reasons": clk.get("reasons")}
         out[str(L)] = row
         rt.close()
     W.close()
-    return {"per_L": out, "peak_tflops": peak, "peak_sustained_tflops": peak_sus,
-            "note": "static FLOPs = layers*(24bLH^2+4bL^2H)+b(2H^2+2HC); back-to-back graph replays"}
+    return {"per_L": out, "peak_tflops": peak, "peak_sustained_tflops": peak_sus, "peak_source": src, "reps": reps,
+            "note": "static FLOPs = layers*(24bLH^2+4bL^2H)+b(2H^2+2HC); median of per-forward CUDA-event times, "
+                    "L2 flushed before each forward"}
 
 
-def roofline_dominant(arlo, torch, dev, stream, step_times):
-    """Dominant kernel: the FFN1 tcgen05 GEMM (+bias+GELU) of the L=128, b=32 runtime
-    (M=4096, N=3072, K=768), the single largest GEMM share of a step, in the tile
-    configuration the runtime graphs use.  Timed live on the launching stream:
-    REPS launches captured in one CUDA graph (as in the runtime graphs, so no host
-    launch gaps), CUDA events around each replay, averaged per launch."""
-    M, N, K = 4096, 3072, 768
-    REPS = 20
-    A = torch.randn(M, K, device=dev).to(torch.bfloat16)
-    Wt = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
-    b = torch.zeros(N, device=dev)
-    out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-    for _ in range(3):
-        arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
-    torch.cuda.synchronize()
-    g = torch.cuda.CUDAGraph()
-    with torch.cuda.graph(g, stream=stream):
-        for _ in range(REPS):
-            arlo.op_gemm(arlo.BF16, A, Wt, b, out, epi=arlo.EPI_BIAS_GELU, stream=stream)
-    g.replay()
-    torch.cuda.synchronize()
-    ts = []
-    for _ in range(10):
-        a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        a.record(stream)
-        g.replay()
-        e.record(stream)
+def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
+    """Roofline of the dominant kernel.  The four GEMMs of the L=128, b=32 runtime (the bucket
+    that serves the most requests, 43 %; M = 4096) are timed in the tile configuration its
+    CUDA graph actually replays (rt.gemm_tiles(32), chosen by timing at runtime creation),
+    each launch bracketed by CUDA events on the launching stream with L2 flushed before it
+    (outside the events), `reps` launches averaged.  The dominant kernel is the GEMM with the
+    largest time; achieved = 2MNK / its mean launch time."""
+    H, F = 768, 3072
+    M = 128 * 32
+    codes = rt128.gemm_tiles(32)
+    shapes = {"qkv": (M, 3 * H, H, arlo.EPI_BIAS, codes[0]), "out_proj": (M, H, H, arlo.EPI_BIAS_RESIDUAL, codes[1]),
+              "ffn1": (M, F, H, arlo.EPI_BIAS_GELU, codes[2]), "ffn2": (M, H, F, arlo.EPI_BIAS_RESIDUAL, codes[3])}
+    peaks, src = load_peaks()
+    peak = peaks["bf16_tflops"]
+    table = {}
+    g = torch.Generator(device=dev).manual_seed(0)
+    for name, (m, n, k, epi, code) in shapes.items():
+        A = torch.randn(m, k, device=dev, generator=g).to(torch.bfloat16)
+        Wt = (0.02 * torch.randn(n, k, device=dev, generator=g)).to(torch.bfloat16)
+        bias = torch.zeros(n, device=dev)
+        res = torch.randn(m, n, device=dev, generator=g).to(torch.bfloat16) if epi == arlo.EPI_BIAS_RESIDUAL else None
+        out = torch.empty(m, n, device=dev, dtype=torch.bfloat16)
+        for _ in range(3):
+            arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
+        ev = []
+        for _ in range(reps):
+            flush.zero_()
+            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
+            e.record(stream)
+            ev.append((a, e))
         torch.cuda.synchronize()
-        ts.append(a.elapsed_time(e) / REPS)
-    t = float(np.mean(ts)) / 1e3
-    choice = arlo.gemm_tile_choice(M, N, K)
-    flops = metrics.gemm_flops(M, N, K)
-    peaks = {}
-    try:
-        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
-    except Exception:
-        pass
-    peak = peaks.get("bf16_tflops", 1590.0)
+        t_us = 1e3 * float(np.mean([a.elapsed_time(e) for a, e in ev]))
+        fl = metrics.gemm_flops(m, n, k)
+        table[name] = {"M": m, "N": n, "K": k, "tile_code": code, "launch_us": t_us,
+                       "tflops": fl / (t_us / 1e6) / 1e12, "frac": fl / (t_us / 1e6) / 1e12 / peak}
+    dom = max(table, key=lambda k: table[k]["launch_us"])
+    d = table[dom]
     traffic = None
     try:
-        traffic = json.load(open(os.path.join(ROOT, "profiles", "traffic.json"))).get("ffn1_gemm_dram_bytes")
+        tj = json.load(open(os.path.join(ROOT, "profiles", "traffic.json")))
+        key = f"{dom}_L128_b32_tile{d['tile_code']}_dram_bytes"
+        traffic = tj.get(key)
     except Exception:
         pass
-    achieved = flops / t / 1e12
-    kname = (f"gemm_tc_pair_kernel<{-choice}, GELU>" if choice < 0 else f"gemm_tc_kernel<{choice}, GELU>")
-    return {"kernel": kname + " (FFN1, M=4096 N=3072 K=768)", "bound": "tensor",
-            "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
-            "traffic": traffic, "peak_source": "MEASURED_PEAKS.json bf16_tflops (burst)" if peaks else
-            "fallback 1590 TFLOP/s (B200_PROFILING.md)", "launch_us": t * 1e6,
-            "algorithmic_flops_per_launch": flops}
+    code = d["tile_code"]
+    kname = (f"gemm_skinny_kernel<{code - 1000}>" if code > 1000 else
+             f"gemm_tc_pair_kernel<{-code}>" if code < 0 else f"gemm_tc_kernel<{code}>")
+    roof = {"kernel": f"{kname} ({dom}, M={d['M']} N={d['N']} K={d['K']}, L=128 b=32 graph tile)", "bound": "tensor",
+            "achieved": round(d["tflops"], 1), "peak": peak, "unit": "TFLOP/s", "frac": round(d["frac"], 4),
+            "traffic": traffic, "peak_source": src + " bf16_tflops (burst)", "launch_us": round(d["launch_us"], 2),
+            "algorithmic_flops_per_launch": metrics.gemm_flops(d["M"], d["N"], d["K"]),
+            "l2": "flushed before each launch"}
+    return roof, table
 
 
 def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False):

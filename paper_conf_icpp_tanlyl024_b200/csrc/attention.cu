@@ -116,7 +116,9 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   pdl_launch_dependents();
   const int h = blockIdx.y, b = blockIdx.z;
   const int H = heads * D;
-  const int len = __ldg(lengths + b);
+  // lengths come from device memory unvalidated (arlo_enqueue, arlo_op_attention): clamp to
+  // [0, L] so a bad length can neither index barriers past kMaxKT nor read the next sequence
+  const int len = min(max(__ldg(lengths + b), 0), L);
   const int q0 = blockIdx.x * (NQ * AQ);
   const int row_base = b * L;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
@@ -548,7 +550,7 @@ __global__ void __launch_bounds__(128) attn_f32_kernel(int B, int L, int heads, 
   if (gw >= B * L * heads) return;
   const int h = gw % heads, row = gw / heads;
   const int b = row / L, t = row - b * L;
-  const int len = __ldg(lengths + b);
+  const int len = min(max(__ldg(lengths + b), 0), L);
   float* orow = o + (size_t)row * H + h * D;
   if ((t / AQ) * AQ >= len) {  // same zero rule as the bf16 path (128-row q-tiles)
     orow[2 * lane] = 0.f;
@@ -585,16 +587,15 @@ int set_attn_trace(unsigned long long* buf) {
 template <int NQ, int MAXKT, int NS>
 cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
   using Cfg = AttnCfg<NQ, MAXKT, NS>;
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, false>,
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = once_per_device(attr_done, [] {
+    cudaError_t r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, false>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
-    if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    if (r == cudaSuccess)
+      r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                Cfg::kSmem);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
+    return r; });
+  if (e != cudaSuccess) return e;
   dim3 grid((p.q_rows + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
   if (g_attn_trace_on)
     return launch_k(attn_tc_kernel<NQ, MAXKT, NS, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,

@@ -5,6 +5,7 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <atomic>
 #include <utility>
 
 namespace arlo {
@@ -151,6 +152,22 @@ __device__ __forceinline__ uint4 ld_dep_v4(const void* p) {
 }
 
 bool pdl_enabled();  // false when ARLO_NO_PDL is set in the environment (A/B measurements)
+
+// Kernel attributes (the >48 KB dynamic shared memory opt-in, ...) belong to the CURRENT
+// device's context, and runtimes of one process may live on several devices and be built
+// from several host threads.  `done` keeps one bit per device index (a static per kernel
+// instantiation); setting an attribute twice is harmless, so a race only repeats the call.
+template <typename SetFn>
+inline cudaError_t once_per_device(std::atomic<uint64_t>& done, SetFn set) {
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  const uint64_t bit = 1ull << (dev & 63);
+  if (done.load(std::memory_order_acquire) & bit) return cudaSuccess;
+  e = set();
+  if (e == cudaSuccess) done.fetch_or(bit, std::memory_order_acq_rel);
+  return e;
+}
 
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,

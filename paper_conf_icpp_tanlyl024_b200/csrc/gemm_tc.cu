@@ -9,15 +9,18 @@
 //
 // Blackwell design (not a port of anything in the paper, whose runtimes are
 // TensorRT engines for sm_86):
-//  * persistent CTAs (grid = min(tiles, #SMs)), static round-robin tile order;
-//  * warp 0 = TMA producer: 128x64 A tile + BNx64 W tile per stage, 128-byte
+//  * persistent CTAs (grid = min(tiles, #SMs)), static round-robin tile order
+//    (N fastest), single-CTA 128 x BN tiles or CTA-pair (cta_group::2) 256 x BN tiles;
+//  * warps 0..EW-1 = epilogue (EW = 8, or 12 for GELU at M <= 8192; Roles<EW>):
+//    warp w reads TMEM lane quarter w % 4 and the 32-column chunks w/4, w/4 + EW/4, ...;
+//    tcgen05.ld, bias / GELU / residual on paired fp32 instructions, RNE to bf16,
+//    st.shared into a 64B-swizzled staging tile, TMA bulk tensor store.  Two TMEM
+//    accumulator stages let the epilogue of tile i overlap the main loop of tile i+1;
+//  * warp EW = TMA producer: 128x64 A tile + BNx64 W tile per stage, 128-byte
 //    swizzle, STAGES-deep smem ring guarded by full/empty mbarriers;
-//  * warp 1 = MMA issuer: one thread issues tcgen05.mma.cta_group::1.kind::f16
-//    (M=128, N=BN, K=16) into a TMEM fp32 accumulator; tcgen05.commit frees
-//    smem stages and signals the epilogue;
-//  * warps 2-5 = epilogue: tcgen05.ld 32 lanes x 32 columns, bias / GELU /
-//    residual in fp32, RNE to bf16, 16-byte stores.  Two TMEM accumulator
-//    buffers let the epilogue of tile i overlap the main loop of tile i+1.
+//  * warp EW+1 = MMA issuer: the converged warp runs the loop, one elected lane issues
+//    tcgen05.mma.kind::f16 (M=128 or 256, N=BN, K=16) into the TMEM fp32 accumulator;
+//    tcgen05.commit frees smem stages and signals the epilogue.
 // Row results never depend on M, the tile width or the grid: the K loop of
 // every output element is the same sequence of K=16 MMAs (cross-L bitwise
 // invariance, SURVEY.md §7 "Cross-L argmax agreement").
@@ -1023,17 +1026,17 @@ typedef CUresult (*EncodeTiledFn)(CUtensorMap*, CUtensorMapDataType, cuuint32_t,
                                   const cuuint32_t*, CUtensorMapInterleave, CUtensorMapSwizzle,
                                   CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
 
+// Resolved once, thread-safely (a function-local static is initialised exactly once even when
+// runtimes are created from several host threads at the same time).
 EncodeTiledFn get_encode_fn() {
-  static EncodeTiledFn fn = nullptr;
-  static bool tried = false;
-  if (!tried) {
-    tried = true;
+  static const EncodeTiledFn fn = []() -> EncodeTiledFn {
     void* p = nullptr;
     cudaDriverEntryPointQueryResult q;
     if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
         q == cudaDriverEntryPointSuccess)
-      fn = reinterpret_cast<EncodeTiledFn>(p);
-  }
+      return reinterpret_cast<EncodeTiledFn>(p);
+    return nullptr;
+  }();
   return fn;
 }
 
@@ -1041,12 +1044,10 @@ template <int BN, int EPI, bool PAIR, int EW>
 cudaError_t launch_cfg_ew(const TcGemmPlan& p, cudaStream_t s) {
   using C = TcCfg<BN, PAIR, 0, EW>;
   auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI, EW> : gemm_tc_kernel<BN, EPI, EW>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = once_per_device(attr_done, [&] {
+    return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
+  if (e != cudaSuccess) return e;
   return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K,
                   p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out);
 }
@@ -1073,12 +1074,10 @@ template <int BN, int EPI>
 cudaError_t launch_skinny_cfg(const TcGemmPlan& p, cudaStream_t s) {
   using C = SkCfg<BN>;
   auto kern = gemm_skinny_kernel<BN, EPI>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = once_per_device(attr_done, [&] {
+    return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
+  if (e != cudaSuccess) return e;
   return launch_k(kern, dim3(p.N / BN, (p.M + BM - 1) / BM), dim3(kSkThreads), C::SMEM, s, p.tmA, p.tmB,
                   (bf16*)p.out, p.M, p.N, p.K, p.a_rows, p.bias, (const bf16*)p.resid, p.ldr);
 }
@@ -1100,12 +1099,10 @@ int set_gemm_trace(unsigned long long* buf) {
 }
 
 int num_sms() {
-  static int n = 0;
-  if (n == 0) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0) n = 148;
-  }
+  int dev = 0, n = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess ||
+      cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess || n <= 0)
+    n = 148;
   return n;
 }
 
@@ -1218,13 +1215,12 @@ cudaError_t launch_ln(const TcGemmPlan& p, cudaStream_t s) {
   constexpr int SMEM = C::SMEM;
   static_assert(SMEM <= 232448, "fused LN smem");
   auto kern = gemm_ln_kernel<BN>;
-  static bool attr_set = false;
-  if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
-    if (e == cudaSuccess) e = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
-    if (e != cudaSuccess) return e;
-    attr_set = true;
-  }
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = once_per_device(attr_done, [&] {
+    cudaError_t r = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, SMEM);
+    if (r == cudaSuccess) r = cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    return r; });
+  if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(p.grid);
   cfg.blockDim = dim3(kThreads);

@@ -152,18 +152,17 @@ template <typename T, int MAXV>
 cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
                      const float* b_c, float* pooled, float* logits, cudaStream_t s) {
   const size_t smem = (size_t)kRows * H * sizeof(T);
-  static bool attr = false;
-  if (!attr) {
-    cudaError_t e = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  static std::atomic<uint64_t> attr_done{0};
+  cudaError_t e = once_per_device(attr_done, [] {
+    cudaError_t r = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          kRows * 2048 * 4);
-    if (e != cudaSuccess) return e;
-    e = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributePreferredSharedMemoryCarveout,
-                             cudaSharedmemCarveoutMaxShared);
-    if (e != cudaSuccess) return e;
-    attr = true;
-  }
+    if (r == cudaSuccess)
+      r = cudaFuncSetAttribute(pooler_kernel<T, MAXV>, cudaFuncAttributePreferredSharedMemoryCarveout,
+                               cudaSharedmemCarveoutMaxShared);
+    return r; });
+  if (e != cudaSuccess) return e;
   dim3 grid((H + kFeat - 1) / kFeat, (B + kRows - 1) / kRows);
-  cudaError_t e = launch_k(pooler_kernel<T, MAXV>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p,
+  e = launch_k(pooler_kernel<T, MAXV>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p,
                            b_p, pooled);
   if (e != cudaSuccess) return e;
   return launch_k(classifier_kernel<T, MAXV>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c,

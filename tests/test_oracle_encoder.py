@@ -247,3 +247,16 @@ def test_forward_batch_stops_at_empty_slot():
     ids = wl.sample_token_ids(cfg, lengths, 8, seed=1)
     out = orc.forward_batch(cfg, w, ids, lengths)
     assert out.shape == (2, 2)
+
+
+def test_label_tie_rule_and_argmax():
+    """orc.label: argmax over the classes, the lowest index winning exact ties (reading S11)."""
+    logits = np.array([[0.25, 0.25], [-1.0, 2.0], [3.0, -3.0], [0.0, 0.0]])
+    np.testing.assert_array_equal(orc.label(logits), [0, 1, 0, 0])
+    cfg = wl.TINY
+    w = wl.make_weights(cfg, seed=3)
+    lengths = np.array([7, 12, 3], np.int32)
+    ids = wl.sample_token_ids(cfg, lengths, 16, seed=8)
+    out = orc.forward_batch(cfg, w, ids, lengths)
+    for i in range(3):
+        assert orc.label(out[i]) == (0 if out[i, 0] >= out[i, 1] else 1)
