@@ -107,6 +107,25 @@ typedef struct arlo_runtime arlo_runtime;
  * Errors: EINVAL, ENOMEM, ECUDA, ENODEV.
  */
 int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out);
+
+/*
+ * Runtime families.  The paper's runtimes run at batch 1 (§5); at M = L
+ * rows a projection streams its whole weight matrix for 2L flops per element, so the
+ * LATENCY family runs every GEMM as a split-K weight-streaming kernel: a cluster of S
+ * CTAs per column tile, S = a function of the weight shape (N, K) only, partial sums
+ * added in a fixed order over distributed shared memory.  The THROUGHPUT family runs
+ * the tile kernels (each output element's K chain in one accumulator).  Within a family
+ * a request's logits are bitwise equal on every runtime L >= its length and in every
+ * batch bucket; across families they agree to bf16 rounding (both within 2e-2 of the
+ * oracle).  DEFAULT = THROUGHPUT: on B200 a batch-1 forward is bound by its chain of
+ * ~87 dependent kernels (~4.5 us each), not by the GEMMs, and the latency family measured
+ * no faster.  fp32 check mode ignores the family (SIMT GEMMs).
+ */
+enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHPUT = 2 };
+int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_weights* w, int32_t family,
+                           arlo_runtime** out);
+/* ARLO_RUNTIME_LATENCY or ARLO_RUNTIME_THROUGHPUT (the family the runtime was built as). */
+int32_t arlo_runtime_family(const arlo_runtime* rt);
 void arlo_runtime_destroy(arlo_runtime* rt);
 /* Launch stream for every later call (a cudaStream_t; NULL = legacy default stream). */
 int arlo_runtime_set_stream(arlo_runtime* rt, void* cuda_stream);

@@ -28,11 +28,13 @@ OK, EINVAL, ETOOLONG, ENOMEM, ECUDA, EINFEASIBLE, ENOCAND, ENODEV = 0, -1, -2, -
 BF16, FP32 = 0, 1
 DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
+RUNTIME_DEFAULT, RUNTIME_LATENCY, RUNTIME_THROUGHPUT = 0, 1, 2
+SKINNY_CODE, SPLITK_CODE = 1000, 2000  # tile codes: kSkinnyCode + BN, kSplitKCode + BN
 
 EXPORTED = [
     "arlo_replace_plan", "arlo_runtime_gemm_tiles",
     "arlo_last_error", "arlo_version", "arlo_weights_count", "arlo_weights_create", "arlo_weights_destroy",
-    "arlo_runtime_create", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
+    "arlo_runtime_create", "arlo_runtime_create_ex", "arlo_runtime_family", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_sched_set_policy", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
     "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
@@ -63,6 +65,8 @@ _sig("arlo_weights_count", _i32, _P(ModelConfigC))
 _sig("arlo_weights_create", C.c_int, _i32, _P(ModelConfigC), _P(_vp), _i32, _P(_vp))
 _sig("arlo_weights_destroy", None, _vp)
 _sig("arlo_runtime_create", C.c_int, _i32, _i32, _vp, _P(_vp))
+_sig("arlo_runtime_create_ex", C.c_int, _i32, _i32, _vp, _i32, _P(_vp))
+_sig("arlo_runtime_family", _i32, _vp)
 _sig("arlo_runtime_destroy", None, _vp)
 _sig("arlo_runtime_set_stream", C.c_int, _vp, _vp)
 _sig("arlo_runtime_length", _i32, _vp)
@@ -168,11 +172,16 @@ class Weights:
 class Runtime:
     """arlo_runtime: one statically shaped per-length runtime (L, max_batch)."""
 
-    def __init__(self, weights: Weights, L: int, max_batch: int):
+    def __init__(self, weights: Weights, L: int, max_batch: int, family: int = RUNTIME_DEFAULT):
         self.weights, self.L, self.max_batch = weights, L, max_batch
         h = _vp()
-        check(lib.arlo_runtime_create(L, max_batch, weights.handle, C.byref(h)))
+        check(lib.arlo_runtime_create_ex(L, max_batch, weights.handle, family, C.byref(h)))
         self.handle = h
+
+    @property
+    def family(self) -> int:
+        """RUNTIME_LATENCY (split-K weight streaming) or RUNTIME_THROUGHPUT (tile kernels)."""
+        return check(lib.arlo_runtime_family(self.handle))
 
     def set_stream(self, stream):
         check(lib.arlo_runtime_set_stream(self.handle, _stream_ptr(stream)))

@@ -151,6 +151,12 @@ __device__ __forceinline__ uint4 ld_dep_v4(const void* p) {
   return v;
 }
 
+__device__ __forceinline__ uint2 ld_dep_v2(const void* p) {
+  uint2 v;
+  asm volatile("ld.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
+  return v;
+}
+
 bool pdl_enabled();  // false when ARLO_NO_PDL is set in the environment (A/B measurements)
 
 // Kernel attributes (the >48 KB dynamic shared memory opt-in, ...) belong to the CURRENT

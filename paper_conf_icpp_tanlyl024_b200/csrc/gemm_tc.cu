@@ -27,6 +27,7 @@
 #include <cuda.h>
 
 #include "common.cuh"
+#include "epilogue.cuh"
 #include "kernels.h"
 #include "ptx.cuh"
 
@@ -132,41 +133,6 @@ constexpr int CW = 32;  // chunk width: TMEM load / staging tile / TMA box (colu
 #ifndef ARLO_EPI_DIRECT
 #define ARLO_EPI_DIRECT 0  // 1: store rows straight from registers instead of smem staging + TMA (A/B)
 #endif
-
-// Epilogue arithmetic of 4 consecutive columns of one row: acc + bias, then GELU or
-// + residual (two bf16x2 words ua, ub), RNE-packed to two bf16x2 words.  Paired fp32
-// instructions (FADD2 / FFMA2); shared by every GEMM kernel so the result of an element
-// does not depend on the tile shape that produced it.
-template <int EPI>
-__device__ __forceinline__ void epi_pack4(const uint32_t* r, float4 b4, uint32_t ua, uint32_t ub, uint32_t& p0,
-                                          uint32_t& p1) {
-#if defined(ARLO_EPI_SCALAR)  // A/B only: the previous scalar epilogue arithmetic
-  float v0 = __uint_as_float(r[0]) + b4.x, v1 = __uint_as_float(r[1]) + b4.y;
-  float v2 = __uint_as_float(r[2]) + b4.z, v3 = __uint_as_float(r[3]) + b4.w;
-  if (EPI == EPI_BIAS_GELU) {
-    v0 = gelu_erf_fast(v0); v1 = gelu_erf_fast(v1); v2 = gelu_erf_fast(v2); v3 = gelu_erf_fast(v3);
-  }
-  if (EPI == EPI_BIAS_RESID) {
-    const float2 fa = unpack_bf16x2(ua), fb = unpack_bf16x2(ub);
-    v0 += fa.x; v1 += fa.y; v2 += fb.x; v3 += fb.y;
-  }
-  p0 = pack_bf16x2(v0, v1);
-  p1 = pack_bf16x2(v2, v3);
-  return;
-#endif
-  float2 x0 = __fadd2_rn(make_float2(__uint_as_float(r[0]), __uint_as_float(r[1])), make_float2(b4.x, b4.y));
-  float2 x1 = __fadd2_rn(make_float2(__uint_as_float(r[2]), __uint_as_float(r[3])), make_float2(b4.z, b4.w));
-  if (EPI == EPI_BIAS_GELU) {
-    x0 = gelu2_erf_fast(x0);
-    x1 = gelu2_erf_fast(x1);
-  }
-  if (EPI == EPI_BIAS_RESID) {
-    x0 = __fadd2_rn(x0, unpack_bf16x2(ua));
-    x1 = __fadd2_rn(x1, unpack_bf16x2(ub));
-  }
-  p0 = pack_bf16x2(x0.x, x0.y);
-  p1 = pack_bf16x2(x1.x, x1.y);
-}
 
 // Residual of this warp's first chunk of a tile (row row0 + lane, columns n0 + 32 cg ...): the
 // residual never depends on the MMA, so the epilogue warps load it BEFORE waiting for the
@@ -625,7 +591,11 @@ struct SkCfg {
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_BYTES = BN * BK * 2;
   static constexpr int STAGE = A_BYTES + B_BYTES;
-  static constexpr int STAGES = (kSmemBudget - 1024) / STAGE > 12 ? 12 : (kSmemBudget - 1024) / STAGE;
+#ifndef ARLO_SKINNY_MAX_STAGES
+#define ARLO_SKINNY_MAX_STAGES 12
+#endif
+  static constexpr int STAGES = (kSmemBudget - 1024) / STAGE > ARLO_SKINNY_MAX_STAGES ? ARLO_SKINNY_MAX_STAGES
+                                                                                      : (kSmemBudget - 1024) / STAGE;
   static constexpr int SMEM = 1024 + STAGES * STAGE + 8 * (2 * STAGES + 1) + 16;
   static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;
   static_assert(SMEM <= 232448, "skinny smem");
@@ -1176,11 +1146,13 @@ bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void*
 bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int lda, const void* W,
                           const float* bias, const void* resid, int ldr, void* out, int epi, int force_bn) {
   if (M <= 0 || N % 64 || K % 64 || K <= 0 || lda < K || lda % 8 || ldr < N || ldr % 8) return false;
+  if (force_bn > kSplitKCode)
+    return tc_plan_gemm_splitk(p, M, N, K, A, lda, W, bias, resid, ldr, out, epi, force_bn - kSplitKCode);
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
   if (choice > kSkinnyCode) {
     const int bn = choice - kSkinnyCode;
     if ((bn != 16 && bn != 32 && bn != 64) || N % bn) return false;
-    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->epi = epi; p->ln = false; p->ew = 4;
+    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->splitk = false; p->epi = epi; p->ln = false; p->ew = 4;
     p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
     p->a_rows = M < BM ? ((M + 7) & ~7) : BM;
     p->grid = (N / bn) * ((M + BM - 1) / BM);
@@ -1193,7 +1165,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   if (bn != 64 && bn != 96 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn < 128) return false;
   if (N % bn) return false;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->epi = epi; p->ln = false;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->splitk = false; p->epi = epi; p->ln = false;
   p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
   const int tile_m = pair ? 2 * BM : BM;
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
@@ -1249,7 +1221,7 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   if (N == 128 && (128 / kEpiGroups) % 32 == 0 && 128 % kEpiGroups == 0) bn = 128;
   if (!bn) return false;
   const int nt = N / bn;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->splitk = false; p->epi = EPI_BIAS_RESID; p->ln = true;
   p->ew = kEpiWarps;
   p->bias = bias; p->resid = resid; p->ldr = N; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
   const int num_m = (M + BM - 1) / BM;
@@ -1262,6 +1234,7 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
 }
 
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s) {
+  if (p.splitk) return splitk_launch(p, s);
   if (p.skinny) {
     switch (p.BN) {
       case 16: return launch_skinny_bn<16>(p, s);

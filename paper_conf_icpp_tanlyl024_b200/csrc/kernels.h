@@ -36,7 +36,12 @@ struct TcGemmPlan {
   int ew;       // epilogue warps of the persistent kernels (8, or 12 for GELU at M <= 8192)
   bool pair;    // CTA-pair (cta_group::2) kernel, 256-row tiles
   bool skinny;  // small-M kernel: one CTA per 128 x BN tile (BN 16/32/64), direct stores
-  int a_rows;   // skinny: A box rows (min(128, M rounded up to 8))
+  int a_rows;   // skinny / split-K: A box rows (min(128, M rounded up to 8))
+  // split-K weight-streaming kernel (latency runtimes): a cluster of `splits` CTAs per
+  // (n-tile, 128-row block), CTA s accumulates K range [s*kc, (s+1)*kc); the partials are
+  // summed in the fixed order s = 0, 1, ... over distributed shared memory
+  bool splitk;
+  int splits, kc, stages, a_stage, smem;
   bool ln;    // fused residual + LayerNorm epilogue over full rows (cluster of N/BN CTAs)
   const float* gamma;
   const float* beta;
@@ -55,11 +60,22 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
 cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s);
 // Tile choice codes: BN (single CTA), -BN (CTA pair), kSkinnyCode + BN (skinny kernel).
 constexpr int kSkinnyCode = 1000;
+constexpr int kSplitKCode = 2000;  // kSplitKCode + BN: split-K kernel (splitk_factor(N, K) splits)
 int tc_choose_bn(int M, int N, int K);
 // out = LN(A W^T + bias + resid; gamma, beta, eps), N = hidden size (128 / 768 / 1024 ...).
 // `out` may alias `resid` (each tile reads its residual before storing the same region).
 bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W, const float* bias,
                      const void* resid, const float* gamma, const float* beta, float eps, void* out);
+
+// Split-K plan (the weight-streaming GEMM of latency runtimes, M = b*L small).  The split
+// factor is splitk_factor(N, K): a function of the weight shape only, so every runtime of
+// the latency family reduces each output element in the same order (cross-L bitwise).
+// bn = 0 lets splitk_bn(M, N, S) choose the tile width (any width gives the same bits).
+int splitk_factor(int N, int K);
+cudaError_t splitk_launch(const TcGemmPlan& p, cudaStream_t s);  // (tc_launch_gemm dispatches here)
+int splitk_bn(int M, int N, int S);
+bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int lda, const void* W,
+                         const float* bias, const void* resid, int ldr, void* out, int epi, int bn = 0);
 
 cudaError_t launch_gemm_simt(DType dt, int M, int N, int K, const void* A, const void* W,
                              const float* bias, const void* resid, void* out, int epi,

@@ -281,6 +281,16 @@ __device__ __forceinline__ float ld_shared_cluster_f32(uint32_t cluster_addr) {
   return v;
 }
 
+// Load 4 consecutive fp32 from the shared memory of a CTA of the cluster (DSMEM; 16-byte aligned).
+__device__ __forceinline__ float4 ld_shared_cluster_v4(uint32_t cluster_addr) {
+  float4 v;
+  asm volatile("ld.shared::cluster.v4.f32 {%0, %1, %2, %3}, [%4];"
+               : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(cluster_addr)
+               : "memory");
+  return v;
+}
+
 // Arrive on an mbarrier of another CTA of the cluster with CTA-scope release (the CUTLASS
 // ClusterBarrier::arrive form): no fence.  Enough when the arrive only hands back a resource
 // whose last use is already complete (e.g. an accumulator whose tcgen05.ld's were waited on and

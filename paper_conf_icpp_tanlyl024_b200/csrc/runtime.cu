@@ -176,6 +176,9 @@ struct Bucket {
 
 struct arlo_runtime {
   int L = 0, max_batch = 0, device = 0;
+  // latency family (ARLO_RUNTIME_LATENCY): every GEMM is the split-K weight-streaming kernel
+  // (gemm_splitk.cu); the throughput family uses the tile kernels chosen per bucket
+  bool latency = false;
   const arlo_weights* w = nullptr;
   DType dt = DT_BF16;
   cudaStream_t own_stream = nullptr, stream = nullptr;
@@ -312,7 +315,49 @@ static int pick_tile(int M, int N, int K, cudaStream_t s, PlanFn plan) {
   return best;
 }
 
+// Latency family: the four GEMMs of every layer (and of the CLS-only last layer) as split-K
+// weight-streaming GEMMs; the split factor depends on (N, K) only (cross-L bitwise within
+// the family), the tile width on M.
+static int plan_bucket_latency(arlo_runtime* rt, Bucket& bk) {
+  const arlo_weights* w = rt->w;
+  const arlo_model_config& c = w->cfg;
+  const int b = bk.b, L = rt->L, M = b * L, H = c.hidden, F = c.ffn;
+  bk.plans.resize(c.layers);
+  bk.fused_ln = false;
+  for (int l = 0; l < c.layers; ++l) {
+    LayerPlans& p = bk.plans[l];
+    const bool ok =
+        tc_plan_gemm_splitk(&p.qkv, M, 3 * H, H, rt->X, H, w->lt(l, LW_QKV), (const float*)w->lt(l, LB_QKV), nullptr,
+                            3 * H, rt->QKV, EPI_BIAS) &&
+        tc_plan_gemm_splitk(&p.o, M, H, H, rt->O, H, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, H, rt->Y,
+                            EPI_BIAS_RESID) &&
+        tc_plan_gemm_splitk(&p.f1, M, F, H, rt->X, H, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, F,
+                            rt->F, EPI_BIAS_GELU) &&
+        tc_plan_gemm_splitk(&p.f2, M, H, F, rt->F, F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, H, rt->Y,
+                            EPI_BIAS_RESID);
+    if (!ok) return set_error(ARLO_ECUDA, "split-K plan: tensor-map encoding failed");
+  }
+  const LayerPlans& p0 = bk.plans[0];
+  bk.tiles[0] = kSplitKCode + p0.qkv.BN; bk.tiles[1] = kSplitKCode + p0.o.BN;
+  bk.tiles[2] = kSplitKCode + p0.f1.BN; bk.tiles[3] = kSplitKCode + p0.f2.BN;
+  bk.cls_prune = getenv("ARLO_NO_CLS_PRUNE") == nullptr;
+  if (bk.cls_prune) {
+    const int l = c.layers - 1;
+    const bool ok =
+        attn_plan(&bk.attn_cls, rt->dt, b, L, c.heads, rt->QKV, 1) &&
+        tc_plan_gemm_splitk(&bk.cls.o, b, H, H, rt->O, L * H, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X,
+                            L * H, rt->Y, EPI_BIAS_RESID) &&
+        tc_plan_gemm_splitk(&bk.cls.f1, b, F, H, rt->X, H, w->lt(l, LW_1), (const float*)w->lt(l, LB_1), nullptr, F,
+                            rt->F, EPI_BIAS_GELU) &&
+        tc_plan_gemm_splitk(&bk.cls.f2, b, H, F, rt->F, F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->X, H,
+                            rt->Y, EPI_BIAS_RESID);
+    if (!ok) return set_error(ARLO_ECUDA, "CLS-row split-K plan: tensor-map encoding failed");
+  }
+  return ARLO_OK;
+}
+
 static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
+  if (rt->latency) return plan_bucket_latency(rt, bk);
   const arlo_weights* w = rt->w;
   const arlo_model_config& c = w->cfg;
   const int M = bk.b * rt->L, H = c.hidden, F = c.ffn;
@@ -399,8 +444,19 @@ extern "C" int arlo_runtime_gemm_tiles(const arlo_runtime* rt, int32_t n, int32_
 }
 
 extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out) {
+  return arlo_runtime_create_ex(L, max_batch, w, ARLO_RUNTIME_DEFAULT, out);
+}
+
+extern "C" int32_t arlo_runtime_family(const arlo_runtime* rt) {
+  return rt ? (rt->latency ? ARLO_RUNTIME_LATENCY : ARLO_RUNTIME_THROUGHPUT) : ARLO_EINVAL;
+}
+
+extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_weights* w, int32_t family,
+                                      arlo_runtime** out) {
   clear_error();
   if (!w || !out) return set_error(ARLO_EINVAL, "arlo_runtime_create: null argument");
+  if (family != ARLO_RUNTIME_DEFAULT && family != ARLO_RUNTIME_LATENCY && family != ARLO_RUNTIME_THROUGHPUT)
+    return set_error(ARLO_EINVAL, "arlo_runtime_create_ex: unknown runtime family %d", family);
   const arlo_model_config& c = w->cfg;
   if (L < 16 || L % 16 || L > c.max_pos)
     return set_error(ARLO_EINVAL, "arlo_runtime_create: need 16 <= L <= max_pos (%d) and L %% 16 == 0, got %d", c.max_pos, L);
@@ -413,6 +469,10 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
   rt->w = w;
   rt->device = w->device;
   rt->dt = c.dtype == ARLO_BF16 ? DT_BF16 : DT_FP32;
+  // batch-1 runtimes (the paper's setting) stream weights with split-K GEMMs
+  // (DEFAULT = THROUGHPUT: measured on B200, the split-K family does not shorten a batch-1 forward;
+  // its 87 dependent kernels cost ~4.5 us each whatever the GEMM kernel)
+  rt->latency = rt->dt == DT_BF16 && family == ARLO_RUNTIME_LATENCY;
   auto fail = [&](int code) { destroy_runtime(rt); return code; };
   cudaError_t e = cudaStreamCreateWithFlags(&rt->own_stream, cudaStreamNonBlocking);
   if (e != cudaSuccess) return fail(cuda_fail(e, "cudaStreamCreate"));

@@ -162,6 +162,9 @@ def test_embedding_ln(arlo_lib, dtype):
     (64, 16, [63, 64]),
     (256, 4, [256, 200, 129, 1, 128]),
     (384, 2, [384, 257, 100]),
+    (192, 3, [192, 191, 129, 128, 1]),
+    (320, 2, [320, 257, 200, 0]),
+    (448, 2, [448, 385, 300, 64]),
 ])
 @pytest.mark.parametrize("dtype", [0, 1])
 def test_attention_masked(arlo_lib, L, heads, lengths, dtype):

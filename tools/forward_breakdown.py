@@ -1,8 +1,8 @@
 """Run forwards of one BERT-base (or BERT-large: 4th arg "large") runtime (for an ncu launch list / per-kernel breakdown).
 
-    python tools/forward_breakdown.py L b [reps] [base|large]
-    ncu --metrics gpu__time_duration.sum --cache-control none --clock-control none --csv \
-        --log-file out.csv python tools/forward_breakdown.py 128 32
+    python tools/forward_breakdown.py L b [reps] [base|large] [default|latency|throughput]
+    ncu --profile-from-start off --metrics gpu__time_duration.sum --cache-control none --clock-control none \
+        --csv --log-file out.csv python tools/forward_breakdown.py 128 32
     python tools/forward_breakdown.py --summarize out.csv
 """
 import collections
@@ -46,14 +46,19 @@ def main():
     reps = int(sys.argv[3]) if len(sys.argv) > 3 else 2
     cfg = wl.BERT_LARGE if len(sys.argv) > 4 and sys.argv[4] == "large" else wl.BERT_BASE
     W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg), arlo.BF16), arlo.BF16)
-    rt = arlo.Runtime(W, L, b)
+    fam = {"default": 0, "latency": 1, "throughput": 2}[sys.argv[5] if len(sys.argv) > 5 else "default"]
+    rt = arlo.Runtime(W, L, b, fam)
     lens = np.full(b, L, np.int32)
     ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L)).cuda()
     ld = torch.from_numpy(lens).cuda()
     out = torch.empty((b, cfg.num_labels), device="cuda")
+    rt.enqueue(b, ids, ld, out)  # warm-up, outside the profiled range
+    torch.cuda.synchronize()
+    torch.cuda.cudart().cudaProfilerStart()  # with `ncu --profile-from-start off`: only these forwards
     for _ in range(reps):
         rt.enqueue(b, ids, ld, out)
     torch.cuda.synchronize()
+    torch.cuda.cudart().cudaProfilerStop()
 
 
 if __name__ == "__main__":
