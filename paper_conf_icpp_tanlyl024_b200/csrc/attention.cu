@@ -29,6 +29,13 @@ constexpr int AQ = 128;      // queries per q-tile (TMEM lanes)
 constexpr int AK = 128;      // keys per K/V tile (TMA unit)
 constexpr int KC = 64;       // keys per softmax chunk (S MMA N)
 constexpr int kTileBytes = 128 * 128;         // 128 rows x 64 bf16 (128 B), SWIZZLE_128B
+// Softmax exponentials: of every 16-key piece, the last kPolyPairs key pairs are evaluated by
+// ex2_poly2 on the FMA pipe, the rest by MUFU ex2 (16/clk/SM, the softmax's binding unit at
+// head dim 64).  A function of the key position only: every runtime computes a key's p alike.
+#ifndef ARLO_EXP_POLY_PAIRS
+#define ARLO_EXP_POLY_PAIRS 0  // measured: 1-4 pairs no faster at L = 64..512 (the softmax is not MUFU-bound)
+#endif
+constexpr int kPolyPairs = ARLO_EXP_POLY_PAIRS;
 
 // Launch shape per runtime length: NQ q-tiles per CTA, up to MAXKT 128-key
 // K/V tiles (L <= 128 * MAXKT), NS S/P slots per q-tile.  NQ = 1 (L <= 128)
@@ -100,10 +107,20 @@ __device__ __forceinline__ void atrace(int slot) {
 // in by TMA once per CTA and are shared by both q-tiles.  Key chunks starting
 // at >= len are never loaded or multiplied; keys >= len inside the last chunk
 // get p = 0.
-template <int NQ_, int MAXKT_, int NS_, bool TRACE>
+//
+// PACK = 2 (runtimes with L = 64): one 128-row tile holds two consecutive sequences
+// (rows b*64 .. b*64+127 of the QKV buffer are sequences b and b+1), so a CTA serves
+// both instead of computing a 128-row tile of which only the first 64 rows are kept.
+// Chunk c (keys 64c .. 64c+63 of the tile) is sequence c's keys: the softmax warps of
+// lane quarters 2c, 2c+1 (rows of sequence c) treat chunk c as their first and only
+// chunk (exactly the arithmetic of an unpacked CTA with len <= 64) and write P = 0 for
+// the other chunk, so O_c = P_c V_c + 0 * V_other: bitwise the unpacked rows (the
+// cross-L contract), in half the CTAs (b = 32: 192 instead of 384, one wave).
+template <int NQ_, int MAXKT_, int NS_, bool TRACE, int PACK>
 __global__ void __launch_bounds__(AttnCfg<NQ_, MAXKT_, NS_>::kThreads, AttnCfg<NQ_, MAXKT_, NS_>::kMinBlocks)
-attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const int32_t* __restrict__ lengths,
+attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int B, int L, int heads, const int32_t* __restrict__ lengths,
                bf16* __restrict__ o) {
+  static_assert(PACK == 1 || (PACK == 2 && NQ_ == 1 && MAXKT_ == 1 && NS_ == 2), "packed tiles: L = 64 shape");
   using Cfg = AttnCfg<NQ_, MAXKT_, NS_>;
   constexpr int NS = Cfg::NS;
   constexpr int NQ = Cfg::NQ, kMaxKT = Cfg::kMaxKT, kKSlots = Cfg::kKSlots;
@@ -114,25 +131,27 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
   // nothing the previous kernels write (QKV) or read (O) is touched before pdl_wait().
   // `lengths` is filled by the runtime's input copy, which precedes every kernel of the graph.
   pdl_launch_dependents();
-  const int h = blockIdx.y, b = blockIdx.z;
+  const int h = blockIdx.y, b = blockIdx.z * PACK;  // (first) sequence of the tile
   const int H = heads * D;
   // lengths come from device memory unvalidated (arlo_enqueue, arlo_op_attention): clamp to
   // [0, L] so a bad length can neither index barriers past kMaxKT nor read the next sequence
-  const int len = min(max(__ldg(lengths + b), 0), L);
+  const int len_a = min(max(__ldg(lengths + b), 0), L);
+  const int len_b = PACK == 2 && b + 1 < B ? min(max(__ldg(lengths + b + 1), 0), L) : 0;
+  const int len = PACK == 2 ? (len_a > len_b ? len_a : len_b) : len_a;  // (PACK: live if either is)
   const int q0 = blockIdx.x * (NQ * AQ);
   const int row_base = b * L;
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   if (q0 >= len) {  // every q-tile wholly padded (or empty slot): zeros
     pdl_wait();
-    const int rows = min(NQ * AQ, L - q0);
+    const int rows = PACK == 2 ? (b + 1 < B ? 2 * L : L) : min(NQ * AQ, L - q0);
     for (int i = threadIdx.x; i < rows * 8; i += kAttnThreads) {
       const int r = i >> 3, c = i & 7;
       *reinterpret_cast<uint4*>(o + (size_t)(row_base + q0 + r) * H + h * D + c * 8) = make_uint4(0, 0, 0, 0);
     }
     return;
   }
-  const int n_kt = (len + AK - 1) / AK;  // K/V tiles
-  const int n_ch = (len + KC - 1) / KC;  // 64-key chunks
+  const int n_kt = PACK == 2 ? 1 : (len + AK - 1) / AK;  // K/V tiles
+  const int n_ch = PACK == 2 ? 2 : (len + KC - 1) / KC;  // 64-key chunks
   int nq = 1;  // live q-tiles (trailing ones may be wholly padded)
   while (nq < NQ && q0 + nq * AQ < len) ++nq;
 
@@ -262,6 +281,10 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
     const int qi = warp >> 3, hf = (warp >> 2) & 1, quarter = warp & 3;
     const int r = quarter * 32 + lane;  // query row within q-tile qi == TMEM lane
     const int qrow = q0 + qi * AQ + r;
+    // PACK: this warp's rows are sequence `seg` of the tile, its only real chunk is chunk seg
+    const int seg = PACK == 2 ? quarter >> 1 : 0;
+    const int lenw = PACK == 2 ? (seg ? len_b : len_a) : len;
+    const bool row_live = PACK == 2 ? (b + seg < B) : (qrow < L);  // row exists in the buffer
     const int bar_id = 1 + qi * 4 + quarter;
     auto pair_sync = [&]() { asm volatile("bar.sync %0, 64;" ::"r"(bar_id) : "memory"); };
     if (qi < nq) {
@@ -283,11 +306,18 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           // paired FFMA2 / FADD2: bitwise the scalar fmaf / += (even keys into ls[0], odd into ls[1])
           const float2 x = __ffma2_rn(make_float2(__uint_as_float(v[e]), __uint_as_float(v[e + 1])),
                                       make_float2(c2, c2), make_float2(-mc, -mc));
-          float p0 = ex2_approx(x.x);
-          float p1 = ex2_approx(x.y);
+          float p0, p1;
+          if (e >= 16 - 2 * kPolyPairs) {  // the last kPolyPairs key pairs of a piece on the FMA pipe
+            const float2 pp = ex2_poly2(x);
+            p0 = pp.x;
+            p1 = pp.y;
+          } else {
+            p0 = ex2_approx(x.x);
+            p1 = ex2_approx(x.y);
+          }
           if (MASK) {
-            if (key0 + e >= len) p0 = 0.f;
-            if (key0 + e + 1 >= len) p1 = 0.f;
+            if (key0 + e >= lenw) p0 = 0.f;
+            if (key0 + e + 1 >= lenw) p1 = 0.f;
           }
           acc = __fadd2_rn(acc, make_float2(p0, p1));
           pk[e >> 1] = pack_bf16x2(p0, p1);
@@ -320,8 +350,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         ptx::tmem_wait_ld();
 #pragma unroll
         for (int e = 0; e < 16; ++e) {
-          if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
-          if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
+          if (full || key0 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+          if (full || key0 + 16 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
         }
         return fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
       };
@@ -333,8 +363,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
         ptx::mbar_wait(&s_full[qi * NS + cur], (c / NS) & 1);
         ptx::tc_fence_after();
         if (warp == 0 && lane == 0) atrace<TRACE>(3 + 3 * (c & 7));
-        const int key0 = c * KC + hf * (KC / 2);
-        const bool full = c * KC + KC <= len;
+        const int key0 = (c - seg) * KC + hf * (KC / 2);  // key index within the warp's sequence
+        const bool full = (c - seg) * KC + KC <= lenw;
         const uint32_t t_chunk = t_s + cur * KC;
         const uint32_t t_p = t_lane + kPCol + (qi * NS + cur) * (KC / 2) + hf * (KC / 4);
         // P slot `cur` was read by PV(c - NS)
@@ -343,7 +373,13 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::tc_fence_after();
         }
         float ls;
-        if constexpr (Cfg::ALIAS) {
+        if (PACK == 2 && (c != seg || lenw == 0)) {
+          // the other sequence's keys (or an empty slot): P = 0, no exp, l unchanged
+          const uint32_t z[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+          ptx::tmem_st_32x32b_x8(t_p, z);
+          ptx::tmem_st_32x32b_x8(t_p + 8, z);
+          ls = 0.f;
+        } else if constexpr (Cfg::ALIAS) {
           // one TMEM read of the warp's 32 S values; max, exp and (rare) redo from registers;
           // P stored last, over the first 16 of these S columns
           // (S stays intact in TMEM until P is stored at the end, so the rare redo re-reads it:
@@ -359,8 +395,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
             float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
             for (int e = 0; e < 16; ++e) {
-              if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
-              if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
+              if (full || key0 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+              if (full || key0 + 16 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
             }
             return fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
           };
@@ -372,11 +408,18 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
               const int ee = e & 15;
               const float2 x = __ffma2_rn(make_float2(__uint_as_float(v[ee]), __uint_as_float(v[ee + 1])),
                                           make_float2(c2, c2), make_float2(-mc, -mc));
-              float p0 = ex2_approx(x.x);
-              float p1 = ex2_approx(x.y);
+              float p0, p1;
+              if (ee >= 16 - 2 * kPolyPairs) {  // same key positions as exp_piece
+                const float2 pp = ex2_poly2(x);
+                p0 = pp.x;
+                p1 = pp.y;
+              } else {
+                p0 = ex2_approx(x.x);
+                p1 = ex2_approx(x.y);
+              }
               if (!full) {
-                if (key0 + e >= len) p0 = 0.f;
-                if (key0 + e + 1 >= len) p1 = 0.f;
+                if (key0 + e >= lenw) p0 = 0.f;
+                if (key0 + e + 1 >= lenw) p1 = 0.f;
               }
               acc = __fadd2_rn(acc, make_float2(p0, p1));
               pk[e >> 1] = pack_bf16x2(p0, p1);
@@ -384,7 +427,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
             return acc.x + acc.y;
           };
           load_s();
-          if (c == 0) {
+          if (c == seg) {
             xs[par * AQ + r] = reg_max();
             pair_sync();
             m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
@@ -425,14 +468,14 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           ptx::tmem_st_32x32b_x8(t_chunk + 8, *reinterpret_cast<uint32_t(*)[8]>(&pk[8]));
         } else {
 #if defined(ARLO_ATTN_C0_TWOPASS)  // A/B only: the previous max pass + exp pass over S
-          if (c == 0) {
+          if (c == seg) {
             xs[par * AQ + r] = half_max(full, t_chunk, key0);
             pair_sync();
             m = fmaxf(xch[qi][0][par * AQ + r], xch[qi][1][par * AQ + r]);
             ls = exp_any(full, t_chunk, m * c2, key0, t_p);
           } else
 #endif
-          if (c == 0) {
+          if (c == seg) {
             // first chunk: row max shared by the pair, then exp, from ONE TMEM read of S
             // (values kept in registers across the pair barrier; bitwise the two-pass result)
             uint32_t va[16], vb[16];
@@ -442,8 +485,8 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
             float mx[4] = {-INFINITY, -INFINITY, -INFINITY, -INFINITY};
 #pragma unroll
             for (int e = 0; e < 16; ++e) {
-              if (full || key0 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
-              if (full || key0 + 16 + e < len) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
+              if (full || key0 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(va[e]));
+              if (full || key0 + 16 + e < lenw) mx[e & 3] = fmaxf(mx[e & 3], __uint_as_float(vb[e]));
             }
             xs[par * AQ + r] = fmaxf(fmaxf(mx[0], mx[1]), fmaxf(mx[2], mx[3]));
             pair_sync();
@@ -513,7 +556,10 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
       uint32_t ov[32];
       ptx::tmem_ld_32x32b_x32(t_o, ov);
       ptx::tmem_wait_ld();
-      if (qrow < L) {
+      if (row_live && PACK == 2 && lenw == 0) {
+#pragma unroll
+        for (int i = 0; i < 4; ++i) orow[i] = make_uint4(0, 0, 0, 0);
+      } else if (row_live) {
 #pragma unroll
         for (int i = 0; i < 4; ++i) {
           uint4 u;
@@ -524,7 +570,7 @@ attn_tc_kernel(const __grid_constant__ CUtensorMap tm, int L, int heads, const i
           orow[i] = u;
         }
       }
-    } else if (qrow < L) {
+    } else if (row_live) {
       // q-tile wholly padded: zero rows (each half writes its 32 columns)
       uint4* orow = reinterpret_cast<uint4*>(o + (size_t)(row_base + qrow) * H + h * D) + hf * 4;
 #pragma unroll
@@ -584,24 +630,24 @@ int set_attn_trace(unsigned long long* buf) {
   return (int)cudaMemcpyToSymbol(g_atrace, &buf, sizeof(buf));
 }
 
-template <int NQ, int MAXKT, int NS>
+template <int NQ, int MAXKT, int NS, int PACK = 1>
 cudaError_t attn_launch_cfg(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s) {
   using Cfg = AttnCfg<NQ, MAXKT, NS>;
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [] {
-    cudaError_t r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, false>,
+    cudaError_t r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, false, PACK>,
                                          cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::kSmem);
     if (r == cudaSuccess)
-      r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+      r = cudaFuncSetAttribute(attn_tc_kernel<NQ, MAXKT, NS, true, PACK>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                Cfg::kSmem);
     return r; });
   if (e != cudaSuccess) return e;
-  dim3 grid((p.q_rows + NQ * AQ - 1) / (NQ * AQ), p.heads, p.B);
+  dim3 grid((p.q_rows + NQ * AQ - 1) / (NQ * AQ), p.heads, (p.B + PACK - 1) / PACK);
   if (g_attn_trace_on)
-    return launch_k(attn_tc_kernel<NQ, MAXKT, NS, true>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
-                    lengths, (bf16*)o);
-  return launch_k(attn_tc_kernel<NQ, MAXKT, NS, false>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.L, p.heads,
-                  lengths, (bf16*)o);
+    return launch_k(attn_tc_kernel<NQ, MAXKT, NS, true, PACK>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.B,
+                    p.L, p.heads, lengths, (bf16*)o);
+  return launch_k(attn_tc_kernel<NQ, MAXKT, NS, false, PACK>, grid, dim3(Cfg::kThreads), Cfg::kSmem, s, p.tm, p.B,
+                  p.L, p.heads, lengths, (bf16*)o);
 }
 
 bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv, int q_rows) {
@@ -625,6 +671,9 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
     // TMEM-read budget: 10.6 vs 10.1 us graph-replayed (gpurun_out/ab22)
     if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
 #else
+#if !defined(ARLO_ATTN_NO_PACK)
+    if (p.L == 64) return attn_launch_cfg<1, 1, 2, 2>(p, lengths, o, s);  // two sequences per 128-row tile
+#endif
     if (p.L <= 128) return attn_launch_cfg<1, 1, 2>(p, lengths, o, s);
 #endif
     if (p.L <= 256) return attn_launch_cfg<1, 2, 2>(p, lengths, o, s);

@@ -51,10 +51,31 @@ __device__ __forceinline__ float rcp_approx(float x) {
   asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
   return r;
 }
+__device__ __forceinline__ float2 f2c(float v) { return make_float2(v, v); }
 __device__ __forceinline__ float ex2_approx(float x) {
   float r;
   asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(r) : "f"(x));
   return r;
+}
+
+// 2^x for two values on the FMA pipe (no MUFU): x = j + f with j = rint(x) (the 1.5 * 2^23
+// shifter), f in [-1/2, 1/2], 2^f by its degree-5 Taylor polynomial (relative error <= 2.4e-6,
+// far below the bf16 rounding of P), then j added to the exponent field.  x is clamped at
+// -127, where the result is 0 as ex2.approx.ftz gives.  The attention softmax evaluates a
+// fixed subset of its exponentials this way (by key position only, so every runtime L
+// computes a given key's p identically) to take load off the 16/clk/SM MUFU unit.
+__device__ __forceinline__ float2 ex2_poly2(float2 x) {
+  x = make_float2(fmaxf(x.x, -127.0f), fmaxf(x.y, -127.0f));
+  const float2 t = __fadd2_rn(x, f2c(12582912.0f));
+  const float2 j = __fadd2_rn(t, f2c(-12582912.0f));  // rint(x), exact
+  const float2 f = __fadd2_rn(x, make_float2(-j.x, -j.y));  // exact
+  float2 q = __ffma2_rn(f, f2c(1.3333558146e-3f), f2c(9.6181291076e-3f));
+  q = __ffma2_rn(q, f, f2c(5.5504108665e-2f));
+  q = __ffma2_rn(q, f, f2c(2.4022650696e-1f));
+  q = __ffma2_rn(q, f, f2c(6.9314718056e-1f));
+  q = __ffma2_rn(q, f, f2c(1.0f));
+  return make_float2(__int_as_float(__float_as_int(q.x) + (__float_as_int(t.x) << 23)),
+                     __int_as_float(__float_as_int(q.y) + (__float_as_int(t.y) << 23)));
 }
 
 __device__ __forceinline__ float gelu_erf_fast(float z) {

@@ -165,6 +165,8 @@ def test_embedding_ln(arlo_lib, dtype):
     (192, 3, [192, 191, 129, 128, 1]),
     (320, 2, [320, 257, 200, 0]),
     (448, 2, [448, 385, 300, 64]),
+    (64, 3, [64, 0, 17]),          # packed tiles (L = 64): odd B, empty slot in a pair
+    (64, 2, [1, 64, 40, 2, 0]),
 ])
 @pytest.mark.parametrize("dtype", [0, 1])
 def test_attention_masked(arlo_lib, L, heads, lengths, dtype):
@@ -254,3 +256,23 @@ def test_gemm_fused_layernorm(arlo_lib, M, N, K):
     arlo_lib.op_gemm_ln(bf16_dev(A), bf16_dev(W), f32_dev(b), Rd, f32_dev(g), f32_dev(be), 1e-12, Rd)
     torch.cuda.synchronize()
     assert torch.equal(Rd, out)
+
+
+@pytest.mark.parametrize("B", [5, 32])
+def test_attention_packed_L64_bitwise(arlo_lib, B):
+    """L = 64 runs two sequences per 128-row tile; every row equals bit for bit the row an
+    unpacked tile computes (the same sequences at L = 128, one sequence per tile)."""
+    heads, H = 12, 768
+    rng = np.random.default_rng(B)
+    lens = rng.integers(1, 65, B).astype(np.int32)
+    lens[0] = 64
+    q64 = rnd((B * 64, 3 * H), 300 + B)
+    q128 = rnd((B * 128, 3 * H), 400 + B)  # garbage in rows 64..127 of each sequence
+    q128.reshape(B, 128, 3 * H)[:, :64] = q64.reshape(B, 64, 3 * H)
+    o64 = torch.empty((B * 64, H), device="cuda", dtype=torch.bfloat16)
+    o128 = torch.empty((B * 128, H), device="cuda", dtype=torch.bfloat16)
+    ld = torch.from_numpy(lens).cuda()
+    arlo_lib.op_attention(0, B, 64, heads, bf16_dev(q64), ld, o64)
+    arlo_lib.op_attention(0, B, 128, heads, bf16_dev(q128), ld, o128)
+    torch.cuda.synchronize()
+    assert torch.equal(o64.view(B, 64, H), o128.view(B, 128, H)[:, :64])
