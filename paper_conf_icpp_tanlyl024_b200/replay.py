@@ -24,6 +24,23 @@ import numpy as np
 from . import workload as wl
 
 
+def derive_runtime_set(curve: dict, tol: float = 0.05, max_len: int = 512):
+    """Runtime max_lengths from a latency staircase (§3.3: within one step the
+    latency changes < 5 %, so a runtime per step): walk L upwards from the start of the current
+    step; when lat(L) exceeds (1 + tol) * lat(step start) the previous L ends the step and
+    becomes a runtime.  curve: {L: latency}.  The last runtime is max_len (Eq. 7)."""
+    Ls = sorted(int(k) for k in curve)
+    out, start, prev = [], Ls[0], Ls[0]
+    for L in Ls[1:]:
+        if curve[L] > (1.0 + tol) * curve[start]:
+            out.append(prev)
+            start = L
+        prev = L
+    if not out or out[-1] != max_len:
+        out.append(max_len)
+    return out
+
+
 def capacities(per_L_ms: dict, slo_ms: float, max_batch: int):
     """M_i: largest profiled batch whose forward latency fits the SLO (>= 1)."""
     caps = {}
@@ -131,10 +148,19 @@ def plan_cluster(arlo, G: int, Ls, lat_ms, shares, rate: float, slo_ms: float):
     of runtime i at batch b; shares[i]: fraction of requests whose ideal runtime is i; rate: offered
     req/s.  Q_i = requests per SLO window in bin i; M_i = slo_capacity.  Returns (N, Q, M)."""
     lat = np.asarray(lat_ms, np.float64)
-    Q = np.asarray(shares, np.float64) * rate * slo_ms / 1e3
     M = np.array([slo_capacity(row, slo_ms) for row in lat])
-    N, _obj = arlo.allocate(G, Q, M, lat)
-    return list(N), Q, M
+    # Eq. 3 (N_i >= floor(Q_i / M_i)) with Eq. 7 can need more than G GPUs at a high offered
+    # rate (EINFEASIBLE): plan for the highest rate the G GPUs can hold, lowering it by 10 % steps
+    for _ in range(200):
+        Q = np.asarray(shares, np.float64) * rate * slo_ms / 1e3
+        try:
+            N, _obj = arlo.allocate(G, Q, M, lat)
+            return list(N), Q, M
+        except arlo.ArloError as e:
+            if e.code != arlo.EINFEASIBLE:
+                raise
+            rate *= 0.9
+    raise RuntimeError(f"no feasible allocation on {G} GPUs")
 
 
 def simulate_cluster(arrivals, lengths, Ls, n_inst, capacity, service_fn, max_batch: int,
@@ -206,6 +232,7 @@ def summarize(arrivals, lengths, done, runtime_of, Ls, slo_ms: float):
            "p99_ms": float(np.percentile(lat_ms, 99)), "slo_violations": float((lat_ms > slo_ms).mean()),
            "per_bucket": {}}
     ideal = wl.ideal_runtime(lengths, Ls)
+    out["demoted"] = float((runtime_of != ideal).mean())  # served by a longer runtime than its ideal one
     for k, L in enumerate(Ls):
         m = ideal == k
         if m.any():
@@ -362,14 +389,15 @@ def dispatch_ablation(arlo, torch, runtimes: dict, cfg, G: int = 8, n_requests: 
     N, _Q, _M = plan_cluster(arlo, G, Ls, lat, shares, 0.7 * sat, slo_ms)
     sat = run(N, zero, "rs")["served_rate"]
     arrivals_fn = wl.mmpp_arrivals if bursty else wl.poisson_arrivals
-    res = {"G": G, "instances": {str(L): int(N[k]) for k, L in enumerate(Ls)}, "rs_saturation_req_s": sat,
+    res = {"G": G, "max_batch": max_batch, "capacity_per_slo_window": {str(L): caps[k] for k, L in enumerate(Ls)},
+           "instances": {str(L): int(N[k]) for k, L in enumerate(Ls)}, "rs_saturation_req_s": sat,
            "arrivals": "MMPP (Twitter-Bursty-like)" if bursty else "Poisson", "points": []}
     for f in loads:
         arr = arrivals_fn(n_requests, f * sat, seed=wl.SEED_ARRIVALS)
         row = {"load": f, "offered_req_s": f * sat}
         for pol in ("rs", "ilb", "ig"):
             r = run(N, arr, pol)
-            row[pol] = {k: r[k] for k in ("mean_ms", "p98_ms", "p99_ms", "slo_violations")}
+            row[pol] = {k: r[k] for k in ("mean_ms", "p98_ms", "p99_ms", "slo_violations", "demoted")}
         res["points"].append(row)
     return res
 

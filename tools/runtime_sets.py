@@ -3,6 +3,7 @@ L369-371 5.2.3: N = 8 vs 16 runtimes).
 
     python tools/runtime_sets.py staircase        # BERT-base forward latency at L = 16..512 step 16, b = 1, 8, 32
     python tools/runtime_sets.py count [G]        # N in {2, 4, 8, 16} runtimes (step 512/N), ILP on G GPUs
+The staircase output includes the runtime set replay.derive_runtime_set() reads off it at b = 1, 8, 32.
 Prints one JSON object.
 """
 import json
@@ -74,7 +75,9 @@ def main():
     s = torch.cuda.Stream()
     W = arlo.Weights(cfg, arlo.upload_weights(cfg, wl.make_weights(cfg), arlo.BF16, dev), arlo.BF16)
     if mode == "staircase":
-        print(json.dumps({"staircase_ms": staircase(W, cfg, s)}))
+        st = staircase(W, cfg, s)
+        derived = {b: replay.derive_runtime_set({int(L): row[b]["ms"] for L, row in st.items()}) for b in ("1", "8", "32")}
+        print(json.dumps({"staircase_ms": st, "derived_runtime_set_tol5pct": derived}))
     else:
         G = int(sys.argv[2]) if len(sys.argv) > 2 else 16
         print(json.dumps({"runtime_count": count(W, cfg, s, G), "G": G}))
