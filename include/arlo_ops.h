@@ -78,6 +78,21 @@ int arlo_op_head(int32_t dtype, int32_t B, int32_t L, int32_t H, int32_t C, cons
                  const void* w_p, const float* b_p, const void* w_c, const float* b_c,
                  float* pooled, float* logits, void* stream);
 
+/*
+ * Steps a5/a8 + a6 (or the next layer's a2) in one launch, as the runtime graphs run them:
+ * x = LN(y; gamma, beta, eps) over M rows of K = hidden (LayerNorm of the residual GEMM's
+ * output, reading S3), then out = epi(x W^T + bias), epi = ARLO_EPI_BIAS or ARLO_EPI_BIAS_GELU.
+ * y, x: [M, K] bf16 DEVICE (x is written: the next residual); W [N, K] bf16; out [M, N] bf16.
+ * The whole persistent grid normalises the rows, meets at a grid barrier (`barrier`: 8 bytes of
+ * zero-initialised DEVICE memory, reusable by later calls on the same stream), then runs the GEMM.
+ * force_bn: a persistent tile code (BN / -BN, see arlo_gemm_tile_choice), 0 = chooser; EINVAL if
+ * that kernel is the skinny one (its grid is not persistent).  Launches with a grid barrier must
+ * not run concurrently with one another on the same device (one runtime stream per device).
+ */
+int arlo_op_ln_gemm(int32_t M, int32_t N, int32_t K, const void* y, const float* gamma, const float* beta, float eps,
+                    void* x, const void* W, const float* bias, void* out, int32_t epi, int32_t force_bn,
+                    void* barrier, void* stream);
+
 /* The tile configuration arlo_op_gemm / the runtime graphs use for (M, N, K):
  * BN for the single-CTA kernel, -BN for the CTA-pair kernel, 1000 + BN for the
  * skinny small-M kernel, 0 if unsupported. */

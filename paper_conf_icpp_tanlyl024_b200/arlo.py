@@ -37,7 +37,7 @@ EXPORTED = [
     "arlo_runtime_create", "arlo_runtime_create_ex", "arlo_runtime_family", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_sched_set_policy", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
-    "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
+    "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_ln_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
     "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
 ]
 
@@ -87,6 +87,7 @@ _sig("arlo_complete", C.c_int, _vp, _i32, _i32)
 _sig("arlo_sched_outstanding", _i32, _vp, _i32, _i32)
 _sig("arlo_op_gemm", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _i32, _i32, _vp)
 _sig("arlo_op_gemm_ln", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp)
+_sig("arlo_op_ln_gemm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp, _vp, _vp, _i32, _i32, _vp, _vp)
 _sig("arlo_op_layernorm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp)
 _sig("arlo_op_embed", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp, _vp)
 _sig("arlo_op_attention", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp)
@@ -293,6 +294,19 @@ def op_gemm_ln(A, W, bias, residual, gamma, beta, eps, out, stream=None):
     N = W.shape[0]
     check(lib.arlo_op_gemm_ln(M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(residual), _ptr(gamma), _ptr(beta), eps,
                               _ptr(out), _stream_ptr(stream)))
+    return out
+
+
+def op_ln_gemm(y, gamma, beta, eps, x, W, bias, out, epi=EPI_BIAS, force_bn=0, barrier=None, stream=None):
+    """x = LN(y) and out = epi(x W^T + bias) in one launch (LayerNorm prologue of a persistent GEMM).
+    barrier: >= 2 zero-initialised int32 on the device (allocated here if None)."""
+    import torch
+    M, K = y.shape
+    N = W.shape[0]
+    if barrier is None:
+        barrier = torch.zeros(2, dtype=torch.int32, device=y.device)
+    check(lib.arlo_op_ln_gemm(M, N, K, _ptr(y), _ptr(gamma), _ptr(beta), eps, _ptr(x), _ptr(W), _ptr(bias),
+                              _ptr(out), epi, force_bn, _ptr(barrier), _stream_ptr(stream)))
     return out
 
 

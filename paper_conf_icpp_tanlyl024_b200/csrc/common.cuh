@@ -196,6 +196,33 @@ inline cudaError_t once_per_device(std::atomic<uint64_t>& done, SetFn set) {
   return e;
 }
 
+// Grid-wide barrier of a PERSISTENT grid (every CTA resident at once: grid <= one CTA per SM).
+// bar[0] counts arrivals and is reset by the last arriver, bar[1] is a generation counter the
+// waiters poll, so the same zero-initialised pair serves every later launch (graph replays).
+// Each CTA's thread 0 reads the generation BEFORE arriving; release / acquire at gpu scope
+// order the CTA's prior writes before the other CTAs' later reads.
+__device__ __forceinline__ unsigned ld_acquire_gpu(const unsigned* p) {
+  unsigned v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void grid_barrier(unsigned* bar) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    const unsigned gen = ld_acquire_gpu(bar + 1);
+    __threadfence();
+    if (atomicAdd(bar, 1u) == gridDim.x * gridDim.y * gridDim.z - 1) {
+      atomicExch(bar, 0u);
+      __threadfence();
+      atomicAdd(bar + 1, 1u);
+    } else {
+      while (ld_acquire_gpu(bar + 1) == gen) __nanosleep(20);
+    }
+    __threadfence();
+  }
+  __syncthreads();
+}
+
 template <typename... KArgs, typename... Args>
 inline cudaError_t launch_k(void (*kern)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t s,
                             Args&&... args) {

@@ -11,6 +11,7 @@
 // 3*H*sizeof(T) read (word, pos, type) + H*sizeof(T) written.
 #include "common.cuh"
 #include "kernels.h"
+#include "layernorm.cuh"
 
 namespace arlo {
 
@@ -22,38 +23,6 @@ namespace {
 constexpr int kRowsPerBlock = ARLO_LN_ROWS;  // one warp per row
 constexpr int kLnThreads = 32 * kRowsPerBlock;
 
-template <typename T> struct Vec;
-template <> struct Vec<bf16> {
-  static constexpr int N = 8;  // 16 B
-  static __device__ __forceinline__ void load(const bf16* p, float* f, bool dep = false) {
-    uint4 u = dep ? ld_dep_v4(p) : __ldg(reinterpret_cast<const uint4*>(p));
-    float2 a = unpack_bf16x2(u.x), b = unpack_bf16x2(u.y), c = unpack_bf16x2(u.z), d = unpack_bf16x2(u.w);
-    f[0] = a.x; f[1] = a.y; f[2] = b.x; f[3] = b.y; f[4] = c.x; f[5] = c.y; f[6] = d.x; f[7] = d.y;
-  }
-  static __device__ __forceinline__ void store(bf16* p, const float* f) {
-    uint4 u;
-    u.x = pack_bf16x2(f[0], f[1]); u.y = pack_bf16x2(f[2], f[3]);
-    u.z = pack_bf16x2(f[4], f[5]); u.w = pack_bf16x2(f[6], f[7]);
-    *reinterpret_cast<uint4*>(p) = u;
-  }
-};
-template <> struct Vec<float> {
-  static constexpr int N = 4;
-  static __device__ __forceinline__ void load(const float* p, float* f, bool dep = false) {
-    float4 v;
-    if (dep) {
-      const uint4 u = ld_dep_v4(p);
-      v = make_float4(__uint_as_float(u.x), __uint_as_float(u.y), __uint_as_float(u.z), __uint_as_float(u.w));
-    } else {
-      v = __ldg(reinterpret_cast<const float4*>(p));
-    }
-    f[0] = v.x; f[1] = v.y; f[2] = v.z; f[3] = v.w;
-  }
-  static __device__ __forceinline__ void store(float* p, const float* f) {
-    *reinterpret_cast<float4*>(p) = make_float4(f[0], f[1], f[2], f[3]);
-  }
-};
-
 // gamma / beta are weights, independent of the predecessor kernel: every CTA stages them in
 // shared memory BEFORE the PDL wait, so their L2 round trip overlaps the previous kernel's tail
 // instead of sitting between the row statistics and the normalisation.
@@ -64,55 +33,6 @@ __device__ __forceinline__ void stage_affine(int H, const float* __restrict__ g,
     *reinterpret_cast<float4*>(sb + i) = __ldg(reinterpret_cast<const float4*>(b + i));
   }
   __syncthreads();
-}
-
-// Normalise the row held in v[MAXV][VN] (only vectors lane + 32 i < nvec valid) and store it.
-// g, b point to the shared-memory copies of gamma / beta.
-template <typename T, int MAXV>
-__device__ __forceinline__ void ln_finish(float (&v)[MAXV][Vec<T>::N], int nvec, int H, int lane,
-                                          const float* g, const float* b,
-                                          float eps, T* __restrict__ out_row) {
-  constexpr int VN = Vec<T>::N;
-  float s = 0.f;
-#pragma unroll
-  for (int i = 0; i < MAXV; ++i) {
-    if (lane + 32 * i < nvec) {
-#pragma unroll
-      for (int j = 0; j < VN; ++j) s += v[i][j];
-    }
-  }
-  const float mean = warp_sum(s) / (float)H;
-  float q = 0.f;
-#pragma unroll
-  for (int i = 0; i < MAXV; ++i) {
-    if (lane + 32 * i < nvec) {
-#pragma unroll
-      for (int j = 0; j < VN; ++j) {
-        const float d = v[i][j] - mean;
-        q += d * d;
-      }
-    }
-  }
-  const float var = warp_sum(q) / (float)H;
-  const float rstd = 1.0f / sqrtf(var + eps);
-#pragma unroll
-  for (int i = 0; i < MAXV; ++i) {
-    const int vi = lane + 32 * i;
-    if (vi < nvec) {
-      const int c0 = vi * VN;
-      float gg[VN], bb[VN], o[VN];
-#pragma unroll
-      for (int j = 0; j < VN; j += 4) {
-        const float4 g4 = *reinterpret_cast<const float4*>(g + c0 + j);
-        const float4 b4 = *reinterpret_cast<const float4*>(b + c0 + j);
-        gg[j] = g4.x; gg[j + 1] = g4.y; gg[j + 2] = g4.z; gg[j + 3] = g4.w;
-        bb[j] = b4.x; bb[j + 1] = b4.y; bb[j + 2] = b4.z; bb[j + 3] = b4.w;
-      }
-#pragma unroll
-      for (int j = 0; j < VN; ++j) o[j] = (v[i][j] - mean) * rstd * gg[j] + bb[j];
-      Vec<T>::store(out_row + c0, o);
-    }
-  }
 }
 
 template <typename T, int MAXV>

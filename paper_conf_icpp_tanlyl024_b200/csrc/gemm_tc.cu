@@ -29,6 +29,7 @@
 #include "common.cuh"
 #include "epilogue.cuh"
 #include "kernels.h"
+#include "layernorm.cuh"
 #include "ptx.cuh"
 
 namespace arlo {
@@ -249,7 +250,7 @@ template <int BN, int EPI, int EW>
 __global__ void __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-               const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
+               const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
   using C = TcCfg<BN, false, 0, EW>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
@@ -292,19 +293,26 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   const uint32_t tmem_base = *tmem_slot;
   pdl_launch_dependents();  // setup above overlapped the previous kernel's tail
 
+  // W never depends on the previous kernel: the first tile's first STAGES W tiles are
+  // requested before the PDL wait (and before the LayerNorm prologue), its A tiles after it
+  const int pre = blockIdx.x < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
+  if (warp == kProducerWarp && lane == 0) {
+    const int n0 = tile_n(blockIdx.x, num_m, num_n) * BN;
+    for (int kb = 0; kb < pre; ++kb) {
+      ptx::mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
+      ptx::tma_load_2d(sB + kb * C::B_BYTES, &tmB, &full[kb], kb * BK, n0);
+    }
+  }
+  if constexpr (EPI != EPI_BIAS_RESID) {
+    if (lnp.y != nullptr) {  // A = LN(y), computed by the whole grid first (layernorm.cuh)
+      pdl_wait();
+      ln_prologue(lnp);
+    }
+  }
+
   if (warp == kProducerWarp) {
     // ------------------------------------------------------------ TMA producer
     if (lane == 0) {
-      // W never depends on the previous kernel: the first tile's first STAGES W
-      // tiles are requested before the PDL wait, its A tiles right after it
-      const int pre = blockIdx.x < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
-      {
-        const int n0 = tile_n(blockIdx.x, num_m, num_n) * BN;
-        for (int kb = 0; kb < pre; ++kb) {
-          ptx::mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
-          ptx::tma_load_2d(sB + kb * C::B_BYTES, &tmB, &full[kb], kb * BK, n0);
-        }
-      }
       pdl_wait();
       if (threadIdx.x == kProducerWarp * 32) trace(0);
       int stage = 0;
@@ -409,7 +417,7 @@ template <int BN, int EPI, int EW>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
-                    const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp) {
+                    const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
   using C = TcCfg<BN, true, 0, EW>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
@@ -454,17 +462,24 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   const uint32_t tmem_base = *tmem_slot;
   pdl_launch_dependents();  // setup above overlapped the previous kernel's tail
 
+  // W tiles of the first tile are requested before the PDL wait (see gemm_tc_kernel)
+  const int pre = pair < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
+  if (warp == kProducerWarp && lane == 0) {
+    const int n0 = tile_n(pair, num_m, num_n) * BN + rank * C::B_ROWS;
+    for (int kb = 0; kb < pre; ++kb) {
+      if (rank == 0) ptx::mbar_arrive_expect_tx(&full[kb], 2 * C::STAGE_BYTES);
+      ptx::tma_load_2d_pair(sB + kb * C::B_BYTES, &tmB, ptx::mapa_shared(&full[kb], 0), kb * BK, n0);
+    }
+  }
+  if constexpr (EPI != EPI_BIAS_RESID) {
+    if (lnp.y != nullptr) {  // A = LN(y), computed by the whole grid first (layernorm.cuh)
+      pdl_wait();
+      ln_prologue(lnp);
+    }
+  }
+
   if (warp == kProducerWarp) {
     if (lane == 0) {
-      // W tiles of the first tile are requested before the PDL wait (see gemm_tc_kernel)
-      const int pre = pair < tiles ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
-      {
-        const int n0 = tile_n(pair, num_m, num_n) * BN + rank * C::B_ROWS;
-        for (int kb = 0; kb < pre; ++kb) {
-          if (rank == 0) ptx::mbar_arrive_expect_tx(&full[kb], 2 * C::STAGE_BYTES);
-          ptx::tma_load_2d_pair(sB + kb * C::B_BYTES, &tmB, ptx::mapa_shared(&full[kb], 0), kb * BK, n0);
-        }
-      }
       pdl_wait();
       if (threadIdx.x == kProducerWarp * 32) trace(0);
       int stage = 0;
@@ -740,22 +755,32 @@ gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
 // sum (y-mean)^2) in fp32 as in the unfused LayerNorm; the normalised row is
 // written once (TMA store).  Removes the LayerNorm kernels and the y round
 // trip through memory.
+constexpr int kMaxLnCluster = 8;  // CTAs per row block (N / BN) of the fused LayerNorm kernel
+
+// Sum of one value per (row, column group) over every CTA of the cluster (the full row of
+// the fused LayerNorm).  Each epilogue warp pushes its 32 rows' partial sums into the
+// exchange buffer of EVERY CTA of the cluster with st.async, which completes transaction
+// bytes on that CTA's stat barrier; each CTA arms its own barrier for the bytes of one use
+// (nt CTAs x kEpiWarps warps x 32 rows x 4 B) and waits on it locally.  No fence: the
+// st.async / complete_tx pair orders the data with the barrier (the previous exchange,
+// an arrive.release.cluster per warp and CTA, cost a MEMBAR.ALL.GPU each).  The sum runs
+// over CTAs and column groups in a fixed order, so every CTA gets the same bits.  Two
+// buffer sets alternate: set s is rewritten only after the exchange between has completed
+// cluster-wide, i.e. after every warp has read set s.
 template <int BN>
 __device__ __forceinline__ float cluster_row_sum(float v, float* red, uint64_t* stat_bar, int& use, int cg,
-                                                 int r_local, int lane, uint32_t nt) {
+                                                 int r_local, int lane, uint32_t nt, uint32_t rank, int warp) {
   const int set = use & 1;
-  float* slot = red + (set * kEpiGroups + cg) * BM + r_local;  // red[set][column group][row]
-  *slot = v;
-  __syncwarp();
-  if (lane == 0) {
-    for (uint32_t k = 0; k < nt; ++k) ptx::mbar_arrive_cluster(ptx::mapa_shared(&stat_bar[set], k));
-  }
-  ptx::mbar_wait_cluster(&stat_bar[set], (use >> 1) & 1);
+  if (warp == 0 && lane == 0) ptx::mbar_arrive_expect_tx(&stat_bar[set], nt * kEpiWarps * 32 * 4);
+  float* base = red + (size_t)set * kMaxLnCluster * kEpiGroups * BM;  // red[set][cta][column group][row]
+  float* slot = base + ((size_t)rank * kEpiGroups + cg) * BM + r_local;
+  for (uint32_t k = 0; k < nt; ++k)
+    ptx::st_async_b32(ptx::mapa_shared(slot, k), __float_as_uint(v), ptx::mapa_shared(&stat_bar[set], k));
+  ptx::mbar_wait(&stat_bar[set], (use >> 1) & 1);
   float tot = 0.f;
   for (uint32_t k = 0; k < nt; ++k) {
 #pragma unroll
-    for (int g = 0; g < kEpiGroups; ++g)
-      tot += ptx::ld_shared_cluster_f32(ptx::mapa_shared(red + (set * kEpiGroups + g) * BM + r_local, k));
+    for (int g = 0; g < kEpiGroups; ++g) tot += base[((size_t)k * kEpiGroups + g) * BM + r_local];
   }
   ++use;
   return tot;
@@ -767,7 +792,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
                                                  const bf16* __restrict__ resid, const float* __restrict__ gamma,
                                                  const float* __restrict__ beta, const CUtensorMap* tmC, uint8_t* stg,
                                                  int& sc, float* red, uint64_t* stat_bar, int& use, uint32_t nt,
-                                                 Release release) {
+                                                 uint32_t rank, int warp, Release release) {
   constexpr int COLS = BN / kEpiGroups;
   static_assert(COLS % 32 == 0, "fused LN epilogue: 32-column chunks");
   constexpr int NC = COLS / 32;
@@ -813,7 +838,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
     ptx::tmem_st_32x32b_x32(t_row + c * 32, r);
   }
   ptx::tmem_wait_st();
-  const float mean = cluster_row_sum<BN>(s1, red, stat_bar, use, cg, r_local, lane, nt) / (float)N;
+  const float mean = cluster_row_sum<BN>(s1, red, stat_bar, use, cg, r_local, lane, nt, rank, warp) / (float)N;
   // pass 2: sum of squared deviations
   float s2 = 0.f;
 #pragma unroll 1
@@ -827,7 +852,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
       s2 = fmaf(d, d, s2);
     }
   }
-  const float var = cluster_row_sum<BN>(s2, red, stat_bar, use, cg, r_local, lane, nt) / (float)N;
+  const float var = cluster_row_sum<BN>(s2, red, stat_bar, use, cg, r_local, lane, nt, rank, warp) / (float)N;
   const float rstd = 1.0f / sqrtf(var + eps);
   // pass 3: normalise, affine, bf16, TMA store
 #pragma unroll 1
@@ -872,7 +897,7 @@ __device__ __forceinline__ void epilogue_ln_tile(uint32_t t_acc, int q, int cg, 
   }
 }
 
-constexpr int kLnReserve = 2 * kEpiGroups * BM * 4 + 16;  // row-statistics exchange buffers + 2 stat barriers
+constexpr int kLnReserve = 2 * kMaxLnCluster * kEpiGroups * BM * 4 + 16;  // row-statistics exchange + 2 barriers
 
 template <int BN>
 __global__ void __launch_bounds__(kThreads, 1)
@@ -886,8 +911,8 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
-  float* red = reinterpret_cast<float*>(sStg + kStagingBytes);  // [2 sets][column groups][128 rows]
-  uint64_t* full = reinterpret_cast<uint64_t*>(red + 2 * kEpiGroups * BM);
+  float* red = reinterpret_cast<float*>(sStg + kStagingBytes);  // [2 sets][8 CTAs][column groups][128 rows]
+  uint64_t* full = reinterpret_cast<uint64_t*>(red + 2 * kMaxLnCluster * kEpiGroups * BM);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
@@ -915,7 +940,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], kEpiWarps);
     }
-    for (int i = 0; i < 2; ++i) ptx::mbar_init(&stat_bar[i], kEpiWarps * nt);
+    for (int i = 0; i < 2; ++i) ptx::mbar_init(&stat_bar[i], 1);  // one arming arrive + the st.async bytes
     ptx::fence_mbar_init();
   }
   if (warp == kMmaWarp) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
@@ -923,23 +948,39 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   ptx::cluster_sync();  // peers' stat barriers are initialised before any remote arrive
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  pdl_begin();
+  pdl_launch_dependents();
 
   if (warp == kProducerWarp) {
     if (lane == 0) {
+      // W never depends on the previous kernel: the first row block's first W stages before the
+      // PDL wait, its A stages after it (as in gemm_tc_kernel)
+      const int pre = cid < num_m ? (kblocks < C::STAGES ? kblocks : C::STAGES) : 0;
+      for (int kb = 0; kb < pre; ++kb) {
+        ptx::mbar_arrive_expect_tx(&full[kb], C::STAGE_BYTES);
+        ptx::tma_load_2d(sB + kb * C::B_BYTES, &tmB, &full[kb], kb * BK, n0);
+      }
+      pdl_wait();
       int stage = 0;
       uint32_t phase = 0;
-      for (int mb = cid; mb < num_m; mb += ncl) {
+      int it = 0;
+      for (int mb = cid; mb < num_m; mb += ncl, ++it) {
         for (int kb = 0; kb < kblocks; ++kb) {
-          ptx::mbar_wait(&empty[stage], phase ^ 1);
-          ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
-          ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, mb * BM);
-          ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          if (it == 0 && kb < pre) {
+            ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, mb * BM);
+          } else {
+            ptx::mbar_wait(&empty[stage], phase ^ 1);
+            ptx::mbar_arrive_expect_tx(&full[stage], C::STAGE_BYTES);
+            ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, mb * BM);
+            ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
+          }
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
         }
       }
+    } else {
+      pdl_wait();
     }
   } else if (warp == kMmaWarp) {
+    pdl_wait();
     {  // converged warp, elected lane issues
       constexpr uint32_t idesc = ptx::idesc_bf16_f32(BM, BN);
       int stage = 0;
@@ -967,6 +1008,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else {
+    pdl_wait();  // residual rows come from the previous kernels
     const int q = warp & 3, cg = warp >> 2;
     uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
     int sc = 0, use = 0;
@@ -977,7 +1019,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::tc_fence_after();
       uint64_t* te = &tempty[acc];
       epilogue_ln_tile<BN>(tmem_base + acc * BN, q, cg, lane, mb * BM + q * 32, n0, M, N, eps, bias, resid, gamma,
-                           beta, &tmC, stg, sc, red, stat_bar, use, nt, [te]() { ptx::mbar_arrive(te); });
+                           beta, &tmC, stg, sc, red, stat_bar, use, nt, rank, warp, [te]() { ptx::mbar_arrive(te); });
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
     if (lane == 0) ptx::bulk_wait<0>();
@@ -1019,7 +1061,7 @@ cudaError_t launch_cfg_ew(const TcGemmPlan& p, cudaStream_t s) {
     return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
   if (e != cudaSuccess) return e;
   return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K,
-                  p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out);
+                  p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out, p.lnp);
 }
 
 template <int BN, int EPI, bool PAIR>
@@ -1152,7 +1194,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   if (choice > kSkinnyCode) {
     const int bn = choice - kSkinnyCode;
     if ((bn != 16 && bn != 32 && bn != 64) || N % bn) return false;
-    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->splitk = false; p->epi = epi; p->ln = false; p->ew = 4;
+    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->splitk = false; p->lnp = LnPrologue{}; p->epi = epi; p->ln = false; p->ew = 4;
     p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
     p->a_rows = M < BM ? ((M + 7) & ~7) : BM;
     p->grid = (N / bn) * ((M + BM - 1) / BM);
@@ -1165,7 +1207,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   if (bn != 64 && bn != 96 && bn != 128 && bn != 192 && bn != 256) return false;
   if (pair && bn < 128) return false;
   if (N % bn) return false;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->splitk = false; p->epi = epi; p->ln = false;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = pair; p->skinny = false; p->splitk = false; p->lnp = LnPrologue{}; p->epi = epi; p->ln = false;
   p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
   const int tile_m = pair ? 2 * BM : BM;
   const int tiles = ((M + tile_m - 1) / tile_m) * (N / bn);
@@ -1216,12 +1258,15 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
                      const void* resid, const float* gamma, const float* beta, float eps, void* out) {
   if (M <= 0 || K % 64 || K <= 0) return false;
   int bn = 0;
-  if (N % 192 == 0 && N / 192 <= 8 && N > 256 && (192 / kEpiGroups) % 32 == 0) bn = 192;
+  // the widest tile that still gives >= 4 CTAs per row block (more CTAs per wave): N = 768 -> 192 x 4,
+  // N = 1024 -> 256 x 4
   if (N % 256 == 0 && N / 256 <= 8 && (256 / kEpiGroups) % 32 == 0 && 256 % kEpiGroups == 0) bn = 256;
+  if (N % 192 == 0 && N / 192 <= 8 && N / 192 >= 4 && (N % 256 || N / 256 < 4) && (192 / kEpiGroups) % 32 == 0)
+    bn = 192;
   if (N == 128 && (128 / kEpiGroups) % 32 == 0 && 128 % kEpiGroups == 0) bn = 128;
   if (!bn) return false;
   const int nt = N / bn;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->splitk = false; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->splitk = false; p->lnp = LnPrologue{}; p->epi = EPI_BIAS_RESID; p->ln = true;
   p->ew = kEpiWarps;
   p->bias = bias; p->resid = resid; p->ldr = N; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
   const int num_m = (M + BM - 1) / BM;
@@ -1230,6 +1275,15 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
+  return true;
+}
+
+bool tc_plan_attach_ln(TcGemmPlan* p, const LnPrologue& lnp) {
+  // persistent tile kernels only (grid <= one CTA per SM: every CTA resident for the grid barrier)
+  if (p->skinny || p->splitk || p->ln || p->epi == EPI_BIAS_RESID) return false;
+  if (lnp.H % 8 || lnp.H > 1024 || lnp.rows <= 0 || !lnp.y || !lnp.x || !lnp.bar) return false;
+  if (p->grid > num_sms()) return false;
+  p->lnp = lnp;
   return true;
 }
 

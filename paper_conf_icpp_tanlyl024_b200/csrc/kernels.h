@@ -26,6 +26,18 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
                              const float* b, float eps, void* out, cudaStream_t s);
 
 // ---- a2/a4/a6/a7: GEMM + fused epilogue ----------------------------------------------------
+// LayerNorm run as the prologue of a persistent GEMM (layernorm.cuh): x = LN(y) over `rows`
+// rows of H, then a grid barrier, then the GEMM on x.  y == nullptr: no prologue.
+struct LnPrologue {
+  const void* y;   // [rows, H] bf16 input (the previous residual GEMM's output)
+  const float* g;  // gamma [H]
+  const float* b;  // beta [H]
+  void* x;         // [rows, H] bf16 output (this GEMM's A operand)
+  unsigned* bar;   // grid barrier {count, generation}: zero-initialised device memory
+  float eps;
+  int rows, H;
+};
+
 // tcgen05 plan: tensor maps are encoded once (at runtime create) and the
 // launch is then a plain kernel launch that CUDA graphs can capture.
 struct TcGemmPlan {
@@ -50,7 +62,11 @@ struct TcGemmPlan {
   const void* resid;
   int ldr;  // residual row stride (elements)
   void* out;
+  LnPrologue lnp;  // (bias / GELU epilogues of the persistent tile kernels only)
 };
+// Attach a LayerNorm prologue to a planned GEMM whose A operand is lnp.x; false if the plan's
+// kernel cannot run it (skinny / split-K / residual epilogue / H > 1024).
+bool tc_plan_attach_ln(TcGemmPlan* p, const LnPrologue& lnp);
 bool tc_plan_gemm(TcGemmPlan* p, int M, int N, int K, const void* A, const void* W,
                   const float* bias, const void* resid, void* out, int epi, int force_bn);
 // Row-strided variant: A row i at A + i*lda, residual row i at resid + i*ldr (elements).

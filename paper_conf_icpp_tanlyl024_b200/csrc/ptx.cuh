@@ -291,6 +291,15 @@ __device__ __forceinline__ float4 ld_shared_cluster_v4(uint32_t cluster_addr) {
   return v;
 }
 
+// Asynchronous 4-byte store into the shared memory of a CTA of the cluster that completes
+// `4 bytes` of transaction count on an mbarrier of that CTA (both shared::cluster addresses):
+// the receiver learns the data has landed from its own barrier, with no fence on either side.
+__device__ __forceinline__ void st_async_b32(uint32_t cluster_addr, uint32_t v, uint32_t cluster_bar) {
+  asm volatile("st.async.shared::cluster.mbarrier::complete_tx::bytes.b32 [%0], %1, [%2];"
+               ::"r"(cluster_addr), "r"(v), "r"(cluster_bar)
+               : "memory");
+}
+
 // Arrive on an mbarrier of another CTA of the cluster with CTA-scope release (the CUTLASS
 // ClusterBarrier::arrive form): no fence.  Enough when the arrive only hands back a resource
 // whose last use is already complete (e.g. an accumulator whose tcgen05.ld's were waited on and

@@ -159,6 +159,9 @@ struct LayerPlans {
 struct Bucket {
   int b = 0;
   std::vector<LayerPlans> plans;  // bf16 only
+  // LayerNorm run as the prologue of the GEMM that consumes it (layernorm.cuh): ln1_in_f1[l] =
+  // layer l's LN1 runs inside its FFN1 GEMM, ln2_in_qkv[l] = layer l's LN2 inside layer l+1's QKV
+  std::vector<char> ln1_in_f1, ln2_in_qkv;
   bool fused_ln = false;          // o / f2 plans carry residual + LayerNorm (no separate LN kernels)
   int tiles[4] = {0, 0, 0, 0};    // measured tile codes of the qkv, o, f1, f2 GEMMs (pick_tile)
   AttnPlan attn;
@@ -189,6 +192,7 @@ struct arlo_runtime {
   int32_t* ids = nullptr;      // [max_batch * L]
   float* logits = nullptr;     // [max_batch * C]
   float* pooled = nullptr;     // [max_batch * H] fp32 pooler output
+  unsigned* gbar = nullptr;    // grid barrier of the LayerNorm-prologue GEMMs (zero-initialised)
   void *X = nullptr, *QKV = nullptr, *O = nullptr, *Y = nullptr, *F = nullptr;
   // pinned host staging
   void* h_stage = nullptr;
@@ -242,7 +246,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "out-proj gemm launch");
     }
-    if (!bk.fused_ln)
+    if (!bk.fused_ln && !(l < (int)bk.ln1_in_f1.size() && bk.ln1_in_f1[l]))
       ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
                                  c.ln_eps, rt->X, s),
                 "ln1 launch");
@@ -257,7 +261,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "ffn2 gemm launch");
     }
-    if (!bk.fused_ln)
+    if (!bk.fused_ln && !(l < (int)bk.ln2_in_qkv.size() && bk.ln2_in_qkv[l]))
       ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
                                  c.ln_eps, rt->X, s),
                 "ln2 launch");
@@ -407,6 +411,27 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
     }
     if (!ok) return set_error(ARLO_ECUDA, "tensor-map encoding failed (cuTensorMapEncodeTiled unavailable?)");
   }
+  // LayerNorm prologues: LN1 of layer l into its FFN1, LN2 of layer l into layer l+1's QKV, where
+  // that GEMM is a persistent tile kernel (every CTA resident: its grid barrier needs it)
+  bk.ln1_in_f1.assign(c.layers, 0);
+  bk.ln2_in_qkv.assign(c.layers, 0);
+  // Opt-in (ARLO_LN_PROLOGUE=1): bitwise the LN kernel + GEMM, but measured slower on B200 (BERT-base
+  // L=128 b=32 0.975 -> 1.063 ms, L=64 b=32 0.683 -> 0.736 ms): the grid barrier and
+  // the grid's 1,500-2,000 warps normalising 2-3 rows each cost more than the LN kernel, whose
+  // 4,096 warps run one row each and overlap the GEMMs on either side through PDL.
+  if (!bk.fused_ln && getenv("ARLO_LN_PROLOGUE") != nullptr) {
+    for (int l = 0; l < c.layers; ++l) {
+      const bool cls_last = getenv("ARLO_NO_CLS_PRUNE") == nullptr && l == c.layers - 1;  // (CLS rows: LN kernel)
+      LnPrologue ln1{rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B), rt->X, rt->gbar,
+                     c.ln_eps, M, H};
+      if (!cls_last) bk.ln1_in_f1[l] = tc_plan_attach_ln(&bk.plans[l].f1, ln1);
+      if (l + 1 < c.layers) {
+        LnPrologue ln2{rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B), rt->X, rt->gbar,
+                       c.ln_eps, M, H};
+        bk.ln2_in_qkv[l] = tc_plan_attach_ln(&bk.plans[l + 1].qkv, ln2);
+      }
+    }
+  }
   bk.cls_prune = !bk.fused_ln && getenv("ARLO_NO_CLS_PRUNE") == nullptr;
   if (bk.cls_prune) {
     const int l = c.layers - 1, b = bk.b, L = rt->L;
@@ -487,6 +512,7 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   size_t off = al(off_ids + 4 * Mmax);
   const size_t off_logits = off; off = al(off + 4 * (size_t)max_batch * c.num_labels);
   const size_t off_pooled = off; off = al(off + 4 * (size_t)max_batch * H);
+  const size_t off_gbar = off; off = al(off + 64);
   const size_t off_X = off; off = al(off + es * Mmax * H);
   const size_t off_QKV = off; off = al(off + es * Mmax * 3 * H);
   const size_t off_O = off; off = al(off + es * Mmax * H);
@@ -502,6 +528,7 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   rt->ids = (int32_t*)(a + off_ids);
   rt->logits = (float*)(a + off_logits);
   rt->pooled = (float*)(a + off_pooled);
+  rt->gbar = (unsigned*)(a + off_gbar);
   rt->X = a + off_X; rt->QKV = a + off_QKV; rt->O = a + off_O; rt->Y = a + off_Y; rt->F = a + off_F;
   rt->h_stage_bytes = off_ids + 4 * Mmax + 4 * (size_t)max_batch * c.num_labels + 64;
   e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
@@ -670,6 +697,24 @@ extern "C" int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, cons
   } else {
     ARLO_CUDA(launch_gemm_simt(DT_FP32, M, N, K, A, W, bias, residual, out, epi, s), "simt gemm");
   }
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_ln_gemm(int32_t M, int32_t N, int32_t K, const void* y, const float* gamma,
+                               const float* beta, float eps, void* x, const void* W, const float* bias, void* out,
+                               int32_t epi, int32_t force_bn, void* barrier, void* stream) {
+  clear_error();
+  if (M < 1 || N % 64 || K % 64 || N < 64 || K < 64 || !y || !gamma || !beta || !x || !W || !bias || !out ||
+      !barrier || (epi != ARLO_EPI_BIAS && epi != ARLO_EPI_BIAS_GELU))
+    return set_error(ARLO_EINVAL, "arlo_op_ln_gemm: bad arguments");
+  TcGemmPlan p;
+  if (!tc_plan_gemm(&p, M, N, K, x, W, bias, nullptr, out, epi, force_bn))
+    return set_error(ARLO_EINVAL, "arlo_op_ln_gemm: plan failed (tile %d)", force_bn);
+  LnPrologue lnp{y, gamma, beta, x, (unsigned*)barrier, eps, M, K};
+  if (!tc_plan_attach_ln(&p, lnp))
+    return set_error(ARLO_EINVAL, "arlo_op_ln_gemm: tile %d cannot run a LayerNorm prologue (skinny / non-persistent)",
+                     force_bn);
+  ARLO_CUDA(tc_launch_gemm(p, (cudaStream_t)stream), "LayerNorm-prologue gemm");
   return ARLO_OK;
 }
 

@@ -276,3 +276,29 @@ def test_attention_packed_L64_bitwise(arlo_lib, B):
     arlo_lib.op_attention(0, B, 128, heads, bf16_dev(q128), ld, o128)
     torch.cuda.synchronize()
     assert torch.equal(o64.view(B, 64, H), o128.view(B, 128, H)[:, :64])
+
+
+@pytest.mark.parametrize("M,N,K,epi,force", [(4096, 3072, 768, 1, 0), (4096, 2304, 768, 0, -192), (300, 3072, 768, 1, 128),
+                                             (2048, 4096, 1024, 1, -256), (777, 384, 128, 0, 64), (16384, 3072, 1024, 0, 0)])
+def test_ln_prologue_gemm_bitwise(arlo_lib, M, N, K, epi, force):
+    """LayerNorm as the prologue of the consuming GEMM (one launch, grid barrier) gives bit for bit
+    the LayerNorm kernel's rows and the GEMM of those rows; repeated launches reuse the barrier."""
+    y = bf16_dev(wl.round_to_bf16(rnd((M, K), 50) * 2 + 0.5))
+    g = f32_dev(wl.round_to_bf16(rnd((K,), 51, 0.1) + 1))
+    be = f32_dev(rnd((K,), 52, 0.02))
+    W, b = bf16_dev(rnd((N, K), 53, 0.02)), f32_dev(rnd((N,), 54, 0.02))
+    x_ref = torch.empty((M, K), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_layernorm(0, y, g, be, 1e-12, x_ref)
+    o_ref = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_gemm(arlo_lib.BF16, x_ref, W, b, o_ref, epi=epi, force_bn=force)
+    bar = torch.zeros(2, dtype=torch.int32, device="cuda")
+    for _ in range(3):
+        x = torch.full((M, K), float("nan"), device="cuda", dtype=torch.bfloat16)
+        o = torch.full((M, N), float("nan"), device="cuda", dtype=torch.bfloat16)
+        arlo_lib.op_ln_gemm(y, g, be, 1e-12, x, W, b, o, epi=epi, force_bn=force, barrier=bar)
+        torch.cuda.synchronize()
+        assert torch.equal(x, x_ref)
+        assert torch.equal(o, o_ref)
+    assert bar[0].item() == 0 and bar[1].item() == 3  # arrivals reset, one generation per launch
+    ref = orc.layer_norm(host64(y), g.cpu().numpy().astype(np.float64), be.cpu().numpy().astype(np.float64), 1e-12)
+    np.testing.assert_allclose(host64(x), ref, rtol=0, atol=2e-2)

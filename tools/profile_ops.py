@@ -1,6 +1,6 @@
 """Launch one hot-path kernel at a bench shape a few times (for ncu --set full captures).
 
-    python tools/profile_ops.py gemm M N K epi      # tcgen05 GEMM (epi 0 bias, 1 gelu, 2 residual)
+    python tools/profile_ops.py gemm M N K epi [code]  # tcgen05 GEMM (epi 0 bias, 1 gelu, 2 residual; tile code)
     python tools/profile_ops.py attn B L heads len  # masked attention, all lengths = len
     python tools/profile_ops.py ln M H              # LayerNorm
     python tools/profile_ops.py embed B L           # embedding + LN (BERT-base tables)
@@ -21,14 +21,15 @@ def main():
     dev = torch.device("cuda")
     reps = 5
     if op == "gemm":
-        M, N, K, epi = a
+        M, N, K, epi = a[:4]
+        code = a[4] if len(a) > 4 else 0
         A = torch.randn(M, K, device=dev).to(torch.bfloat16)
         W = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
         b = torch.zeros(N, device=dev)
         R = torch.randn(M, N, device=dev).to(torch.bfloat16)
         out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
         for _ in range(reps):
-            arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R if epi == 2 else None)
+            arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R if epi == 2 else None, force_bn=code)
     elif op == "attn":
         B, L, heads, n = a
         qkv = torch.randn(B * L, 3 * 64 * heads, device=dev).to(torch.bfloat16)
