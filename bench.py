@@ -509,8 +509,10 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
     """Roofline of the dominant kernel.  The four GEMMs of the L=128, b=32 runtime (the bucket
     that serves the most requests, 43 %; M = 4096) are timed in the tile configuration its
     CUDA graph actually replays (rt.gemm_tiles(32), chosen by timing at runtime creation),
-    each launch bracketed by CUDA events on the launching stream with L2 flushed before it
-    (outside the events), `reps` launches averaged.  The dominant kernel is the GEMM with the
+    each launch bracketed by CUDA events on the launching stream, `reps` launches averaged.
+    Before each launch (outside the events) L2 is flushed and the activations are rewritten,
+    as in the forward: A (and the residual) were just produced by the previous kernel and sit
+    in L2, the layer's weights come from HBM.  The dominant kernel is the GEMM with the
     largest time; achieved = 2MNK / its mean launch time."""
     H, F = 768, 3072
     M = 128 * 32
@@ -527,11 +529,15 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
         bias = torch.zeros(n, device=dev)
         res = torch.randn(m, n, device=dev, generator=g).to(torch.bfloat16) if epi == arlo.EPI_BIAS_RESIDUAL else None
         out = torch.empty(m, n, device=dev, dtype=torch.bfloat16)
+        A0, R0 = A.clone(), (res.clone() if res is not None else None)
         for _ in range(3):
             arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
         ev = []
         for _ in range(reps):
             flush.zero_()
+            A.copy_(A0)  # the predecessor's output: L2-resident, the weights are not
+            if res is not None:
+                res.copy_(R0)
             a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(stream)
             arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
@@ -558,7 +564,7 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
             "achieved": round(d["tflops"], 1), "peak": peak, "unit": "TFLOP/s", "frac": round(d["frac"], 4),
             "traffic": traffic, "peak_source": src + " bf16_tflops (burst)", "launch_us": round(d["launch_us"], 2),
             "algorithmic_flops_per_launch": metrics.gemm_flops(d["M"], d["N"], d["K"]),
-            "l2": "flushed before each launch"}
+            "l2": "flushed before each launch, then A / residual rewritten (L2-resident as in the forward), W cold"}
     return roof, table
 
 

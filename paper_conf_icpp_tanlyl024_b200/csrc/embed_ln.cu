@@ -21,6 +21,9 @@ namespace {
 #define ARLO_LN_ROWS 16  // rows (warps) per CTA: 16 -> 4.08 us at M=4096 vs 4.40 (8), 4.10 (32); gpurun_out/ab23
 #endif
 constexpr int kRowsPerBlock = ARLO_LN_ROWS;  // one warp per row
+#ifndef ARLO_LN_SMEM
+#define ARLO_LN_SMEM 1  // stage gamma / beta in shared memory (A/B: 0 reads them through L1)
+#endif
 constexpr int kLnThreads = 32 * kRowsPerBlock;
 
 // gamma / beta are weights, independent of the predecessor kernel: every CTA stages them in
@@ -41,9 +44,17 @@ __global__ void __launch_bounds__(kLnThreads) layernorm_kernel(int M, int H, con
                                                         const float* __restrict__ b, float eps,
                                                         T* __restrict__ out) {
   constexpr int VN = Vec<T>::N;
+#if ARLO_LN_SMEM
   extern __shared__ float s_aff[];  // [gamma H | beta H]
   pdl_launch_dependents();
   stage_affine(H, g, b, s_aff, s_aff + H);
+  const float* ga = s_aff;
+  const float* be = s_aff + H;
+#else  // A/B: gamma / beta straight from L1/L2 (no shared memory: CTAs fit beside a GEMM's)
+  pdl_launch_dependents();
+  const float* ga = g;
+  const float* be = b;
+#endif
   pdl_wait();
   const int lane = threadIdx.x & 31;
   const int row = blockIdx.x * kRowsPerBlock + (threadIdx.x >> 5);
@@ -54,7 +65,7 @@ __global__ void __launch_bounds__(kLnThreads) layernorm_kernel(int M, int H, con
 #pragma unroll
   for (int i = 0; i < MAXV; ++i)
     if (lane + 32 * i < nvec) Vec<T>::load(src + (lane + 32 * i) * VN, v[i], true);  // predecessor's output
-  ln_finish<T, MAXV>(v, nvec, H, lane, s_aff, s_aff + H, eps, out + (size_t)row * H);
+  ln_finish<T, MAXV>(v, nvec, H, lane, ga, be, eps, out + (size_t)row * H);
 }
 
 template <typename T, int MAXV>
@@ -132,10 +143,10 @@ cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float
   const int maxv = round_maxv(H / vn);
   dim3 grid((M + kRowsPerBlock - 1) / kRowsPerBlock), block(kLnThreads);
   if (dt == DT_BF16) {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, 8 * H, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<bf16, MV>, grid, block, ARLO_LN_SMEM ? 8 * H : 0, s,
         M, H, (const bf16*)in, g, b, eps, (bf16*)out));
   } else {
-    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<float, MV>, grid, block, 8 * H, s,
+    ARLO_MAXV_SWITCH(maxv, return launch_k(layernorm_kernel<float, MV>, grid, block, ARLO_LN_SMEM ? 8 * H : 0, s,
         M, H, (const float*)in, g, b, eps, (float*)out));
   }
   return cudaGetLastError();

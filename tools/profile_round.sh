@@ -1,24 +1,29 @@
-# Round profile artifacts (run under gpurun; results land in gpurun_out/prof/):
-#   bench JSON, ncu launch list of the bench step (cold-cache, serialised: shares not absolutes),
-#   ncu --set full of the top kernels, per-kernel metric summaries.
-set -x
-mkdir -p gpurun_out/prof
+# Round profile artifacts (one gpurun call; results in gpurun_out/${1:-prof}/):
+#   bench JSON (+ extras), ncu launch list of the bench's timed steps (cold-cache, serialised: compare
+#   SHARES, not absolutes), ncu --set full of the four GEMMs of the L=128 b=32 graph in the tile codes
+#   the graph uses (from the bench extras) and of attention / LayerNorm, per-kernel metric summaries.
+out=gpurun_out/${1:-prof}
+mkdir -p $out
 python __graft_entry__.py > /dev/null
-timeout 900 python bench.py > gpurun_out/prof/bench.json 2> gpurun_out/prof/bench.err
+timeout 900 python bench.py --extras-out $out/bench_extras.json > $out/bench.json 2> $out/bench.err
 ARLO_PROFILE_TIMED=1 timeout 900 ncu --profile-from-start off --metrics gpu__time_duration.sum --clock-control none -c 3000 --csv \
-    --log-file gpurun_out/prof/launches.csv python bench.py --steps 2 --warmup 1 --no-extras --no-cpu-baseline \
-    > gpurun_out/prof/bench_under_ncu.log 2>&1
-python tools/forward_breakdown.py --summarize gpurun_out/prof/launches.csv > gpurun_out/prof/launches_summary.txt 2>&1
+    --log-file $out/launches.csv python bench.py --steps 2 --warmup 1 --no-extras --no-cpu-baseline \
+    > $out/bench_under_ncu.log 2>&1
+python tools/forward_breakdown.py --summarize $out/launches.csv > $out/launches_summary.txt 2>&1
 full() {  # name, kernel regex, command...
   name=$1; shift; k=$1; shift
   timeout 600 ncu --set full --clock-control none --import-source on -k regex:$k -s 2 -c 1 \
-      -o gpurun_out/prof/$name "$@" > gpurun_out/prof/$name.log 2>&1
+      -o $out/$name "$@" > $out/$name.log 2>&1
 }
-full ffn1_gemm gemm_tc_pair python tools/profile_ops.py gemm 4096 3072 768 1
-full ffn1_gemm_large gemm_tc_pair python tools/profile_ops.py gemm 32768 4096 1024 1
-full skinny_gemm gemm_skinny python tools/profile_ops.py gemm 64 768 3072 0
+codes=$(python -c "import json; d=json.load(open('$out/bench_extras.json'))['gemm_tiles']['128']['32']; print(*d)")
+set -- $codes
+full qkv_L128b32 gemm python tools/profile_ops.py gemm 4096 2304 768 0 $1
+full out_L128b32 gemm python tools/profile_ops.py gemm 4096 768 768 2 $2
+full ffn1_L128b32 gemm python tools/profile_ops.py gemm 4096 3072 768 1 $3
+full ffn2_L128b32 gemm python tools/profile_ops.py gemm 4096 768 3072 2 $4
+full ffn1_large gemm_tc_pair python tools/profile_ops.py gemm 32768 4096 1024 1
+full attn_l64 attn_tc python tools/profile_ops.py attn 32 64 12 64
 full attn_l128 attn_tc python tools/profile_ops.py attn 32 128 12 128
 full attn_l512 attn_tc python tools/profile_ops.py attn 64 512 16 512
 full layernorm layernorm python tools/profile_ops.py ln 4096 768
-full embed embed_ln python tools/profile_ops.py embed 32 128
-full pooler pooler python tools/profile_ops.py head 32 128
+python tools/ncu_summary.py $out/*.ncu-rep > $out/ncu_summary.txt 2>&1
