@@ -121,7 +121,18 @@ int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arl
  * ~87 dependent kernels (~4.5 us each), not by the GEMMs, and the latency family measured
  * no faster.  fp32 check mode ignores the family (SIMT GEMMs).
  */
-enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHPUT = 2 };
+enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHPUT = 2, ARLO_RUNTIME_FUSED = 3 };
+/*
+ * ARLO_RUNTIME_FUSED: the whole forward (embedding .. logits) as ONE persistent kernel of one
+ * CTA per SM running a static task graph (GEMM units, attention per (sequence, head),
+ * LayerNorm row groups, head), tasks waiting on per-step completion counters instead of
+ * kernel boundaries; weights stream ahead of the dependency chain (the
+ * batch-1 setting of PAPER.md:L282 §5).  Needs bf16, max_batch*L <= 256, L <= 128, hidden and
+ * ffn multiples of 128, hidden <= 1024 (EINVAL otherwise).  GEMM units split K by a factor of
+ * the weight shape only, so within the family a request's logits are bitwise equal on every
+ * runtime L >= its length and in every bucket; against the other families they agree to
+ * bf16 rounding.  arlo_runtime_gemm_tiles reports 3000 + the split factor of each GEMM.
+ */
 int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_weights* w, int32_t family,
                            arlo_runtime** out);
 /* ARLO_RUNTIME_LATENCY or ARLO_RUNTIME_THROUGHPUT (the family the runtime was built as). */

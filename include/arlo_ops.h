@@ -106,6 +106,11 @@ int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K);
 int arlo_debug_gemm_trace(void* buf);
 /* Same for the bf16 attention kernel: >= 64 * 2048 uint64 entries. */
 int arlo_debug_attn_trace(void* buf);
+/* Same for the fused persistent forward (ARLO_RUNTIME_FUSED): >= 6 uint64 per task of the
+ * plan (the task array in CTA order); stamps per task: [type | layer << 8 | a << 24 | b << 40 |
+ * cta << 52, compute begin, ready (dependency met / accumulator full), end (after its completion
+ * signal), producer dependency met (GEMM units), 0] in %globaltimer ns (tools/fused_trace.py). */
+int arlo_debug_fused_trace(void* buf);
 
 #ifdef __cplusplus
 }

@@ -28,8 +28,8 @@ OK, EINVAL, ETOOLONG, ENOMEM, ECUDA, EINFEASIBLE, ENOCAND, ENODEV = 0, -1, -2, -
 BF16, FP32 = 0, 1
 DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
-RUNTIME_DEFAULT, RUNTIME_LATENCY, RUNTIME_THROUGHPUT = 0, 1, 2
-SKINNY_CODE, SPLITK_CODE = 1000, 2000  # tile codes: kSkinnyCode + BN, kSplitKCode + BN
+RUNTIME_DEFAULT, RUNTIME_LATENCY, RUNTIME_THROUGHPUT, RUNTIME_FUSED = 0, 1, 2, 3
+SKINNY_CODE, SPLITK_CODE, FUSED_CODE = 1000, 2000, 3000  # tile codes: kSkinnyCode + BN, kSplitKCode + BN, kFusedCode + S
 
 EXPORTED = [
     "arlo_replace_plan", "arlo_runtime_gemm_tiles",
@@ -38,7 +38,7 @@ EXPORTED = [
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_sched_set_policy", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
     "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_ln_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
-    "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_gemm_tile_choice",
+    "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_debug_fused_trace", "arlo_gemm_tile_choice",
 ]
 
 
@@ -93,6 +93,7 @@ _sig("arlo_op_embed", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp,
 _sig("arlo_op_attention", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp)
 _sig("arlo_debug_gemm_trace", C.c_int, _vp)
 _sig("arlo_debug_attn_trace", C.c_int, _vp)
+_sig("arlo_debug_fused_trace", C.c_int, _vp)
 _sig("arlo_gemm_tile_choice", _i32, _i32, _i32, _i32)
 _sig("arlo_op_head", C.c_int, _i32, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _vp, _vp)
 

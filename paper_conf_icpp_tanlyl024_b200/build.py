@@ -24,7 +24,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 BUILD = os.path.join(PKG, "build")
 LIB = os.path.join(PKG, "libarlo.so")
-SOURCES = ["embed_ln.cu", "gemm_simt.cu", "gemm_tc.cu", "gemm_splitk.cu", "attention.cu", "head.cu", "runtime.cu", "sched.cpp"]
+SOURCES = ["embed_ln.cu", "gemm_simt.cu", "gemm_tc.cu", "gemm_splitk.cu", "encoder_fused.cu", "attention.cu", "head.cu", "runtime.cu", "sched.cpp"]
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 
 

@@ -1136,6 +1136,23 @@ bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint
   return r == CUDA_SUCCESS;
 }
 
+// 3-D bf16 map {inner, mid, outer} with packed strides (mid stride = inner, outer stride =
+// inner * mid elements): tile-contiguous activations [tiles][rows][inner] (encoder_fused.cu).
+bool encode_tmap_bf16_3d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t mid, uint64_t outer,
+                         uint32_t box_inner, uint32_t box_mid, int swizzle_bytes) {
+  EncodeTiledFn fn = get_encode_fn();
+  if (!fn) return false;
+  cuuint64_t dims[3] = {inner, mid, outer};
+  cuuint64_t strides[2] = {inner * 2, inner * mid * 2};
+  cuuint32_t box[3] = {box_inner, box_mid, 1};
+  cuuint32_t estr[3] = {1, 1, 1};
+  CUresult r = fn(tm, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 3, const_cast<void*>(base), dims, strides, box, estr,
+                  CU_TENSOR_MAP_INTERLEAVE_NONE,
+                  swizzle_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
+                  CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 // Tile choice: a function of (M, N, K) only (never of the data), minimising a
 // wave-quantised time estimate fitted to graph-replayed B200 sweeps
 // (tools/gemm_sweep.py --set small/base/large/mid: over 39 shapes the pick is

@@ -77,6 +77,7 @@ cudaError_t tc_launch_gemm(const TcGemmPlan& p, cudaStream_t s);
 // Tile choice codes: BN (single CTA), -BN (CTA pair), kSkinnyCode + BN (skinny kernel).
 constexpr int kSkinnyCode = 1000;
 constexpr int kSplitKCode = 2000;  // kSplitKCode + BN: split-K kernel (splitk_factor(N, K) splits)
+constexpr int kFusedCode = 3000;   // kFusedCode + split factor: unit of the fused persistent forward
 int tc_choose_bn(int M, int N, int K);
 // out = LN(A W^T + bias + resid; gamma, beta, eps), N = hidden size (128 / 768 / 1024 ...).
 // `out` may alias `resid` (each tile reads its residual before storing the same region).
@@ -115,9 +116,23 @@ cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, con
                         const float* b_p, const void* w_c, const float* b_c, float* pooled,
                         float* logits, cudaStream_t s);
 
+// ---- fused persistent forward (encoder_fused.cu): the whole batch-1 forward as one kernel ----
+struct FusedPlanImpl;
+bool fused_supported(int B, int L, int H, int heads, int F);
+int fused_split(int N, int K);  // split-K factor of the fused family's GEMM units (weight shape only)
+// t = the canonical weight tensors of arlo_weights_create; nullptr if unsupported / allocation failed
+FusedPlanImpl* fused_create(int B, int L, int layers, int H, int heads, int F, int C, int vocab, float eps,
+                            const void* const* t, const int32_t* ids, const int32_t* lengths, int32_t* err, void* X,
+                            void* X1, void* QKV, void* CTX, void* HB, float* pooled, float* logits);
+cudaError_t fused_launch(const FusedPlanImpl* p, cudaStream_t s);
+void fused_destroy(FusedPlanImpl* p);
+cudaError_t set_fused_trace(unsigned long long* buf);  // profiling hook, nullptr = off
+
 // Resolve cuTensorMapEncodeTiled through the runtime (no link-time libcuda dependency).
 // row_elems = row stride in elements (0: rows are contiguous, stride = inner).
 bool encode_tmap_bf16_2d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t outer,
                          uint32_t box_inner, uint32_t box_outer, int swizzle_bytes, uint64_t row_elems = 0);
+bool encode_tmap_bf16_3d(CUtensorMap* tm, const void* base, uint64_t inner, uint64_t mid, uint64_t outer,
+                         uint32_t box_inner, uint32_t box_mid, int swizzle_bytes);
 
 }  // namespace arlo

@@ -173,6 +173,7 @@ struct Bucket {
   bool cls_prune = false;
   LayerPlans cls;
   AttnPlan attn_cls;
+  FusedPlanImpl* fused = nullptr;  // fused family: the whole forward as one persistent kernel
   cudaGraphExec_t exec = nullptr;
   size_t nodes = 0;
 };
@@ -182,6 +183,8 @@ struct arlo_runtime {
   // latency family (ARLO_RUNTIME_LATENCY): every GEMM is the split-K weight-streaming kernel
   // (gemm_splitk.cu); the throughput family uses the tile kernels chosen per bucket
   bool latency = false;
+  // fused family (ARLO_RUNTIME_FUSED): one persistent kernel per forward (encoder_fused.cu)
+  bool fused = false;
   const arlo_weights* w = nullptr;
   DType dt = DT_BF16;
   cudaStream_t own_stream = nullptr, stream = nullptr;
@@ -212,6 +215,10 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
   const arlo_model_config& c = w->cfg;
   const int b = bk.b, L = rt->L, H = c.hidden, F = c.ffn, M = b * L;
   const DType dt = rt->dt;
+  if (rt->fused) {
+    ARLO_CUDA(fused_launch(bk.fused, s), "fused forward launch");
+    return ARLO_OK;
+  }
   ARLO_CUDA(launch_embed_ln(dt, b, L, H, c.vocab, rt->ids, rt->lengths, w->word(), w->pos(), w->type(), w->emb_g(),
                             w->emb_b(), c.ln_eps, rt->X, rt->err, s),
             "embed_ln launch");
@@ -452,8 +459,10 @@ static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
 
 static void destroy_runtime(arlo_runtime* rt) {
   if (!rt) return;
-  for (auto& bk : rt->buckets)
+  for (auto& bk : rt->buckets) {
     if (bk.exec) cudaGraphExecDestroy(bk.exec);
+    fused_destroy(bk.fused);
+  }
   if (rt->arena) cudaFree(rt->arena);
   if (rt->h_stage) cudaFreeHost(rt->h_stage);
   if (rt->own_stream) cudaStreamDestroy(rt->own_stream);
@@ -473,19 +482,27 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
 }
 
 extern "C" int32_t arlo_runtime_family(const arlo_runtime* rt) {
-  return rt ? (rt->latency ? ARLO_RUNTIME_LATENCY : ARLO_RUNTIME_THROUGHPUT) : ARLO_EINVAL;
+  return rt ? (rt->fused ? (int32_t)ARLO_RUNTIME_FUSED : rt->latency ? (int32_t)ARLO_RUNTIME_LATENCY : (int32_t)ARLO_RUNTIME_THROUGHPUT)
+            : ARLO_EINVAL;
 }
 
 extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_weights* w, int32_t family,
                                       arlo_runtime** out) {
   clear_error();
   if (!w || !out) return set_error(ARLO_EINVAL, "arlo_runtime_create: null argument");
-  if (family != ARLO_RUNTIME_DEFAULT && family != ARLO_RUNTIME_LATENCY && family != ARLO_RUNTIME_THROUGHPUT)
+  if (family != ARLO_RUNTIME_DEFAULT && family != ARLO_RUNTIME_LATENCY && family != ARLO_RUNTIME_THROUGHPUT &&
+      family != ARLO_RUNTIME_FUSED)
     return set_error(ARLO_EINVAL, "arlo_runtime_create_ex: unknown runtime family %d", family);
   const arlo_model_config& c = w->cfg;
   if (L < 16 || L % 16 || L > c.max_pos)
     return set_error(ARLO_EINVAL, "arlo_runtime_create: need 16 <= L <= max_pos (%d) and L %% 16 == 0, got %d", c.max_pos, L);
   if (max_batch < 1 || max_batch > 64) return set_error(ARLO_EINVAL, "arlo_runtime_create: need 1 <= max_batch <= 64");
+  if (family == ARLO_RUNTIME_FUSED &&
+      (c.dtype != ARLO_BF16 || !fused_supported(max_batch, L, c.hidden, c.heads, c.ffn)))
+    return set_error(ARLO_EINVAL,
+                     "arlo_runtime_create_ex: the fused family needs bf16, max_batch*L <= 256, L <= 128, "
+                     "hidden and ffn multiples of 128, hidden <= 1024 (got L=%d max_batch=%d H=%d F=%d)",
+                     L, max_batch, c.hidden, c.ffn);
   DeviceGuard g(w->device);
   arlo_runtime* rt = new (std::nothrow) arlo_runtime;
   if (!rt) return set_error(ARLO_ENOMEM, "out of host memory");
@@ -498,6 +515,7 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   // (DEFAULT = THROUGHPUT: measured on B200, the split-K family does not shorten a batch-1 forward;
   // its 87 dependent kernels cost ~4.5 us each whatever the GEMM kernel)
   rt->latency = rt->dt == DT_BF16 && family == ARLO_RUNTIME_LATENCY;
+  rt->fused = family == ARLO_RUNTIME_FUSED;
   auto fail = [&](int code) { destroy_runtime(rt); return code; };
   cudaError_t e = cudaStreamCreateWithFlags(&rt->own_stream, cudaStreamNonBlocking);
   if (e != cudaSuccess) return fail(cuda_fail(e, "cudaStreamCreate"));
@@ -546,7 +564,14 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
     bk.b = bs[i];
     if (!attn_plan(&bk.attn, rt->dt, bk.b, L, c.heads, rt->QKV))
       return fail(set_error(ARLO_EINVAL, "attention plan failed (bf16 attention needs L <= 512)"));
-    if (rt->dt == DT_BF16) {
+    if (rt->fused) {
+      bk.fused = fused_create(bk.b, L, c.layers, c.hidden, c.heads, c.ffn, c.num_labels, c.vocab, c.ln_eps,
+                              w->t.data(), rt->ids, rt->lengths, rt->err, rt->X, rt->Y, rt->QKV, rt->O, rt->F,
+                              rt->pooled, rt->logits);
+      if (!bk.fused) return fail(set_error(ARLO_ECUDA, "fused forward plan failed (tensor maps / device memory)"));
+      bk.tiles[0] = kFusedCode + 1; bk.tiles[1] = kFusedCode + fused_split(c.hidden, c.hidden);
+      bk.tiles[2] = kFusedCode + 1; bk.tiles[3] = kFusedCode + fused_split(c.hidden, c.ffn);
+    } else if (rt->dt == DT_BF16) {
       int rc = plan_bucket(rt, bk);
       if (rc) return fail(rc);
     }
@@ -770,6 +795,11 @@ extern "C" int arlo_debug_gemm_trace(void* buf) {
 extern "C" int32_t arlo_gemm_tile_choice(int32_t M, int32_t N, int32_t K) {
   if (M < 1 || N % 64 || K % 64 || N < 64 || K < 64) return 0;
   return tc_choose_bn(M, N, K);
+}
+
+extern "C" int arlo_debug_fused_trace(void* buf) {
+  cudaError_t e = set_fused_trace((unsigned long long*)buf);
+  return e == cudaSuccess ? ARLO_OK : cuda_fail(e, "arlo_debug_fused_trace");
 }
 
 extern "C" int arlo_debug_attn_trace(void* buf) {

@@ -1,10 +1,10 @@
 """Batch-1 latency of the two runtime families and the split-K GEMMs at small M.
 
-    python tools/latency_bench.py [bert-base|bert-large] > gpurun_out/latency.json
+    python tools/latency_bench.py [bert-base|bert-large] [families,...] > gpurun_out/latency.json
 
 Per runtime L: median of 50 graph replays (CUDA events per replay) of a b = 1 forward in
-the latency family (split-K weight streaming) and the throughput family (bucket 1 of a
-max_batch = 32 runtime).  Per GEMM shape at M = 64: the split-K kernel vs the skinny /
+the latency family (split-K weight streaming), the throughput family (bucket 1 of a
+max_batch = 32 runtime) and, at L <= 128, the fused family (one persistent kernel).  Per GEMM shape at M = 64: the split-K kernel vs the skinny /
 tile kernel the chooser picks, as weight-streaming bandwidth (weight bytes / time) with
 the weights cold (L2 flushed before each launch) and the activations warm.
 """
@@ -71,8 +71,13 @@ def main():
     out = {"config": name, "forward_ms": {}, "gemm_M64": {}}
     for L in ((64, 128, 256, 512) if name == "bert-base" else (128, 256, 512)):
         row = {}
-        for fam, mb in (("latency", 1), ("throughput", 32)):
-            rt = arlo.Runtime(W, L, mb, arlo.RUNTIME_LATENCY if fam == "latency" else arlo.RUNTIME_THROUGHPUT)
+        fams = [("latency", 1, arlo.RUNTIME_LATENCY), ("throughput", 32, arlo.RUNTIME_THROUGHPUT)]
+        if L <= 128:
+            fams.append(("fused", 1, arlo.RUNTIME_FUSED))
+        if len(sys.argv) > 2:
+            fams = [f for f in fams if f[0] in sys.argv[2].split(",")]
+        for fam, mb, code in fams:
+            rt = arlo.Runtime(W, L, mb, code)
             rt.set_stream(stream)
             row[fam] = time_forward(rt, cfg, L, 1, stream)
             row[fam + "_tiles"] = rt.gemm_tiles(1)

@@ -27,3 +27,5 @@ full attn_l128 attn_tc python tools/profile_ops.py attn 32 128 12 128
 full attn_l512 attn_tc python tools/profile_ops.py attn 64 512 16 512
 full layernorm layernorm python tools/profile_ops.py ln 4096 768
 python tools/ncu_summary.py $out/*.ncu-rep > $out/ncu_summary.txt 2>&1
+# keep the pulled-back directory small (gpurun merges <= 64 MiB): the reports stay on the box
+mkdir -p /tmp/ncu_reps && mv $out/*.ncu-rep /tmp/ncu_reps/ 2>/dev/null
