@@ -1,7 +1,8 @@
 """Time the tcgen05 GEMM at several shapes / tile choices with CUDA events (warm L2).
 
     python tools/gemm_sweep.py [--epi E] [--set base|large|small|all] [force ...]
-        force: 0 auto, 64/128/192/256 single CTA, -128/-192/-256 CTA pair
+        force: 0 auto, 64/128/192/256 single CTA, -128/-192/-256 CTA pair, 4064/4096/4128 dual
+        (single-CTA tiles, two CTAs per SM)
         epi:   0 bias, 1 bias+GELU, 2 bias+residual
 """
 import argparse
@@ -72,7 +73,8 @@ def main():
         line = f"{M:6d} {N:5d} {K:5d} choice={arlo.gemm_tile_choice(M, N, K):5d}:"
         fl = 2.0 * M * N * K
         for f in forces:
-            if N % (f - 1000 if f > 1000 else abs(f or 64)):
+            bn = f - 4000 if f > 4000 else f - 1000 if f > 1000 else abs(f or 64)
+            if N % bn:
                 line += f"  {f:5d}=   n/a  "
                 continue
             t = time_op(lambda st: arlo.op_gemm(arlo.BF16, A, W, b, out, epi=a.epi, residual=R, force_bn=f, stream=st))
