@@ -50,7 +50,16 @@ constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 stagi
 #define ARLO_STG_BUFS 2
 #endif
 constexpr int kStgBufs = ARLO_STG_BUFS;         // staging tiles per epilogue warp (TMA stores in flight)
-constexpr int kStagingBytes = kEpiWarps * kStgBufs * kStgBytes;
+// Per epilogue warp: kStgBufs output staging tiles, then the bias of the warp's chunks of the
+// current tile (32 fp32 per chunk, <= 4 chunks), staged before the accumulator wait so that the
+// epilogue math reads bias from shared memory, not from L2 (a cold __ldg per chunk cost ~400
+// cycles of the ~1100-cycle chunk: tools/gemm_trace.py sub-stamps, profiles/r02_gemm_sweep.txt).
+#ifndef ARLO_BIAS_SMEM
+#define ARLO_BIAS_SMEM 1  // A/B hook: 0 reads bias with __ldg inside the chunk loop
+#endif
+constexpr int kBiasWarpBytes = ARLO_BIAS_SMEM ? 4 * 32 * 4 : 0;
+constexpr int kWarpStg = kStgBufs * kStgBytes + kBiasWarpBytes;
+constexpr int kStagingBytes = kEpiWarps * kWarpStg;
 
 // Warp-role layout of the persistent kernels for EW epilogue warps (EW / 4 column groups per
 // TMEM lane quarter), then the TMA producer and the MMA warp.  EW = 8 by default; the
@@ -62,7 +71,7 @@ template <int EW>
 struct Roles {
   static_assert(EW % 4 == 0, "epilogue warps cover the four TMEM lane quarters");
   static constexpr int kEpi = EW, kGroups = EW / 4, kProducer = EW, kMma = EW + 1, kThreads = 32 * (EW + 2);
-  static constexpr int kStaging = EW * kStgBufs * kStgBytes;
+  static constexpr int kStaging = EW * kWarpStg;
 };
 constexpr int kSmemBudget = 229376;            // 224 KB of the 227 KB opt-in maximum
 
@@ -77,6 +86,10 @@ __device__ __forceinline__ unsigned long long gtimer() {
 }
 __device__ __forceinline__ void trace(int slot) {
   if (g_trace != nullptr && slot < 64) g_trace[blockIdx.x * 64 + slot] = gtimer();
+}
+// clock64 sub-stamps of the epilogue of a CTA's first tile (warp 0, lane 0): slots 32..63
+__device__ __forceinline__ void trace_clk(int slot) {
+  if (g_trace != nullptr && slot < 64) g_trace[blockIdx.x * 64 + slot] = clock64();
 }
 
 // Tile rasterisation of the persistent kernels: N fastest.  The CTAs (pairs) running at
@@ -106,9 +119,21 @@ constexpr int tmem_cols_for(int n) {
 // PAIR = false: one CTA computes a 128 x BN tile; PAIR = true: a CTA pair
 // (cluster of 2, cta_group::2) computes a 256 x BN tile, each CTA holding 128
 // rows of A, BN/2 rows of W and its 128 x BN half of the accumulator.
-template <int BN, bool PAIR, int RESERVE = 0, int EW = kEpiWarps>
+// Residual epilogue (EPI_BIAS_RESID, ARLO_RESID_TMA): the producer TMA-loads the CTA's 128 x BN
+// residual tile into shared memory ({32 columns x 128 rows} boxes, 64-byte swizzle = the output
+// staging layout) while the main loop runs; the epilogue reads the residual from there, writes the
+// bf16 result in place and TMA-stores it from the same buffer.  The residual's L2 round trip left
+// the critical path of the epilogue (it cost ~1000-1300 of a ~1800-cycle chunk, gemm_trace
+// sub-stamps) and the per-warp output staging tiles are not needed.
+#ifndef ARLO_RESID_TMA
+#define ARLO_RESID_TMA 1
+#endif
+template <int BN>
+constexpr int resid_buf_bytes() { return BN * 128 * 2; }
+
+template <int BN, bool PAIR, int RESERVE = 0, int EW = kEpiWarps, bool RESID_BUF = false>
 struct TcCfg {
-  static constexpr int kStagingBytes = Roles<EW>::kStaging;
+  static constexpr int kStagingBytes = RESID_BUF ? EW * kBiasWarpBytes + resid_buf_bytes<BN>() : Roles<EW>::kStaging;
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
   static constexpr int B_BYTES = B_ROWS * BK * 2;
@@ -116,7 +141,7 @@ struct TcCfg {
   static constexpr int STAGES_FIT = (kSmemBudget - kStagingBytes - RESERVE) / STAGE_BYTES;
   static constexpr int STAGES = STAGES_FIT > 8 ? 8 : STAGES_FIT;
   static constexpr int TMEM_COLS = tmem_cols_for(kAccStages * BN);
-  static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages) + 16;
+  static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 * kAccStages + 2) + 16;
   static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + kStagingBytes + BAR_BYTES + RESERVE;
   static_assert(SMEM <= 232448, "shared memory budget");
 };
@@ -149,12 +174,30 @@ __device__ __forceinline__ void prefetch_first_resid(uint4 (&rv)[CW / 8], const 
   for (int j = 0; j < CW / 8; ++j) rv[j] = ld_dep_v4(res4 + j);
 }
 
+// Bias of this warp's chunks cg, cg + G, ... of the tile at column n0 -> the warp's bias slots
+// (lane j writes column 32 c + j; the math then reads float4 broadcasts).  Called before the
+// accumulator wait; the warp's previous tile has finished reading the slots.
+template <int BN, int kEpiGroups>
+__device__ __forceinline__ void stage_bias(float* sbias, const float* __restrict__ bias, int n0, int cg, int lane) {
+  constexpr int NCH = BN / CW;
+  constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;
+  static_assert(!ARLO_BIAS_SMEM || NCMAX * CW * 4 <= kBiasWarpBytes, "bias slots");
+  if (!ARLO_BIAS_SMEM) return;
+#pragma unroll
+  for (int k = 0; k < NCMAX; ++k) {
+    const int c = cg + k * kEpiGroups;
+    if (c < NCH) sbias[k * CW + lane] = __ldg(bias + n0 + c * CW + lane);
+  }
+  __syncwarp();
+}
+
 template <int BN, int EPI, int kEpiGroups, typename Release>
 __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int lane, int row0, int n0, int M,
                                               int ldr, const float* __restrict__ bias,
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
                                               uint8_t* stg, int& sc, Release release, bf16* __restrict__ outp,
-                                              int N, const uint4* rv_first) {
+                                              int N, const uint4* rv_first, uint8_t* rbuf = nullptr,
+                                              const float* sbias = nullptr) {
   static_assert(BN % CW == 0, "tile width must be a multiple of 32");
   constexpr int NCH = BN / CW;                                 // chunks per row block
   constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;  // chunks per warp (max)
@@ -170,31 +213,45 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
     if (lane == 0) release();
     return;
   }
+  const bool stamp = threadIdx.x == 0 && g_trace != nullptr && sc < 64;  // (sc: chunks stored so far)
+  const bool first_tile = sc == 0;
+  if (stamp && first_tile) trace_clk(32);
   uint32_t r[2][CW];
   uint4 rv[2][RV];
-  if (EPI == EPI_BIAS_RESID && row_ok) {  // prefetched by the caller before the accumulator wait
+  const bool rsm = rbuf != nullptr;  // residual tile in shared memory (TMA-prefetched), output in place
+  if (EPI == EPI_BIAS_RESID && row_ok && !rsm) {  // prefetched by the caller before the accumulator wait
 #pragma unroll
     for (int j = 0; j < RV; ++j) rv[0][j] = rv_first[j];
   }
   ptx::tmem_ld_32x32b_x32(t_row + cg * CW, r[0]);
   ptx::tmem_wait_ld();
+  if (stamp && first_tile) trace_clk(33);
 #pragma unroll
   for (int k = 0; k < NCMAX; ++k) {
     if (k >= nc) break;
     const int c = cg + k * kEpiGroups;  // chunk index within the tile
     const int cur = k & 1, nxt = cur ^ 1;
+    if (stamp && first_tile && k < 6) trace_clk(34 + 5 * k);
+    // this chunk's 32 rows x 32 columns in the residual buffer (64-byte rows, 64B swizzle)
+    uint8_t* rchunk = rsm ? rbuf + c * (BM * CW * 2) + q * (32 * CW * 2) : nullptr;
+    if (EPI == EPI_BIAS_RESID && rsm) {
+#pragma unroll
+      for (int j = 0; j < RV; ++j)
+        rv[cur][j] = *reinterpret_cast<const uint4*>(rchunk + lane * (CW * 2) + ((j ^ ((lane >> 1) & 3)) * 16));
+    }
     if (k + 1 < nc) {
       ptx::tmem_ld_32x32b_x32(t_row + (c + kEpiGroups) * CW, r[nxt]);
-      if (EPI == EPI_BIAS_RESID && row_ok) {
+      if (EPI == EPI_BIAS_RESID && row_ok && !rsm) {
 #pragma unroll
         for (int j = 0; j < RV; ++j) rv[nxt][j] = ld_dep_v4(res4 + (c + kEpiGroups) * RV + j);
       }
     }
-    const float4* bias4 = reinterpret_cast<const float4*>(bias + n0 + c * CW);
+    const float4* bias4 = ARLO_BIAS_SMEM ? reinterpret_cast<const float4*>(sbias) + k * (CW / 4)
+                                         : reinterpret_cast<const float4*>(bias + n0 + c * CW);
     uint32_t pk[CW / 2];
 #pragma unroll
     for (int j = 0; j < CW / 4; ++j) {
-      const float4 b4 = __ldg(bias4 + j);
+      const float4 b4 = ARLO_BIAS_SMEM ? bias4[j] : __ldg(bias4 + j);
       uint32_t ua = 0, ub = 0;
       if (EPI == EPI_BIAS_RESID) {
         const uint4 u = rv[cur][j >> 1];
@@ -217,12 +274,15 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       }
       continue;
     }
+    if (stamp && first_tile && k < 6) trace_clk(35 + 5 * k);
     // staging buffer sc % kStgBufs was last used kStgBufs chunks ago: make sure its TMA store has read it
-    uint8_t* buf = stg + (sc % kStgBufs) * kStgBytes;
-    if (sc >= kStgBufs) {
+    // (the residual epilogue stores in place from the residual buffer instead)
+    uint8_t* buf = rsm ? rchunk : stg + (sc % kStgBufs) * kStgBytes;
+    if (!rsm && sc >= kStgBufs) {
       if (lane == 0) ptx::bulk_wait_read<kStgBufs - 1>();
       __syncwarp();
     }
+    if (stamp && first_tile && k < 6) trace_clk(36 + 5 * k);
 #pragma unroll
     for (int j = 0; j < CW / 8; ++j) {
       // TMA 64B swizzle of a 64-byte row: 16-byte chunk index ^= address bits [7:8]
@@ -237,7 +297,9 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       ptx::bulk_commit();
     }
     ++sc;
+    if (stamp && first_tile && k < 6) trace_clk(37 + 5 * k);
     ptx::tmem_wait_ld();
+    if (stamp && first_tile && k < 6) trace_clk(38 + 5 * k);
     if (k == (nc >= 2 ? nc - 2 : 0)) {  // the last TMEM load of this warp has completed
       ptx::tc_fence_before();
       __syncwarp();
@@ -249,22 +311,27 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
 template <int BN, int EPI, int EW>
 __global__ void __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-               const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
+               const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR, int M, int N, int K,
+               const float* __restrict__ bias,
                const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
-  using C = TcCfg<BN, false, 0, EW>;
+  constexpr bool kResidBuf = ARLO_RESID_TMA && EPI == EPI_BIAS_RESID;
+  using C = TcCfg<BN, false, 0, EW, kResidBuf>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
-  constexpr int kStagingBytes = R::kStaging;
+  constexpr int kStagingBytes = C::kStagingBytes;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
+  uint8_t* rbuf = sStg + kEpiWarps * kBiasWarpBytes;  // (kResidBuf) the CTA's 128 x BN residual tile
   uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kAccStages);
+  uint64_t* rfull = tempty + kAccStages;  // residual tile landed (producer: expect_tx + TMA)
+  uint64_t* rfree = rfull + 1;            // residual buffer read and stored from (one arrive per epilogue warp)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rfree + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int num_m = (M + BM - 1) / BM;
@@ -284,6 +351,9 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], kEpiWarps);  // one arrive per epilogue warp
     }
+    ptx::mbar_init(rfull, 1);
+    ptx::mbar_init(rfree, kEpiWarps);
+    if (kResidBuf) ptx::tma_prefetch_desc(&tmR);
     ptx::fence_mbar_init();
   }
   if (warp == kMmaWarp) ptx::tmem_alloc(tmem_slot, C::TMEM_COLS);
@@ -321,6 +391,15 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
         const int m0 = tile_m(tile, num_m, num_n) * BM, n0 = tile_n(tile, num_m, num_n) * BN;
         trace(2 + 6 * it);
+        // residual tile: issued as soon as the previous tile's epilogue has freed the buffer (polled
+        // between k-blocks so the main loop never waits for it), at the latest after the last k-block
+        bool r_issued = !kResidBuf;
+        auto issue_resid = [&]() {
+          ptx::mbar_arrive_expect_tx(rfull, (uint32_t)resid_buf_bytes<BN>());
+          for (int c = 0; c < BN / CW; ++c)
+            ptx::tma_load_2d(rbuf + c * (BM * CW * 2), &tmR, rfull, n0 + c * CW, m0);
+          r_issued = true;
+        };
         for (int kb = 0; kb < kblocks; ++kb) {
           if (it == 0 && kb < pre) {
             ptx::tma_load_2d(sA + stage * C::A_BYTES, &tmA, &full[stage], kb * BK, m0);
@@ -331,6 +410,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             ptx::tma_load_2d(sB + stage * C::B_BYTES, &tmB, &full[stage], kb * BK, n0);
           }
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+          if (!r_issued && (it == 0 || ptx::mbar_test(rfree, (it - 1) & 1))) issue_resid();
+        }
+        if (!r_issued) {
+          ptx::mbar_wait(rfree, (it - 1) & 1);
+          issue_resid();
         }
       }
     } else {
@@ -376,7 +460,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     // two warps sharing a quarter take one column half each.
     pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
+    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * kWarpStg;
+    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kBiasWarpBytes : stg + kStgBufs * kStgBytes);
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -384,13 +469,21 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     for (int tile = blockIdx.x; tile < tiles; tile += gridDim.x, ++it) {
       const int m0 = tile_m(tile, num_m, num_n) * BM, n0 = tile_n(tile, num_m, num_n) * BN;
       uint4 rv0[CW / 8];
-      prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
+      if (!kResidBuf) prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
+      stage_bias<BN, kEpiGroups>(sbias, bias, n0, cg, lane);
       ptx::mbar_wait(&tfull[acc], acc_phase);
+      if (kResidBuf) ptx::mbar_wait(rfull, it & 1);  // this tile's residual has landed
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       uint64_t* te = &tempty[acc];
       epilogue_tile<BN, EPI, kEpiGroups>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid,
-                                         &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N, rv0);
+                                         &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N, rv0,
+                                         kResidBuf ? rbuf : nullptr, sbias);
+      if (kResidBuf) {  // the buffer is free once this warp's in-place TMA stores have read it
+        if (lane == 0) ptx::bulk_wait_read<0>();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(rfree);
+      }
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -416,22 +509,27 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 template <int BN, int EPI, int EW>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                    const __grid_constant__ CUtensorMap tmC, int M, int N, int K, const float* __restrict__ bias,
+                    const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR, int M, int N,
+                    int K, const float* __restrict__ bias,
                     const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
-  using C = TcCfg<BN, true, 0, EW>;
+  constexpr bool kResidBuf = ARLO_RESID_TMA && EPI == EPI_BIAS_RESID;
+  using C = TcCfg<BN, true, 0, EW, kResidBuf>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
-  constexpr int kStagingBytes = R::kStaging;
+  constexpr int kStagingBytes = C::kStagingBytes;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
+  uint8_t* rbuf = sStg + kEpiWarps * kBiasWarpBytes;  // (kResidBuf) this CTA's 128 x BN residual rows
   uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
   uint64_t* tempty = tfull + kAccStages;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + kAccStages);
+  uint64_t* rfull = tempty + kAccStages;  // (local to each CTA of the pair)
+  uint64_t* rfree = rfull + 1;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(rfree + 1);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const uint32_t rank = ptx::cluster_ctarank();
@@ -453,6 +551,9 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       ptx::mbar_init(&tfull[a], 1);
       ptx::mbar_init(&tempty[a], 2 * kEpiWarps);  // both CTAs' epilogue warps
     }
+    ptx::mbar_init(rfull, 1);
+    ptx::mbar_init(rfree, kEpiWarps);
+    if (kResidBuf) ptx::tma_prefetch_desc(&tmR);
     ptx::fence_mbar_init();
   }
   if (warp == kMmaWarp) ptx::tmem_alloc_pair(tmem_slot, C::TMEM_COLS);
@@ -494,6 +595,15 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
         const int m0 = tile_m(tile, num_m, num_n) * 2 * BM + rank * BM;
         const int n0 = tile_n(tile, num_m, num_n) * BN + rank * C::B_ROWS;
 #endif
+        // this CTA's 128 residual rows of the tile, full BN columns (see gemm_tc_kernel)
+        bool r_issued = !kResidBuf;
+        auto issue_resid = [&]() {
+          const int nr0 = tile_n(tile, num_m, num_n) * BN;
+          ptx::mbar_arrive_expect_tx(rfull, (uint32_t)resid_buf_bytes<BN>());
+          for (int c = 0; c < BN / CW; ++c)
+            ptx::tma_load_2d(rbuf + c * (BM * CW * 2), &tmR, rfull, nr0 + c * CW, m0);
+          r_issued = true;
+        };
         for (int kb = 0; kb < kblocks; ++kb) {
           const uint32_t fb = ptx::mapa_shared(&full[stage], 0);
           if (it == 0 && kb < pre) {
@@ -505,6 +615,11 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
             ptx::tma_load_2d_pair(sB + stage * C::B_BYTES, &tmB, fb, kb * BK, n0);
           }
           if (++stage == C::STAGES) { stage = 0; phase ^= 1; }
+          if (!r_issued && (it == 0 || ptx::mbar_test(rfree, (it - 1) & 1))) issue_resid();
+        }
+        if (!r_issued) {
+          ptx::mbar_wait(rfree, (it - 1) & 1);
+          issue_resid();
         }
       }
     } else {
@@ -549,7 +664,8 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   } else {
     pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
+    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * kWarpStg;
+    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kBiasWarpBytes : stg + kStgBufs * kStgBytes);
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -557,8 +673,10 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     for (int tile = pair; tile < tiles; tile += npairs, ++it) {
       const int m0 = tile_m(tile, num_m, num_n) * 2 * BM + rank * BM, n0 = tile_n(tile, num_m, num_n) * BN;
       uint4 rv0[CW / 8];
-      prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
+      if (!kResidBuf) prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
+      stage_bias<BN, kEpiGroups>(sbias, bias, n0, cg, lane);
       ptx::mbar_wait(&tfull[acc], acc_phase);
+      if (kResidBuf) ptx::mbar_wait(rfull, it & 1);  // this tile's residual has landed
       ptx::tc_fence_after();
       if (warp == 0 && lane == 0) trace(6 + 6 * it);
       const uint32_t te = ptx::mapa_shared(&tempty[acc], 0);
@@ -570,7 +688,12 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
 #else
                                ptx::mbar_arrive_remote(te);
 #endif
-                             }, outp, N, rv0);
+                             }, outp, N, rv0, kResidBuf ? rbuf : nullptr, sbias);
+      if (kResidBuf) {
+        if (lane == 0) ptx::bulk_wait_read<0>();
+        __syncwarp();
+        if (lane == 0) ptx::mbar_arrive(rfree);
+      }
       if (warp == 0 && lane == 0) trace(7 + 6 * it);
       if (++acc == kAccStages) { acc = 0; acc_phase ^= 1; }
     }
@@ -1010,7 +1133,7 @@ gemm_ln_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   } else {
     pdl_wait();  // residual rows come from the previous kernels
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = sStg + warp * kStgBufs * kStgBytes;
+    uint8_t* stg = sStg + warp * kWarpStg;
     int sc = 0, use = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -1054,14 +1177,14 @@ EncodeTiledFn get_encode_fn() {
 
 template <int BN, int EPI, bool PAIR, int EW>
 cudaError_t launch_cfg_ew(const TcGemmPlan& p, cudaStream_t s) {
-  using C = TcCfg<BN, PAIR, 0, EW>;
+  using C = TcCfg<BN, PAIR, 0, EW, ARLO_RESID_TMA && EPI == EPI_BIAS_RESID>;
   auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI, EW> : gemm_tc_kernel<BN, EPI, EW>;
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [&] {
     return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
   if (e != cudaSuccess) return e;
-  return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.M, p.N, p.K,
-                  p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out, p.lnp);
+  return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.tmR, p.M, p.N,
+                  p.K, p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out, p.lnp);
 }
 
 template <int BN, int EPI, bool PAIR>
@@ -1237,6 +1360,9 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128, (uint64_t)lda)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
+  // residual rows (stride ldr), {32 columns x 128 rows} boxes in the output staging layout
+  if (epi == EPI_BIAS_RESID && !encode_tmap_bf16_2d(&p->tmR, resid, (uint64_t)N, (uint64_t)M, CW, BM, CW * 2, (uint64_t)ldr))
+    return false;
   return true;
 }
 

@@ -44,6 +44,7 @@ struct TcGemmPlan {
   CUtensorMap tmA;  // activations [M, K] bf16, box {64, 128}, 128B swizzle
   CUtensorMap tmB;  // weights     [N, K] bf16, box {64, BN (BN/2 for a pair)}, 128B swizzle
   CUtensorMap tmC;  // output      [M, N] bf16, box {32, 32}, 64B swizzle (epilogue TMA stores)
+  CUtensorMap tmR;  // residual    [M, N] bf16 (row stride ldr), box {32, 128}, 64B swizzle (EPI_BIAS_RESID)
   int M, N, K, BN, epi, grid;
   int ew;       // epilogue warps of the persistent kernels (8, or 12 for GELU at M <= 8192)
   bool pair;    // CTA-pair (cta_group::2) kernel, 256-row tiles

@@ -54,3 +54,17 @@ print("per tile (median): mainloop issue span %s" % " ".join(f"{x:.2f}" for x in
 print("                   epilogue span       %s" % " ".join(f"{x:.2f}" for x in epil))
 print("                   MMA idle before acc %s" % " ".join(f"{x:.2f}" for x in wait))
 print("end: median %.2f max %.2f us" % (np.nanmedian(rel[:, 1]), np.nanmax(rel[:, 1])))
+
+# clock64 sub-stamps of warp 0's epilogue on each CTA's first tile (slots 32..63): 32 epi start,
+# 33 first TMEM chunk in registers, then per chunk k: 34+5k start, 35+5k math done, 36+5k staging
+# buffer free, 37+5k TMA store issued, 38+5k next chunk's TMEM load landed
+raw = buf.cpu().numpy().reshape(148, 64)[:grid].astype(np.float64)
+if (raw[:, 33] > 0).any():
+    d = lambda a, b: np.median(raw[:, b] - raw[:, a])
+    print("epilogue warp 0, first tile (median cycles): start->tmem %.0f" % d(32, 33))
+    for k in range(6):
+        if (raw[:, 34 + 5 * k] > 0).sum() < grid // 2:
+            break
+        print("  chunk %d: math %.0f  stg-wait %.0f  smem+store %.0f  tmem-wait %.0f  (from start %.0f)" % (
+            k, d(34 + 5 * k, 35 + 5 * k), d(35 + 5 * k, 36 + 5 * k), d(36 + 5 * k, 37 + 5 * k), d(37 + 5 * k, 38 + 5 * k),
+            d(32, 38 + 5 * k)))
