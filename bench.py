@@ -377,6 +377,17 @@ def main():
         extras["per_L_latency_ms_restricted"] = per_L_table(runtimes, torch, dev, stream, cfg, restricted=True)
         pl = extras["per_L_latency_ms"]
         result["per_L_b1_ms"] = {L: rnd(pl[L]["1"]["median"]) for L in pl}
+        # the paper's batch-1 runtimes in the LATENCY family (LayerNorm folded into
+        # the GEMMs): max_batch = 1 runtimes, one forward of b = 1 at length L
+        lat_rts = {}
+        for L in RUNTIME_LS:
+            lat_rts[L] = arlo.Runtime(W, L, 1, arlo.RUNTIME_LATENCY)
+            lat_rts[L].set_stream(stream)
+        lt = per_L_table(lat_rts, torch, dev, stream, cfg, b_list=(1,))
+        extras["per_L_latency_family_b1_ms"] = lt
+        result["per_L_b1_latency_family_ms"] = {L: rnd(lt[L]["1"]["median"]) for L in lt}
+        for rt in lat_rts.values():
+            rt.close()
         extras["paper_context"] = {
             "note": "context only: RTX 3090, FP32 TensorRT static shape, batch 1 (BASELINE.md section 1)",
             "bert_base_L512_b1_ms": {"paper_rtx3090": 4.86, "this_b200_bf16": pl["512"]["1"]["median"],
@@ -568,7 +579,7 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
     return roof, table
 
 
-def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False):
+def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False, b_list=None):
     """Offline-profiler table (A4): latency of one forward vs batch bucket for every runtime.
     restricted=False: every request has length L (roofline mode, SURVEY 8(d)(i));
     restricted=True: lengths drawn from the skewed distribution restricted to (L-64, L] (8(d)(ii)),
@@ -576,7 +587,7 @@ def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False):
     table = {}
     for L, rt in runtimes.items():
         row = {}
-        for b in ((1, 8, 32) if restricted else (1, 2, 4, 8, 16, 32)):
+        for b in b_list or ((1, 8, 32) if restricted else (1, 2, 4, 8, 16, 32)):
             lens = (wl.sample_lengths(b, seed=7 + b, lo=L - 64, hi=L) if restricted else np.full(b, L)).astype(np.int32)
             ids = torch.from_numpy(wl.sample_token_ids(cfg, lens, L, seed=5)).to(dev)
             ld = torch.from_numpy(lens).to(dev)

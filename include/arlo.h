@@ -109,19 +109,24 @@ typedef struct arlo_runtime arlo_runtime;
 int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weights* w, arlo_runtime** out);
 
 /*
- * Runtime families.  The paper's runtimes run at batch 1 (§5); at M = L
- * rows a projection streams its whole weight matrix for 2L flops per element, so the
- * LATENCY family runs every GEMM as a split-K weight-streaming kernel: a cluster of S
- * CTAs per column tile, S = a function of the weight shape (N, K) only, partial sums
- * added in a fixed order over distributed shared memory.  The THROUGHPUT family runs
- * the tile kernels (each output element's K chain in one accumulator).  Within a family
- * a request's logits are bitwise equal on every runtime L >= its length and in every
- * batch bucket; across families they agree to bf16 rounding (both within 2e-2 of the
- * oracle).  DEFAULT = THROUGHPUT: on B200 a batch-1 forward is bound by its chain of
- * ~87 dependent kernels (~4.5 us each), not by the GEMMs, and the latency family measured
- * no faster.  fp32 check mode ignores the family (SIMT GEMMs).
+ * Runtime families (bf16; fp32 check mode ignores the family: SIMT GEMMs + LayerNorm kernels).
+ * Within a family a request's logits are bitwise equal on every runtime L >= its length and in
+ * every batch bucket; across families they agree to bf16 rounding (all within 2e-2 of the oracle).
+ *  THROUGHPUT (DEFAULT): tcgen05 tile GEMMs (each output element's K chain in one accumulator),
+ *    attention, LayerNorm kernels: 3 + 7 * layers kernels per forward.
+ *  LATENCY: the paper's batch-1 runtimes (§5).  The same tile GEMMs with every
+ *    LayerNorm folded into the GEMMs around it (include/arlo_ops.h arlo_op_gemm_fold): residual
+ *    GEMMs emit row statistics, the consuming GEMMs run on gamma-scaled weights and normalise in
+ *    their epilogue, no LayerNorm kernel (3 + 5 * layers kernels).  Measured on B200: batch-1
+ *    forwards 6-9 % faster than THROUGHPUT; at batch 32 the heavier epilogues cost more than the
+ *    LayerNorm launches they replace, hence not the default.
+ *  FUSED: see below.
+ *  SPLITK: every GEMM a split-K weight-streaming kernel (a cluster of S CTAs per column tile,
+ *    S a function of (N, K) only, partials added in a fixed order over distributed shared memory)
+ *    + LayerNorm kernels; measured no faster than THROUGHPUT at batch 1.
  */
-enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHPUT = 2, ARLO_RUNTIME_FUSED = 3 };
+enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHPUT = 2, ARLO_RUNTIME_FUSED = 3,
+       ARLO_RUNTIME_SPLITK = 4 };
 /*
  * ARLO_RUNTIME_FUSED: the whole forward (embedding .. logits) as ONE persistent kernel of one
  * CTA per SM running a static task graph (GEMM units, attention per (sequence, head),
@@ -135,7 +140,7 @@ enum { ARLO_RUNTIME_DEFAULT = 0, ARLO_RUNTIME_LATENCY = 1, ARLO_RUNTIME_THROUGHP
  */
 int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_weights* w, int32_t family,
                            arlo_runtime** out);
-/* ARLO_RUNTIME_LATENCY or ARLO_RUNTIME_THROUGHPUT (the family the runtime was built as). */
+/* The family the runtime was built as (never ARLO_RUNTIME_DEFAULT). */
 int32_t arlo_runtime_family(const arlo_runtime* rt);
 void arlo_runtime_destroy(arlo_runtime* rt);
 /* Launch stream for every later call (a cudaStream_t; NULL = legacy default stream). */

@@ -93,6 +93,28 @@ int arlo_op_ln_gemm(int32_t M, int32_t N, int32_t K, const void* y, const float*
                     void* x, const void* W, const float* bias, void* out, int32_t epi, int32_t force_bn,
                     void* barrier, void* stream);
 
+/*
+ * LayerNorm fold epilogues of the tcgen05 GEMM (the throughput runtimes fold every LayerNorm into
+ * the GEMMs around it instead of launching it; BERT post-LN, PAPER.md:L422 [17]).
+ * Row statistics st[g][row][2] = (sum, sum of squares) of the 32 bf16 values of granule g of a row
+ * (fp32, column order), granule-major with st_ld >= M rows per granule plane; a consumer adds the
+ * granules in order and uses var = E[y^2] - mean^2.
+ *   epi ARLO_EPI_LNFOLD (3) / ARLO_EPI_LNFOLD_GELU (4): A = y [M, K] (not normalised), W = W' [N, K]
+ *     (= bf16(W * gamma)), v0 = s [N] (row sums of W'), v1 = c [N] (= W beta + b), st_in = statistics
+ *     of A's rows (K / 32 granules; row i's statistics are those of row i * st_in_stride):
+ *     out = bf16(rstd_i * acc - rstd_i * mean_i * s_n + c_n) (then GELU, erf form).
+ *   epi ARLO_EPI_RESID_LN (5): out = bf16((acc + v0_n) + LN(r)) with LN(r) = ((r - mean) * rstd) *
+ *     v1_n + v2_n from the residual rows r and their statistics st_in (N / 32 granules; st_in = NULL:
+ *     plain residual r); st_out (optional) receives the statistics of the bf16 output rows.
+ * Device pointers; M >= 1, N and K multiples of 64; force_bn as for arlo_op_gemm (no split-K).
+ * Errors: EINVAL, ECUDA.
+ */
+enum { ARLO_EPI_LNFOLD = 3, ARLO_EPI_LNFOLD_GELU = 4, ARLO_EPI_RESID_LN = 5 };
+int arlo_op_gemm_fold(int32_t M, int32_t N, int32_t K, const void* A, const void* W, const float* v0,
+                      const float* v1, const float* v2, const float* st_in, int32_t st_in_stride,
+                      float* st_out, int32_t st_ld, float eps, const void* residual, void* out, int32_t epi,
+                      int32_t force_bn, void* stream);
+
 /* The tile configuration arlo_op_gemm / the runtime graphs use for (M, N, K):
  * BN for the single-CTA kernel, -BN for the CTA-pair kernel, 1000 + BN for the
  * skinny small-M kernel, 0 if unsupported. */

@@ -28,7 +28,8 @@ OK, EINVAL, ETOOLONG, ENOMEM, ECUDA, EINFEASIBLE, ENOCAND, ENODEV = 0, -1, -2, -
 BF16, FP32 = 0, 1
 DISPATCH_RS, DISPATCH_ILB, DISPATCH_IG = 0, 1, 2
 EPI_BIAS, EPI_BIAS_GELU, EPI_BIAS_RESIDUAL = 0, 1, 2
-RUNTIME_DEFAULT, RUNTIME_LATENCY, RUNTIME_THROUGHPUT, RUNTIME_FUSED = 0, 1, 2, 3
+EPI_LNFOLD, EPI_LNFOLD_GELU, EPI_RESID_LN = 3, 4, 5
+RUNTIME_DEFAULT, RUNTIME_LATENCY, RUNTIME_THROUGHPUT, RUNTIME_FUSED, RUNTIME_SPLITK = 0, 1, 2, 3, 4
 SKINNY_CODE, SPLITK_CODE, FUSED_CODE = 1000, 2000, 3000  # tile codes: kSkinnyCode + BN, kSplitKCode + BN, kFusedCode + S
 
 EXPORTED = [
@@ -37,7 +38,7 @@ EXPORTED = [
     "arlo_runtime_create", "arlo_runtime_create_ex", "arlo_runtime_family", "arlo_runtime_destroy", "arlo_runtime_set_stream", "arlo_runtime_length",
     "arlo_runtime_max_batch", "arlo_infer", "arlo_enqueue", "arlo_runtime_kernel_count", "arlo_runtime_bucket", "arlo_allocate",
     "arlo_sched_create", "arlo_sched_destroy", "arlo_sched_set_params", "arlo_sched_set_policy", "arlo_dispatch", "arlo_complete", "arlo_sched_outstanding",
-    "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_ln_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
+    "arlo_op_gemm", "arlo_op_gemm_ln", "arlo_op_gemm_fold", "arlo_op_ln_gemm", "arlo_op_layernorm", "arlo_op_embed", "arlo_op_attention", "arlo_op_head",
     "arlo_debug_gemm_trace", "arlo_debug_attn_trace", "arlo_debug_fused_trace", "arlo_gemm_tile_choice",
 ]
 
@@ -86,6 +87,7 @@ _sig("arlo_dispatch", C.c_int, _vp, _i32, _P(_i32), _P(_i32))
 _sig("arlo_complete", C.c_int, _vp, _i32, _i32)
 _sig("arlo_sched_outstanding", _i32, _vp, _i32, _i32)
 _sig("arlo_op_gemm", C.c_int, _i32, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _i32, _i32, _vp)
+_sig("arlo_op_gemm_fold", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _i32, _vp, _i32, _f32, _vp, _vp, _i32, _i32, _vp)
 _sig("arlo_op_gemm_ln", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _vp, _vp, _vp, _f32, _vp, _vp)
 _sig("arlo_op_ln_gemm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp, _vp, _vp, _i32, _i32, _vp, _vp)
 _sig("arlo_op_layernorm", C.c_int, _i32, _i32, _i32, _vp, _vp, _vp, _f32, _vp, _vp)
@@ -182,7 +184,7 @@ class Runtime:
 
     @property
     def family(self) -> int:
-        """RUNTIME_LATENCY (split-K weight streaming) or RUNTIME_THROUGHPUT (tile kernels)."""
+        """RUNTIME_THROUGHPUT, RUNTIME_LATENCY (LayerNorm fold), RUNTIME_FUSED or RUNTIME_SPLITK."""
         return check(lib.arlo_runtime_family(self.handle))
 
     def set_stream(self, stream):
@@ -287,6 +289,18 @@ def op_gemm(dtype, A, W, bias, out, epi=EPI_BIAS, residual=None, force_bn=0, str
     N = W.shape[0]
     check(lib.arlo_op_gemm(dtype, M, N, K, _ptr(A), _ptr(W), _ptr(bias), _ptr(residual), _ptr(out), epi,
                            force_bn, _stream_ptr(stream)))
+    return out
+
+
+def op_gemm_fold(A, W, v0, out, epi, v1=None, v2=None, st_in=None, st_in_stride=1, st_out=None, st_ld=None,
+                 eps=1e-12, residual=None, force_bn=0, stream=None):
+    """LayerNorm-fold epilogues (arlo_op_gemm_fold; include/arlo_ops.h).  Statistics tensors are
+    granule-major [G, st_ld, 2] (st_ld defaults to M)."""
+    M, K = A.shape
+    N = W.shape[0]
+    check(lib.arlo_op_gemm_fold(M, N, K, _ptr(A), _ptr(W), _ptr(v0), _ptr(v1), _ptr(v2), _ptr(st_in), st_in_stride,
+                                _ptr(st_out), st_ld or M, eps, _ptr(residual), _ptr(out), epi, force_bn,
+                                _stream_ptr(stream)))
     return out
 
 

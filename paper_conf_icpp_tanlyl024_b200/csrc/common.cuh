@@ -172,10 +172,39 @@ __device__ __forceinline__ uint4 ld_dep_v4(const void* p) {
   return v;
 }
 
+__device__ __forceinline__ float4 ld_dep_f4(const void* p) {
+  const uint4 u = ld_dep_v4(p);
+  return make_float4(__uint_as_float(u.x), __uint_as_float(u.y), __uint_as_float(u.z), __uint_as_float(u.w));
+}
+
 __device__ __forceinline__ uint2 ld_dep_v2(const void* p) {
   uint2 v;
   asm volatile("ld.global.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "l"(p) : "memory");
   return v;
+}
+
+// Mean and 1/sqrt(var + eps) of a row from its granule statistics (FoldArgs; granule-major
+// st[g][row][2], plane stride `ld` rows): the G = H/32 granules added in column order, var =
+// E[y^2] - mean^2 (clamped at 0).  Loads go out in groups of 8 (a chain of dependent L2 loads
+// under GEMM traffic cost microseconds per tile).
+__device__ __forceinline__ float2 fold_row_stats(const float* st, size_t row, int ld, int G, int H, float eps) {
+  const float2* p = reinterpret_cast<const float2*>(st) + row;
+  float s1 = 0.f, s2 = 0.f;
+  for (int g0 = 0; g0 < G; g0 += 8) {
+    float2 v[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      if (g0 + i < G) v[i] = __ldcg(p + (size_t)(g0 + i) * ld);
+#pragma unroll
+    for (int i = 0; i < 8; ++i)
+      if (g0 + i < G) {
+        s1 += v[i].x;
+        s2 += v[i].y;
+      }
+  }
+  const float mean = s1 / (float)H;
+  const float var = fmaxf(s2 / (float)H - mean * mean, 0.f);
+  return make_float2(mean, 1.0f / sqrtf(var + eps));
 }
 
 bool pdl_enabled();  // false when ARLO_NO_PDL is set in the environment (A/B measurements)

@@ -114,7 +114,42 @@ __global__ void __launch_bounds__(kLnThreads) embed_ln_kernel(int B, int L, int 
   ln_finish<T, MAXV>(v, nvec, H, lane, s_aff, s_aff + H, eps, out + (size_t)row * H);
 }
 
+// LayerNorm fold (runtime.cu): a GEMM consuming LN(y) = (y - mu) rstd * gamma + beta runs on y with
+//   W'[n, k] = bf16(W[n, k] * gamma[k]),  s[n] = sum_k W'[n, k],  c[n] = sum_k W[n, k] beta[k] + b[n]
+// and the epilogue out = rstd * acc - rstd * mu * s[n] + c[n].  One warp per output row n; the sums
+// in fp64 (lane-strided, then a fixed shuffle tree), computed once per weight set.
+__global__ void __launch_bounds__(128) fold_weights_kernel(int N, int K, const bf16* __restrict__ W,
+                                                           const float* __restrict__ gamma,
+                                                           const float* __restrict__ beta, const float* __restrict__ b,
+                                                           bf16* __restrict__ Wf, float* __restrict__ s,
+                                                           float* __restrict__ c) {
+  const int n = blockIdx.x * 4 + (threadIdx.x >> 5), lane = threadIdx.x & 31;
+  if (n >= N) return;
+  double ss = 0.0, cc = 0.0;
+  for (int k = lane; k < K; k += 32) {
+    const float w = __bfloat162float(W[(size_t)n * K + k]);
+    const bf16 wf = __float2bfloat16_rn(w * gamma[k]);
+    Wf[(size_t)n * K + k] = wf;
+    ss += (double)__bfloat162float(wf);
+    cc += (double)w * (double)beta[k];
+  }
+  for (int o = 16; o > 0; o >>= 1) {
+    ss += __shfl_xor_sync(0xffffffffu, ss, o);
+    cc += __shfl_xor_sync(0xffffffffu, cc, o);
+  }
+  if (lane == 0) {
+    s[n] = (float)ss;
+    c[n] = (float)(cc + (double)b[n]);
+  }
+}
+
 }  // namespace
+
+cudaError_t launch_fold_weights(int N, int K, const void* W, const float* gamma, const float* beta, const float* b,
+                                void* Wf, float* s, float* c, cudaStream_t st) {
+  fold_weights_kernel<<<(N + 3) / 4, 128, 0, st>>>(N, K, (const bf16*)W, gamma, beta, b, (bf16*)Wf, s, c);
+  return cudaGetLastError();
+}
 
 #define ARLO_MAXV_SWITCH(maxv, ...)            \
   switch (maxv) {                              \

@@ -271,7 +271,7 @@ bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int 
   if (stages < 2) stages = 2;  // (a budget too small for two stages is exceeded)
   if (stages > kblocks) stages = kblocks;
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->epi = epi; p->grid = (int)ctas; p->ew = 4;
-  p->pair = false; p->skinny = false; p->ln = false; p->splitk = true; p->lnp = LnPrologue{};
+  p->pair = false; p->skinny = false; p->ln = false; p->splitk = true; p->fold = FoldArgs{}; p->lnp = LnPrologue{};
   p->splits = S; p->kc = kc; p->stages = stages; p->a_stage = a_stage; p->a_rows = a_rows;
   p->smem = fixed + stages * (a_stage + b_stage);
   p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;

@@ -58,6 +58,11 @@ constexpr int kStgBufs = ARLO_STG_BUFS;         // staging tiles per epilogue wa
 #define ARLO_BIAS_SMEM 1  // A/B hook: 0 reads bias with __ldg inside the chunk loop
 #endif
 constexpr int kBiasWarpBytes = ARLO_BIAS_SMEM ? 4 * 32 * 4 : 0;
+// Column vectors an epilogue stages per warp and chunk: bias (EPI 0-2), s and c (LN fold), bias,
+// gamma and beta (residual + on-the-fly LayerNorm).  The fold epilogues always stage them.
+constexpr int nvec_of(int epi) { return epi == EPI_RESID_LN ? 3 : epi >= EPI_LNFOLD ? 2 : 1; }
+constexpr int col_warp_bytes(int epi) { return epi >= EPI_LNFOLD ? 4 * 32 * 4 * nvec_of(epi) : kBiasWarpBytes; }
+constexpr bool is_resid(int epi) { return epi == EPI_BIAS_RESID || epi == EPI_RESID_LN; }
 constexpr int kWarpStg = kStgBufs * kStgBytes + kBiasWarpBytes;
 constexpr int kStagingBytes = kEpiWarps * kWarpStg;
 
@@ -131,9 +136,10 @@ constexpr int tmem_cols_for(int n) {
 template <int BN>
 constexpr int resid_buf_bytes() { return BN * 128 * 2; }
 
-template <int BN, bool PAIR, int RESERVE = 0, int EW = kEpiWarps, bool RESID_BUF = false>
+template <int BN, bool PAIR, int RESERVE = 0, int EW = kEpiWarps, bool RESID_BUF = false, int COLB = kBiasWarpBytes>
 struct TcCfg {
-  static constexpr int kStagingBytes = RESID_BUF ? EW * kBiasWarpBytes + resid_buf_bytes<BN>() : Roles<EW>::kStaging;
+  static constexpr int kStagingBytes =
+      RESID_BUF ? EW * COLB + resid_buf_bytes<BN>() : EW * (kStgBufs * kStgBytes + COLB);
   static constexpr int A_BYTES = BM * BK * 2;
   static constexpr int B_ROWS = PAIR ? BN / 2 : BN;
   static constexpr int B_BYTES = B_ROWS * BK * 2;
@@ -166,7 +172,7 @@ constexpr int CW = 32;  // chunk width: TMEM load / staging tile / TMA box (colu
 template <int BN, int EPI>
 __device__ __forceinline__ void prefetch_first_resid(uint4 (&rv)[CW / 8], const bf16* resid, int row0, int lane,
                                                      int n0, int cg, int M, int ldr) {
-  if (EPI != EPI_BIAS_RESID || cg * CW >= BN) return;  // (a warp without chunks loads nothing)
+  if (!is_resid(EPI) || cg * CW >= BN) return;  // (a warp without chunks loads nothing)
   const int row = row0 + lane;
   if (row >= M) return;
   const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0) + cg * (CW / 8);
@@ -174,21 +180,83 @@ __device__ __forceinline__ void prefetch_first_resid(uint4 (&rv)[CW / 8], const 
   for (int j = 0; j < CW / 8; ++j) rv[j] = ld_dep_v4(res4 + j);
 }
 
-// Bias of this warp's chunks cg, cg + G, ... of the tile at column n0 -> the warp's bias slots
-// (lane j writes column 32 c + j; the math then reads float4 broadcasts).  Called before the
-// accumulator wait; the warp's previous tile has finished reading the slots.
-template <int BN, int kEpiGroups>
-__device__ __forceinline__ void stage_bias(float* sbias, const float* __restrict__ bias, int n0, int cg, int lane) {
+// Column vectors of this warp's chunks cg, cg + G, ... of the tile at column n0 -> the warp's
+// slots [chunk k][vector v][32 columns] (lane j writes column 32 c + j; the math reads float4
+// broadcasts): bias, or s and c (LN fold), or bias, gamma and beta (residual LN).  Called before
+// the accumulator wait; the warp's previous tile has finished reading the slots.
+template <int BN, int EPI, int kEpiGroups>
+__device__ __forceinline__ void stage_colv(float* sv, const float* __restrict__ v0, const FoldArgs& fa, int n0, int cg,
+                                           int lane) {
   constexpr int NCH = BN / CW;
   constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;
-  static_assert(!ARLO_BIAS_SMEM || NCMAX * CW * 4 <= kBiasWarpBytes, "bias slots");
-  if (!ARLO_BIAS_SMEM) return;
+  constexpr int NV = nvec_of(EPI);
+  static_assert(NCMAX * CW * 4 * NV <= col_warp_bytes(EPI) || (!ARLO_BIAS_SMEM && EPI < EPI_LNFOLD), "column slots");
+  if (!ARLO_BIAS_SMEM && EPI < EPI_LNFOLD) return;
 #pragma unroll
   for (int k = 0; k < NCMAX; ++k) {
     const int c = cg + k * kEpiGroups;
-    if (c < NCH) sbias[k * CW + lane] = __ldg(bias + n0 + c * CW + lane);
+    if (c < NCH) {
+      const int col = n0 + c * CW + lane;
+      sv[(k * NV) * CW + lane] = __ldg(v0 + col);
+      if (NV >= 2) sv[(k * NV + 1) * CW + lane] = fa.v1 ? __ldg(fa.v1 + col) : 0.f;
+      if (NV >= 3) sv[(k * NV + 2) * CW + lane] = fa.v2 ? __ldg(fa.v2 + col) : 0.f;
+    }
   }
   __syncwarp();
+}
+
+
+// Epilogue arithmetic of one 32-column chunk of a row for the LayerNorm-fold modes (paired fp32):
+//  EPI_LNFOLD(_GELU): x = acc * rstd + (nrm * s + c), nrm = -rstd * mean (rowst = (nrm, rstd)); GELU;
+//  EPI_RESID_LN: x = (acc + b) + LN(r), LN(r) = ((r - mean) * rstd) * gamma + beta
+//    (rowst = (mean, rstd) of the residual row; mean 0 / rstd 1 / gamma 1 / beta 0 = plain residual
+//    is not used: a plain residual passes rowst.y < 0).
+template <int EPI>
+__device__ __forceinline__ uint32_t epi_fold_pair(float2 a, float2 v0, float2 v1, float2 v2, uint32_t ru, float2 rowst) {
+  float2 x;
+  if constexpr (EPI == EPI_LNFOLD || EPI == EPI_LNFOLD_GELU) {  // v0 = s, v1 = c
+    x = __ffma2_rn(a, f2(rowst.y), __ffma2_rn(f2(rowst.x), v0, v1));
+    if (EPI == EPI_LNFOLD_GELU) x = gelu2_erf_fast(x);
+  } else {  // v0 = bias, v1 = gamma, v2 = beta
+    float2 rr = unpack_bf16x2(ru);
+    if (rowst.y >= 0.f) rr = __ffma2_rn(__fmul2_rn(__fadd2_rn(rr, f2(-rowst.x)), f2(rowst.y)), v1, v2);
+    x = __fadd2_rn(__fadd2_rn(a, v0), rr);
+  }
+  return pack_bf16x2(x.x, x.y);
+}
+
+template <int EPI>
+__device__ __forceinline__ void epi_fold_chunk(const uint32_t* acc, const float* sv, const uint32_t* ru, float2 rowst,
+                                               uint32_t* pk) {
+  constexpr int NV = nvec_of(EPI);
+  const float4* s0 = reinterpret_cast<const float4*>(sv);
+  const float4* s1 = s0 + CW / 4;
+  const float4* s2 = s1 + CW / 4;
+#pragma unroll
+  for (int j = 0; j < CW / 4; ++j) {  // 4 columns: 2 pairs
+    const float4 a0 = s0[j], a1 = s1[j];
+    const float4 a2 = NV >= 3 ? s2[j] : make_float4(0.f, 0.f, 0.f, 0.f);
+    const float2 x0 = make_float2(__uint_as_float(acc[4 * j]), __uint_as_float(acc[4 * j + 1]));
+    const float2 x1 = make_float2(__uint_as_float(acc[4 * j + 2]), __uint_as_float(acc[4 * j + 3]));
+    pk[2 * j] = epi_fold_pair<EPI>(x0, make_float2(a0.x, a0.y), make_float2(a1.x, a1.y), make_float2(a2.x, a2.y),
+                                   ru[2 * j], rowst);
+    pk[2 * j + 1] = epi_fold_pair<EPI>(x1, make_float2(a0.z, a0.w), make_float2(a1.z, a1.w),
+                                       make_float2(a2.z, a2.w), ru[2 * j + 1], rowst);
+  }
+}
+
+// (sum y, sum y^2) of 16 packed bf16 words (32 columns) in column order, continuing (s1, s2).
+__device__ __forceinline__ float2 fold_granule(const uint32_t* pk, int nw, float2 acc) {
+  float s1 = acc.x, s2 = acc.y;
+#pragma unroll
+  for (int j = 0; j < 16; ++j) {
+    if (j < nw) {
+      const float2 y = unpack_bf16x2(pk[j]);
+      s1 += y.x; s2 = fmaf(y.x, y.x, s2);
+      s1 += y.y; s2 = fmaf(y.y, y.y, s2);
+    }
+  }
+  return make_float2(s1, s2);
 }
 
 template <int BN, int EPI, int kEpiGroups, typename Release>
@@ -197,7 +265,8 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
                                               const bf16* __restrict__ resid, const CUtensorMap* tmC,
                                               uint8_t* stg, int& sc, Release release, bf16* __restrict__ outp,
                                               int N, const uint4* rv_first, uint8_t* rbuf = nullptr,
-                                              const float* sbias = nullptr) {
+                                              const float* sbias = nullptr, float2 rowst = make_float2(0.f, 1.f),
+                                              float* st_out = nullptr, int st_ld = 0) {
   static_assert(BN % CW == 0, "tile width must be a multiple of 32");
   constexpr int NCH = BN / CW;                                 // chunks per row block
   constexpr int NCMAX = (NCH + kEpiGroups - 1) / kEpiGroups;  // chunks per warp (max)
@@ -219,7 +288,8 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   uint32_t r[2][CW];
   uint4 rv[2][RV];
   const bool rsm = rbuf != nullptr;  // residual tile in shared memory (TMA-prefetched), output in place
-  if (EPI == EPI_BIAS_RESID && row_ok && !rsm) {  // prefetched by the caller before the accumulator wait
+  constexpr int NV = nvec_of(EPI);
+  if (is_resid(EPI) && row_ok && !rsm) {  // prefetched by the caller before the accumulator wait
 #pragma unroll
     for (int j = 0; j < RV; ++j) rv[0][j] = rv_first[j];
   }
@@ -234,31 +304,39 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
     if (stamp && first_tile && k < 6) trace_clk(34 + 5 * k);
     // this chunk's 32 rows x 32 columns in the residual buffer (64-byte rows, 64B swizzle)
     uint8_t* rchunk = rsm ? rbuf + c * (BM * CW * 2) + q * (32 * CW * 2) : nullptr;
-    if (EPI == EPI_BIAS_RESID && rsm) {
+    if (is_resid(EPI) && rsm) {
 #pragma unroll
       for (int j = 0; j < RV; ++j)
         rv[cur][j] = *reinterpret_cast<const uint4*>(rchunk + lane * (CW * 2) + ((j ^ ((lane >> 1) & 3)) * 16));
     }
     if (k + 1 < nc) {
       ptx::tmem_ld_32x32b_x32(t_row + (c + kEpiGroups) * CW, r[nxt]);
-      if (EPI == EPI_BIAS_RESID && row_ok && !rsm) {
+      if (is_resid(EPI) && row_ok && !rsm) {
 #pragma unroll
         for (int j = 0; j < RV; ++j) rv[nxt][j] = ld_dep_v4(res4 + (c + kEpiGroups) * RV + j);
       }
     }
-    const float4* bias4 = ARLO_BIAS_SMEM ? reinterpret_cast<const float4*>(sbias) + k * (CW / 4)
-                                         : reinterpret_cast<const float4*>(bias + n0 + c * CW);
     uint32_t pk[CW / 2];
+    if constexpr (EPI < EPI_LNFOLD) {
+      const float4* bias4 = ARLO_BIAS_SMEM ? reinterpret_cast<const float4*>(sbias) + k * (CW / 4)
+                                           : reinterpret_cast<const float4*>(bias + n0 + c * CW);
 #pragma unroll
-    for (int j = 0; j < CW / 4; ++j) {
-      const float4 b4 = ARLO_BIAS_SMEM ? bias4[j] : __ldg(bias4 + j);
-      uint32_t ua = 0, ub = 0;
-      if (EPI == EPI_BIAS_RESID) {
-        const uint4 u = rv[cur][j >> 1];
-        ua = (j & 1) ? u.z : u.x;
-        ub = (j & 1) ? u.w : u.y;
+      for (int j = 0; j < CW / 4; ++j) {
+        const float4 b4 = ARLO_BIAS_SMEM ? bias4[j] : __ldg(bias4 + j);
+        uint32_t ua = 0, ub = 0;
+        if (EPI == EPI_BIAS_RESID) {
+          const uint4 u = rv[cur][j >> 1];
+          ua = (j & 1) ? u.z : u.x;
+          ub = (j & 1) ? u.w : u.y;
+        }
+        epi_pack4<EPI>(&r[cur][4 * j], b4, ua, ub, pk[2 * j], pk[2 * j + 1]);
       }
-      epi_pack4<EPI>(&r[cur][4 * j], b4, ua, ub, pk[2 * j], pk[2 * j + 1]);
+    } else {
+      const float* sv = sbias + k * NV * CW;  // this chunk's column vectors
+      epi_fold_chunk<EPI>(&r[cur][0], sv, reinterpret_cast<const uint32_t*>(rv[cur]), rowst, pk);
+      if (EPI == EPI_RESID_LN && st_out != nullptr && row_ok)  // granule (= chunk) statistics of the output
+        reinterpret_cast<float2*>(st_out)[(size_t)((n0 + c * CW) / 32) * st_ld + row] =
+            fold_granule(pk, 16, make_float2(0.f, 0.f));
     }
     if (ARLO_EPI_DIRECT) {
       if (row_ok) {
@@ -313,9 +391,11 @@ __global__ void __launch_bounds__(Roles<EW>::kThreads, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR, int M, int N, int K,
                const float* __restrict__ bias,
-               const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
-  constexpr bool kResidBuf = ARLO_RESID_TMA && EPI == EPI_BIAS_RESID;
-  using C = TcCfg<BN, false, 0, EW, kResidBuf>;
+               const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp,
+               const FoldArgs fa) {
+  constexpr bool kResidBuf = ARLO_RESID_TMA && is_resid(EPI);
+  constexpr int kColB = col_warp_bytes(EPI);
+  using C = TcCfg<BN, false, 0, EW, kResidBuf, kColB>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
   constexpr int kStagingBytes = C::kStagingBytes;
@@ -324,7 +404,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
-  uint8_t* rbuf = sStg + kEpiWarps * kBiasWarpBytes;  // (kResidBuf) the CTA's 128 x BN residual tile
+  uint8_t* rbuf = sStg + kEpiWarps * kColB;  // (kResidBuf) the CTA's 128 x BN residual tile
   uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
@@ -460,8 +540,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     // two warps sharing a quarter take one column half each.
     pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * kWarpStg;
-    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kBiasWarpBytes : stg + kStgBufs * kStgBytes);
+    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * (kStgBufs * kStgBytes + kColB);
+    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kColB : stg + kStgBufs * kStgBytes);
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -470,7 +550,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int m0 = tile_m(tile, num_m, num_n) * BM, n0 = tile_n(tile, num_m, num_n) * BN;
       uint4 rv0[CW / 8];
       if (!kResidBuf) prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
-      stage_bias<BN, kEpiGroups>(sbias, bias, n0, cg, lane);
+      stage_colv<BN, EPI, kEpiGroups>(sbias, bias, fa, n0, cg, lane);
+      // LayerNorm fold: this row's statistics (of A's rows, or of the residual rows)
+      float2 rowst = make_float2(0.f, -1.f);
+      if constexpr (EPI >= EPI_LNFOLD) {
+        const int grow = m0 + q * 32 + lane;
+        const int Hs = EPI == EPI_RESID_LN ? N : K;
+        if (fa.st_in != nullptr && grow < M) {
+          const float2 ms = fold_row_stats(fa.st_in, (size_t)grow * fa.st_in_stride, fa.st_ld, Hs / 32, Hs, fa.eps);
+          rowst = EPI == EPI_RESID_LN ? ms : make_float2(-ms.x * ms.y, ms.y);
+        } else if (EPI != EPI_RESID_LN) {
+          rowst = make_float2(0.f, 1.f);
+        }
+      }
       ptx::mbar_wait(&tfull[acc], acc_phase);
       if (kResidBuf) ptx::mbar_wait(rfull, it & 1);  // this tile's residual has landed
       ptx::tc_fence_after();
@@ -478,7 +570,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       uint64_t* te = &tempty[acc];
       epilogue_tile<BN, EPI, kEpiGroups>(tmem_base + acc * BN, q, cg, lane, m0 + q * 32, n0, M, ldr, bias, resid,
                                          &tmC, stg, sc, [te]() { ptx::mbar_arrive(te); }, outp, N, rv0,
-                                         kResidBuf ? rbuf : nullptr, sbias);
+                                         kResidBuf ? rbuf : nullptr, sbias, rowst, fa.st_out, fa.st_ld);
       if (kResidBuf) {  // the buffer is free once this warp's in-place TMA stores have read it
         if (lane == 0) ptx::bulk_wait_read<0>();
         __syncwarp();
@@ -511,9 +603,11 @@ __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(Roles<EW>::kThreads,
 gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                     const __grid_constant__ CUtensorMap tmC, const __grid_constant__ CUtensorMap tmR, int M, int N,
                     int K, const float* __restrict__ bias,
-                    const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp) {
-  constexpr bool kResidBuf = ARLO_RESID_TMA && EPI == EPI_BIAS_RESID;
-  using C = TcCfg<BN, true, 0, EW, kResidBuf>;
+                    const bf16* __restrict__ resid, int ldr, bf16* __restrict__ outp, const LnPrologue lnp,
+               const FoldArgs fa) {
+  constexpr bool kResidBuf = ARLO_RESID_TMA && is_resid(EPI);
+  constexpr int kColB = col_warp_bytes(EPI);
+  using C = TcCfg<BN, true, 0, EW, kResidBuf, kColB>;
   using R = Roles<EW>;
   constexpr int kEpiWarps = R::kEpi, kEpiGroups = R::kGroups, kProducerWarp = R::kProducer, kMmaWarp = R::kMma;
   constexpr int kStagingBytes = C::kStagingBytes;
@@ -522,7 +616,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   uint8_t* sA = smem;
   uint8_t* sB = smem + C::STAGES * C::A_BYTES;
   uint8_t* sStg = sB + C::STAGES * C::B_BYTES;
-  uint8_t* rbuf = sStg + kEpiWarps * kBiasWarpBytes;  // (kResidBuf) this CTA's 128 x BN residual rows
+  uint8_t* rbuf = sStg + kEpiWarps * kColB;  // (kResidBuf) this CTA's 128 x BN residual rows
   uint64_t* full = reinterpret_cast<uint64_t*>(sStg + kStagingBytes);
   uint64_t* empty = full + C::STAGES;
   uint64_t* tfull = empty + C::STAGES;
@@ -664,8 +758,8 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   } else {
     pdl_wait();
     const int q = warp & 3, cg = warp >> 2;
-    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * kWarpStg;
-    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kBiasWarpBytes : stg + kStgBufs * kStgBytes);
+    uint8_t* stg = kResidBuf ? nullptr : sStg + warp * (kStgBufs * kStgBytes + kColB);
+    float* sbias = reinterpret_cast<float*>(kResidBuf ? sStg + warp * kColB : stg + kStgBufs * kStgBytes);
     int sc = 0;
     int acc = 0;
     uint32_t acc_phase = 0;
@@ -674,7 +768,19 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       const int m0 = tile_m(tile, num_m, num_n) * 2 * BM + rank * BM, n0 = tile_n(tile, num_m, num_n) * BN;
       uint4 rv0[CW / 8];
       if (!kResidBuf) prefetch_first_resid<BN, EPI>(rv0, resid, m0 + q * 32, lane, n0, cg, M, ldr);
-      stage_bias<BN, kEpiGroups>(sbias, bias, n0, cg, lane);
+      stage_colv<BN, EPI, kEpiGroups>(sbias, bias, fa, n0, cg, lane);
+      // LayerNorm fold: this row's statistics (of A's rows, or of the residual rows)
+      float2 rowst = make_float2(0.f, -1.f);
+      if constexpr (EPI >= EPI_LNFOLD) {
+        const int grow = m0 + q * 32 + lane;
+        const int Hs = EPI == EPI_RESID_LN ? N : K;
+        if (fa.st_in != nullptr && grow < M) {
+          const float2 ms = fold_row_stats(fa.st_in, (size_t)grow * fa.st_in_stride, fa.st_ld, Hs / 32, Hs, fa.eps);
+          rowst = EPI == EPI_RESID_LN ? ms : make_float2(-ms.x * ms.y, ms.y);
+        } else if (EPI != EPI_RESID_LN) {
+          rowst = make_float2(0.f, 1.f);
+        }
+      }
       ptx::mbar_wait(&tfull[acc], acc_phase);
       if (kResidBuf) ptx::mbar_wait(rfull, it & 1);  // this tile's residual has landed
       ptx::tc_fence_after();
@@ -688,7 +794,7 @@ gemm_tc_pair_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
 #else
                                ptx::mbar_arrive_remote(te);
 #endif
-                             }, outp, N, rv0, kResidBuf ? rbuf : nullptr, sbias);
+                             }, outp, N, rv0, kResidBuf ? rbuf : nullptr, sbias, rowst, fa.st_out, fa.st_ld);
       if (kResidBuf) {
         if (lane == 0) ptx::bulk_wait_read<0>();
         __syncwarp();
@@ -743,7 +849,7 @@ template <int BN, int EPI>
 __global__ void __launch_bounds__(kSkThreads, 1)
 gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB, bf16* __restrict__ out,
                    int M, int N, int K, int a_rows, const float* __restrict__ bias, const bf16* __restrict__ resid,
-                   int ldr) {
+                   int ldr, const FoldArgs fa) {
   using C = SkCfg<BN>;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -823,15 +929,53 @@ gemm_skinny_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
     // epilogue: thread = row (TMEM lane), BN columns, straight 16-byte stores
     const int row = m0 + warp * 32 + lane;
     const bool row_ok = row < M;
+    float2 rowst = make_float2(0.f, -1.f);  // LayerNorm fold (see gemm_tc_kernel)
+    if constexpr (EPI >= EPI_LNFOLD) {
+      const int Hs = EPI == EPI_RESID_LN ? N : K;
+      if (fa.st_in != nullptr && row_ok) {
+        const float2 ms = fold_row_stats(fa.st_in, (size_t)row * fa.st_in_stride, fa.st_ld, Hs / 32, Hs, fa.eps);
+        rowst = EPI == EPI_RESID_LN ? ms : make_float2(-ms.x * ms.y, ms.y);
+      } else if (EPI != EPI_RESID_LN) {
+        rowst = make_float2(0.f, 1.f);
+      }
+    }
     ptx::mbar_wait(tfull, 0);
     ptx::tc_fence_after();
     const uint32_t t_row = tmem + ((uint32_t)(warp * 32) << 16);
+    float2 gst = make_float2(0.f, 0.f);
 #pragma unroll
     for (int c0 = 0; c0 < BN; c0 += 16) {
       uint32_t r[16];
       ptx::tmem_ld_32x32b_x16(t_row + c0, r);
       ptx::tmem_wait_ld();
-      if (row_ok) {
+      if (row_ok && EPI >= EPI_LNFOLD) {
+        uint32_t ru[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+        if (EPI == EPI_RESID_LN) {
+          const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0 + c0);
+          const uint4 u0 = ld_dep_v4(res4), u1 = ld_dep_v4(res4 + 1);
+          ru[0] = u0.x; ru[1] = u0.y; ru[2] = u0.z; ru[3] = u0.w; ru[4] = u1.x; ru[5] = u1.y; ru[6] = u1.z; ru[7] = u1.w;
+        }
+        uint32_t pk[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const int col = n0 + c0 + 2 * j;
+          const float2 a = make_float2(__uint_as_float(r[2 * j]), __uint_as_float(r[2 * j + 1]));
+          const float2 v0 = make_float2(__ldg(bias + col), __ldg(bias + col + 1));
+          const float2 v1 = fa.v1 ? make_float2(__ldg(fa.v1 + col), __ldg(fa.v1 + col + 1)) : f2(0.f);
+          const float2 v2 = EPI == EPI_RESID_LN && fa.v2 ? make_float2(__ldg(fa.v2 + col), __ldg(fa.v2 + col + 1)) : f2(0.f);
+          pk[j] = epi_fold_pair<EPI>(a, v0, v1, v2, ru[j], rowst);
+        }
+        uint4* o4 = reinterpret_cast<uint4*>(out + (size_t)row * N + n0 + c0);
+        o4[0] = make_uint4(pk[0], pk[1], pk[2], pk[3]);
+        o4[1] = make_uint4(pk[4], pk[5], pk[6], pk[7]);
+        if (EPI == EPI_RESID_LN && fa.st_out != nullptr) {  // 32-column granules: two 16-column steps
+          gst = fold_granule(pk, 8, gst);
+          if (c0 & 16) {
+            reinterpret_cast<float2*>(fa.st_out)[(size_t)((n0 + c0) / 32) * fa.st_ld + row] = gst;
+            gst = make_float2(0.f, 0.f);
+          }
+        }
+      } else if (row_ok) {
         uint4 rv[2];
         if (EPI == EPI_BIAS_RESID) {
           const uint4* res4 = reinterpret_cast<const uint4*>(resid + (size_t)row * ldr + n0 + c0);
@@ -1177,19 +1321,19 @@ EncodeTiledFn get_encode_fn() {
 
 template <int BN, int EPI, bool PAIR, int EW>
 cudaError_t launch_cfg_ew(const TcGemmPlan& p, cudaStream_t s) {
-  using C = TcCfg<BN, PAIR, 0, EW, ARLO_RESID_TMA && EPI == EPI_BIAS_RESID>;
+  using C = TcCfg<BN, PAIR, 0, EW, ARLO_RESID_TMA && is_resid(EPI), col_warp_bytes(EPI)>;
   auto kern = PAIR ? gemm_tc_pair_kernel<BN, EPI, EW> : gemm_tc_kernel<BN, EPI, EW>;
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [&] {
     return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
   if (e != cudaSuccess) return e;
   return launch_k(kern, dim3(p.grid), dim3(Roles<EW>::kThreads), C::SMEM, s, p.tmA, p.tmB, p.tmC, p.tmR, p.M, p.N,
-                  p.K, p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out, p.lnp);
+                  p.K, p.bias, (const bf16*)p.resid, p.ldr, (bf16*)p.out, p.lnp, p.fold);
 }
 
 template <int BN, int EPI, bool PAIR>
 cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
-  if constexpr (EPI == EPI_BIAS_GELU) {
+  if constexpr (EPI == EPI_BIAS_GELU || EPI == EPI_LNFOLD_GELU) {
     if (p.ew == 12) return launch_cfg_ew<BN, EPI, PAIR, 12>(p, s);
   }
   return launch_cfg_ew<BN, EPI, PAIR, kEpiWarps>(p, s);
@@ -1201,6 +1345,9 @@ cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
     case EPI_BIAS: return launch_cfg<BN, EPI_BIAS, PAIR>(p, s);
     case EPI_BIAS_GELU: return launch_cfg<BN, EPI_BIAS_GELU, PAIR>(p, s);
     case EPI_BIAS_RESID: return launch_cfg<BN, EPI_BIAS_RESID, PAIR>(p, s);
+    case EPI_LNFOLD: return launch_cfg<BN, EPI_LNFOLD, PAIR>(p, s);
+    case EPI_LNFOLD_GELU: return launch_cfg<BN, EPI_LNFOLD_GELU, PAIR>(p, s);
+    case EPI_RESID_LN: return launch_cfg<BN, EPI_RESID_LN, PAIR>(p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -1214,7 +1361,7 @@ cudaError_t launch_skinny_cfg(const TcGemmPlan& p, cudaStream_t s) {
     return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::SMEM); });
   if (e != cudaSuccess) return e;
   return launch_k(kern, dim3(p.N / BN, (p.M + BM - 1) / BM), dim3(kSkThreads), C::SMEM, s, p.tmA, p.tmB,
-                  (bf16*)p.out, p.M, p.N, p.K, p.a_rows, p.bias, (const bf16*)p.resid, p.ldr);
+                  (bf16*)p.out, p.M, p.N, p.K, p.a_rows, p.bias, (const bf16*)p.resid, p.ldr, p.fold);
 }
 
 template <int BN>
@@ -1223,6 +1370,9 @@ cudaError_t launch_skinny_bn(const TcGemmPlan& p, cudaStream_t s) {
     case EPI_BIAS: return launch_skinny_cfg<BN, EPI_BIAS>(p, s);
     case EPI_BIAS_GELU: return launch_skinny_cfg<BN, EPI_BIAS_GELU>(p, s);
     case EPI_BIAS_RESID: return launch_skinny_cfg<BN, EPI_BIAS_RESID>(p, s);
+    case EPI_LNFOLD: return launch_skinny_cfg<BN, EPI_LNFOLD>(p, s);
+    case EPI_LNFOLD_GELU: return launch_skinny_cfg<BN, EPI_LNFOLD_GELU>(p, s);
+    case EPI_RESID_LN: return launch_skinny_cfg<BN, EPI_RESID_LN>(p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -1332,9 +1482,10 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
     return tc_plan_gemm_splitk(p, M, N, K, A, lda, W, bias, resid, ldr, out, epi, force_bn - kSplitKCode);
   const int choice = force_bn ? force_bn : tc_choose_bn(M, N, K);
   if (choice > kSkinnyCode) {
-    const int bn = choice - kSkinnyCode;
+    int bn = choice - kSkinnyCode;
+    if (epi == EPI_RESID_LN && bn == 16) bn = 32;  // statistics granule: 32 columns of one CTA
     if ((bn != 16 && bn != 32 && bn != 64) || N % bn) return false;
-    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->splitk = false; p->lnp = LnPrologue{}; p->epi = epi; p->ln = false; p->ew = 4;
+    p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = true; p->splitk = false; p->fold = FoldArgs{}; p->lnp = LnPrologue{}; p->epi = epi; p->ln = false; p->ew = 4;
     p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
     p->a_rows = M < BM ? ((M + 7) & ~7) : BM;
     p->grid = (N / bn) * ((M + BM - 1) / BM);
@@ -1356,12 +1507,14 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
 #ifndef ARLO_GELU_EW12_MAX_M
 #define ARLO_GELU_EW12_MAX_M 8192  // A/B hook: 0 keeps 8 epilogue warps everywhere
 #endif
-  p->ew = (epi == EPI_BIAS_GELU && M <= ARLO_GELU_EW12_MAX_M) ? 12 : kEpiWarps;
+  p->ew = ((epi == EPI_BIAS_GELU || epi == EPI_LNFOLD_GELU) && M <= ARLO_GELU_EW12_MAX_M) ? 12 : kEpiWarps;
+  p->fold = FoldArgs{};
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, BM, 128, (uint64_t)lda)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, pair ? bn / 2 : bn, 128)) return false;
   if (!encode_tmap_bf16_2d(&p->tmC, out, (uint64_t)N, (uint64_t)M, CW, 32, CW * 2)) return false;
   // residual rows (stride ldr), {32 columns x 128 rows} boxes in the output staging layout
-  if (epi == EPI_BIAS_RESID && !encode_tmap_bf16_2d(&p->tmR, resid, (uint64_t)N, (uint64_t)M, CW, BM, CW * 2, (uint64_t)ldr))
+  if ((epi == EPI_BIAS_RESID || epi == EPI_RESID_LN) &&
+      !encode_tmap_bf16_2d(&p->tmR, resid, (uint64_t)N, (uint64_t)M, CW, BM, CW * 2, (uint64_t)ldr))
     return false;
   return true;
 }
@@ -1409,7 +1562,7 @@ bool tc_plan_gemm_ln(TcGemmPlan* p, int M, int N, int K, const void* A, const vo
   if (N == 128 && (128 / kEpiGroups) % 32 == 0 && 128 % kEpiGroups == 0) bn = 128;
   if (!bn) return false;
   const int nt = N / bn;
-  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->splitk = false; p->lnp = LnPrologue{}; p->epi = EPI_BIAS_RESID; p->ln = true;
+  p->M = M; p->N = N; p->K = K; p->BN = bn; p->pair = false; p->skinny = false; p->splitk = false; p->lnp = LnPrologue{}; p->epi = EPI_BIAS_RESID; p->ln = true; p->fold = FoldArgs{};
   p->ew = kEpiWarps;
   p->bias = bias; p->resid = resid; p->ldr = N; p->out = out; p->gamma = gamma; p->beta = beta; p->eps = eps;
   const int num_m = (M + BM - 1) / BM;

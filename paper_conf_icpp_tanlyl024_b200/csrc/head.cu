@@ -40,7 +40,7 @@ __device__ __forceinline__ void unpack16(const uint4& u, float* f) {
 template <typename T, int MAXV>
 __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const T* __restrict__ x,
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
-                                                     float* __restrict__ pooled) {
+                                                     float* __restrict__ pooled, const HeadLn ln) {
   // [kRows][nvec] raw 16-byte vectors of T: lane-consecutive vectors are bank-conflict free
   // (fp32 staging with 8 floats per lane put lanes 4 apart on the same banks: 8-way STS,
   // 2x LDS.128 wavefronts; the pooler was shared-memory bound at 22 us for b = 32)
@@ -60,6 +60,14 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
   pdl_wait();
   const int b0 = blockIdx.y * kRows;
   const int nb = min(kRows, B - b0);
+  // LayerNorm fold: the CLS rows are the last layer's un-normalised output y; normalise them while
+  // staging (x = bf16((y - mean) rstd * gamma + beta), layernorm.cuh's per-element arithmetic)
+  __shared__ float2 s_ms[kRows];
+  if (sizeof(T) == 2 && ln.st != nullptr) {
+    if (threadIdx.x < nb)
+      s_ms[threadIdx.x] = fold_row_stats(ln.st, (size_t)(b0 + threadIdx.x) * L, ln.st_ld, H / 32, H, ln.eps);
+    __syncthreads();
+  }
   {
     constexpr int kPer = MAXV;  // kRows * nvec / 256 <= MAXV vectors per thread
     static_assert(kRows * 32 == 256, "one staged vector per thread per 32 of a row");
@@ -74,6 +82,20 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
     for (int t = 0; t < kPer; ++t) {
       const int i = threadIdx.x + 256 * t;
       const int r = i / nvec, c = i - r * nvec;
+      if (sizeof(T) == 2 && ln.st != nullptr && r < nb) {
+        const float2 ms = s_ms[r];
+        uint32_t w[4] = {u[t].x, u[t].y, u[t].z, u[t].w};
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const int col = c * 8 + 2 * e;
+          const float2 y = unpack_bf16x2(w[e]);
+          const float o0 = __fmaf_rn(__fmul_rn(__fsub_rn(y.x, ms.x), ms.y), __ldg(ln.gamma + col), __ldg(ln.beta + col));
+          const float o1 = __fmaf_rn(__fmul_rn(__fsub_rn(y.y, ms.x), ms.y), __ldg(ln.gamma + col + 1),
+                                     __ldg(ln.beta + col + 1));
+          w[e] = pack_bf16x2(o0, o1);
+        }
+        u[t] = make_uint4(w[0], w[1], w[2], w[3]);
+      }
       if (r < kRows) xs[r * nvec + c] = r < nb ? u[t] : make_uint4(0, 0, 0, 0);
     }
   }
@@ -150,7 +172,7 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
 
 template <typename T, int MAXV>
 cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
-                     const float* b_c, float* pooled, float* logits, cudaStream_t s) {
+                     const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
   const size_t smem = (size_t)kRows * H * sizeof(T);
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [] {
@@ -163,7 +185,7 @@ cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p,
   if (e != cudaSuccess) return e;
   dim3 grid((H + kFeat - 1) / kFeat, (B + kRows - 1) / kRows);
   e = launch_k(pooler_kernel<T, MAXV>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p,
-                           b_p, pooled);
+                           b_p, pooled, ln);
   if (e != cudaSuccess) return e;
   return launch_k(classifier_kernel<T, MAXV>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c,
                   b_c, logits);
@@ -171,27 +193,27 @@ cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p,
 
 template <typename T>
 cudaError_t launch_dt(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
-                      const float* b_c, float* pooled, float* logits, cudaStream_t s) {
+                      const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
   const int maxv = (H * (int)sizeof(T) + 511) / 512;
   switch (maxv) {
-    case 1: return launch_t<T, 1>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    case 2: return launch_t<T, 2>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    case 3: return launch_t<T, 3>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    case 4: return launch_t<T, 4>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    case 5: case 6: return launch_t<T, 6>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    case 7: case 8: return launch_t<T, 8>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
-    default: return launch_t<T, 16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+    case 1: return launch_t<T, 1>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 2: return launch_t<T, 2>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 3: return launch_t<T, 3>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 4: return launch_t<T, 4>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 5: case 6: return launch_t<T, 6>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 7: case 8: return launch_t<T, 8>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    default: return launch_t<T, 16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
   }
 }
 
 }  // namespace
 
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p,
-                        const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s) {
+                        const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
   if (B <= 0) return cudaSuccess;
   if (H > 2048 || H % 8) return cudaErrorInvalidValue;
-  return dt == DT_BF16 ? launch_dt<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s)
-                       : launch_dt<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s);
+  return dt == DT_BF16 ? launch_dt<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln)
+                       : launch_dt<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, HeadLn{});
 }
 
 }  // namespace arlo

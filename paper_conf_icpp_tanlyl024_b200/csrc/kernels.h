@@ -11,7 +11,32 @@
 namespace arlo {
 
 enum DType { DT_BF16 = 0, DT_FP32 = 1 };
-enum Epi { EPI_BIAS = 0, EPI_BIAS_GELU = 1, EPI_BIAS_RESID = 2 };
+enum Epi {
+  EPI_BIAS = 0, EPI_BIAS_GELU = 1, EPI_BIAS_RESID = 2,
+  // LayerNorm folded into the GEMMs (runtime.cu, ARLO_NO_LN_FOLD=1 disables):
+  //  EPI_LNFOLD / _GELU: A = y (a residual sum, NOT normalised), W' = W * gamma (column scaled),
+  //    out = rstd_r * acc - rstd_r * mu_r * s_n + c_n (s = W' row sums, c = W beta + b), mu_r and
+  //    rstd_r from the per-row statistics of y (FoldArgs::st_in), then GELU for _GELU;
+  //  EPI_RESID_LN: out = (acc + b_n) + LN(r) with LN(r) = (r - mu_r) * rstd_r * gamma_n + beta_n
+  //    computed on the fly from the residual rows r and their statistics (plain r when st_in is
+  //    null), and the statistics of the bf16 output written to FoldArgs::st_out.
+  EPI_LNFOLD = 3, EPI_LNFOLD_GELU = 4, EPI_RESID_LN = 5
+};
+
+// Row statistics of an activation y[M, H] for the LayerNorm fold: per row, per 32-column granule
+// g, the fp32 sums (sum_j y, sum_j y^2) over its 32 bf16 values in column order, stored
+// granule-major st[g][row][2] with a fixed row capacity `st_ld` (a warp's 32 rows are contiguous:
+// coalesced stores by the producing epilogue and loads by the consumer).  A consumer adds the
+// H/32 granules in order: every kernel and tile shape produces the same bits.
+struct FoldArgs {
+  const float* v1;    // EPI_LNFOLD*: c [N];  EPI_RESID_LN: gamma [N] of the residual's LayerNorm
+  const float* v2;    // EPI_RESID_LN: beta [N]
+  const float* st_in; // EPI_LNFOLD*: statistics of A's rows (K/32 granules); EPI_RESID_LN: of the residual rows
+  int st_in_stride;   // row stride of st_in in rows (1, or L for the CLS rows of a full layer)
+  float* st_out;      // EPI_RESID_LN: statistics of the output rows (N/32 granules)
+  float eps;
+  int st_ld;          // rows per granule plane of st_in and st_out (their allocated row count)
+};
 
 int num_sms();
 int set_gemm_trace(unsigned long long* buf);  // profiling hook, nullptr = off
@@ -24,6 +49,9 @@ cudaError_t launch_embed_ln(DType dt, int B, int L, int H, int vocab, const int3
                             int32_t* err_flag, cudaStream_t s);
 cudaError_t launch_layernorm(DType dt, int M, int H, const void* in, const float* g,
                              const float* b, float eps, void* out, cudaStream_t s);
+// LayerNorm fold: W' = bf16(W * gamma) (column scale), s = row sums of W', c = W beta + b (see EPI_LNFOLD)
+cudaError_t launch_fold_weights(int N, int K, const void* W, const float* gamma, const float* beta, const float* b,
+                                void* Wf, float* s, float* c, cudaStream_t st);
 
 // ---- a2/a4/a6/a7: GEMM + fused epilogue ----------------------------------------------------
 // LayerNorm run as the prologue of a persistent GEMM (layernorm.cuh): x = LN(y) over `rows`
@@ -64,6 +92,7 @@ struct TcGemmPlan {
   int ldr;  // residual row stride (elements)
   void* out;
   LnPrologue lnp;  // (bias / GELU epilogues of the persistent tile kernels only)
+  FoldArgs fold;   // EPI_LNFOLD, EPI_LNFOLD_GELU, EPI_RESID_LN
 };
 // Attach a LayerNorm prologue to a planned GEMM whose A operand is lnp.x; false if the plan's
 // kernel cannot run it (skinny / split-K / residual epilogue / H > 1024).
@@ -113,9 +142,18 @@ bool attn_plan(AttnPlan* p, DType dt, int B, int L, int heads, const void* qkv, 
 cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cudaStream_t s);
 
 // ---- a9: CLS pooler + classifier ----------------------------------------------------------
+// ln: optional LayerNorm applied to the CLS rows on the fly (the LN fold leaves the last layer's
+// output un-normalised): x = bf16((y - mu) rstd * gamma + beta), mu / rstd from the row statistics
+struct HeadLn {
+  const float* st;  // granule statistics [H/32][st_ld][2] of y (row of sequence i: i * L), or nullptr
+  const float* gamma;
+  const float* beta;
+  float eps;
+  int st_ld;
+};
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p,
                         const float* b_p, const void* w_c, const float* b_c, float* pooled,
-                        float* logits, cudaStream_t s);
+                        float* logits, cudaStream_t s, HeadLn ln = HeadLn{});
 
 // ---- fused persistent forward (encoder_fused.cu): the whole batch-1 forward as one kernel ----
 struct FusedPlanImpl;

@@ -86,10 +86,24 @@ static int check_device(int device) {
 using namespace arlo;
 
 // ------------------------------------------------------------------------ weights
+// LayerNorm-folded copies of the weights that consume a LayerNorm output (launch_fold_weights):
+// per layer l, the QKV projection folded with layer l-1's LN2 (l >= 1) and FFN1 with layer l's LN1.
+struct FoldLayer {
+  void* wq = nullptr;  // [3H, H] bf16 = W_qkv * gamma2(l-1)
+  float* sq = nullptr;  // [3H] row sums of wq
+  float* cq = nullptr;  // [3H] W_qkv beta2(l-1) + b_qkv
+  void* w1 = nullptr;   // [F, H] bf16 = W_1 * gamma1(l)
+  float* s1 = nullptr;
+  float* c1 = nullptr;
+};
+
 struct arlo_weights {
   int device;
   arlo_model_config cfg;
   std::vector<const void*> t;  // canonical order
+  std::mutex fold_mu;          // the fold cache is built once, by the first runtime that needs it
+  void* fold_buf = nullptr;
+  std::vector<FoldLayer> fold;
   const void* word() const { return t[0]; }
   const void* pos() const { return t[1]; }
   const void* type() const { return t[2]; }
@@ -149,7 +163,53 @@ extern "C" int arlo_weights_create(int32_t device, const arlo_model_config* cfg,
   return ARLO_OK;
 }
 
-extern "C" void arlo_weights_destroy(arlo_weights* w) { delete w; }
+extern "C" void arlo_weights_destroy(arlo_weights* w) {
+  if (w && w->fold_buf) {
+    DeviceGuard g(w->device);
+    cudaFree(w->fold_buf);
+  }
+  delete w;
+}
+
+// Build the LayerNorm-folded weight copies (once per weight set).  bf16 only.
+static int ensure_fold(arlo_weights* w, cudaStream_t s) {
+  std::lock_guard<std::mutex> lk(w->fold_mu);
+  if (w->fold_buf) return ARLO_OK;
+  const arlo_model_config& c = w->cfg;
+  const size_t H = c.hidden, F = c.ffn, nl = c.layers;
+  auto al = [](size_t x) { return (x + 255) & ~size_t(255); };
+  const size_t per = al(6 * H * H) + 3 * al(4 * 3 * H) + al(2 * F * H) + 2 * al(4 * F);
+  void* buf = nullptr;
+  cudaError_t e = cudaMalloc(&buf, per * nl);
+  if (e != cudaSuccess) return set_error(ARLO_ENOMEM, "LayerNorm-fold weights (%zu bytes): %s", per * nl, cudaGetErrorString(e));
+  std::vector<FoldLayer> fl(nl);
+  for (size_t l = 0; l < nl; ++l) {
+    char* p = (char*)buf + per * l;
+    FoldLayer& f = fl[l];
+    f.wq = p; p += al(6 * H * H);
+    f.sq = (float*)p; p += al(4 * 3 * H);
+    f.cq = (float*)p; p += al(4 * 3 * H);
+    p += al(4 * 3 * H);
+    f.w1 = p; p += al(2 * F * H);
+    f.s1 = (float*)p; p += al(4 * F);
+    f.c1 = (float*)p;
+    if (l >= 1)
+      e = launch_fold_weights(3 * H, H, w->lt(l, LW_QKV), (const float*)w->lt(l - 1, LN2_G), (const float*)w->lt(l - 1, LN2_B),
+                              (const float*)w->lt(l, LB_QKV), f.wq, f.sq, f.cq, s);
+    if (e == cudaSuccess)
+      e = launch_fold_weights(F, H, w->lt(l, LW_1), (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
+                              (const float*)w->lt(l, LB_1), f.w1, f.s1, f.c1, s);
+    if (e != cudaSuccess) break;
+  }
+  if (e == cudaSuccess) e = cudaStreamSynchronize(s);
+  if (e != cudaSuccess) {
+    cudaFree(buf);
+    return cuda_fail(e, "LayerNorm-fold weights");
+  }
+  w->fold_buf = buf;
+  w->fold = std::move(fl);
+  return ARLO_OK;
+}
 
 // ------------------------------------------------------------------------ runtime
 struct LayerPlans {
@@ -180,12 +240,17 @@ struct Bucket {
 
 struct arlo_runtime {
   int L = 0, max_batch = 0, device = 0;
-  // latency family (ARLO_RUNTIME_LATENCY): every GEMM is the split-K weight-streaming kernel
-  // (gemm_splitk.cu); the throughput family uses the tile kernels chosen per bucket
+  // split-K family (ARLO_RUNTIME_SPLITK): every GEMM is the split-K weight-streaming kernel
+  // (gemm_splitk.cu); the other families use the tile kernels chosen per bucket
   bool latency = false;
   // fused family (ARLO_RUNTIME_FUSED): one persistent kernel per forward (encoder_fused.cu)
   bool fused = false;
-  const arlo_weights* w = nullptr;
+  // LayerNorm fold (throughput family, bf16; ARLO_NO_LN_FOLD=1 disables): no LayerNorm kernels;
+  // the residual GEMMs emit row statistics (S1 after the out-projection, S2 after FFN2), the
+  // consuming GEMMs run on folded weights, the next residual GEMM and the pooler normalise on the fly
+  bool ln_fold = false;
+  float *S1 = nullptr, *S2 = nullptr;  // [max_batch * L][H/32][2] granule statistics
+  arlo_weights* w = nullptr;
   DType dt = DT_BF16;
   cudaStream_t own_stream = nullptr, stream = nullptr;
   // arena (one allocation)
@@ -209,6 +274,14 @@ static int bucket_index(const arlo_runtime* rt, int n) {
   return -1;
 }
 
+// Timing experiments only (tools/forward_costs.py): ARLO_DEBUG_SKIP=ln,attn drops those kernels
+// from the captured forward (wrong results) so that the forward-time difference is their cost
+// inside the graph, where every kernel's prologue overlaps its predecessor (PDL).
+static bool debug_skip(const char* what) {
+  const char* e = getenv("ARLO_DEBUG_SKIP");
+  return e != nullptr && strstr(e, what) != nullptr;
+}
+
 // Enqueue one forward at bucket size b (the body every graph captures).
 static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
   const arlo_weights* w = rt->w;
@@ -222,6 +295,24 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
   ARLO_CUDA(launch_embed_ln(dt, b, L, H, c.vocab, rt->ids, rt->lengths, w->word(), w->pos(), w->type(), w->emb_g(),
                             w->emb_b(), c.ln_eps, rt->X, rt->err, s),
             "embed_ln launch");
+  if (rt->ln_fold) {
+    // LayerNorm fold: 4 GEMMs + attention per layer, no LayerNorm kernel (plans carry the fold)
+    for (int l = 0; l < c.layers; ++l) {
+      const bool cls = bk.cls_prune && l == c.layers - 1;
+      ARLO_CUDA(tc_launch_gemm(bk.plans[l].qkv, s), "qkv gemm launch");
+      if (!debug_skip("attn")) ARLO_CUDA(attn_launch(cls ? bk.attn_cls : bk.attn, rt->lengths, rt->O, s), "attention launch");
+      const LayerPlans& p = cls ? bk.cls : bk.plans[l];
+      ARLO_CUDA(tc_launch_gemm(p.o, s), "out-proj gemm launch");
+      ARLO_CUDA(tc_launch_gemm(p.f1, s), "ffn1 gemm launch");
+      ARLO_CUDA(tc_launch_gemm(p.f2, s), "ffn2 gemm launch");
+    }
+    const int l = c.layers - 1;
+    HeadLn hl{rt->S2, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B), c.ln_eps, rt->max_batch * L};
+    ARLO_CUDA(launch_head(dt, b, bk.cls_prune ? 1 : L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1),
+                          w->hd(2), (const float*)w->hd(3), rt->pooled, rt->logits, s, hl),
+              "head launch");
+    return ARLO_OK;
+  }
   for (int l = 0; l < c.layers; ++l) {
     if (bk.cls_prune && l == c.layers - 1) {
       // last layer on the b CLS rows only (see Bucket::cls_prune)
@@ -245,7 +336,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  rt->QKV, EPI_BIAS, s),
                 "qkv gemm launch");
     }
-    ARLO_CUDA(attn_launch(bk.attn, rt->lengths, rt->O, s), "attention launch");
+    if (!debug_skip("attn")) ARLO_CUDA(attn_launch(bk.attn, rt->lengths, rt->O, s), "attention launch");
     if (dt == DT_BF16) {
       ARLO_CUDA(tc_launch_gemm(bk.plans[l].o, s), "out-proj gemm launch");
     } else {
@@ -253,7 +344,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "out-proj gemm launch");
     }
-    if (!bk.fused_ln && !(l < (int)bk.ln1_in_f1.size() && bk.ln1_in_f1[l]))
+    if (!bk.fused_ln && !(l < (int)bk.ln1_in_f1.size() && bk.ln1_in_f1[l]) && !debug_skip("ln"))
       ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN1_G), (const float*)w->lt(l, LN1_B),
                                  c.ln_eps, rt->X, s),
                 "ln1 launch");
@@ -268,7 +359,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
                                  EPI_BIAS_RESID, s),
                 "ffn2 gemm launch");
     }
-    if (!bk.fused_ln && !(l < (int)bk.ln2_in_qkv.size() && bk.ln2_in_qkv[l]))
+    if (!bk.fused_ln && !(l < (int)bk.ln2_in_qkv.size() && bk.ln2_in_qkv[l]) && !debug_skip("ln"))
       ARLO_CUDA(launch_layernorm(dt, M, H, rt->Y, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B),
                                  c.ln_eps, rt->X, s),
                 "ln2 launch");
@@ -367,8 +458,81 @@ static int plan_bucket_latency(arlo_runtime* rt, Bucket& bk) {
   return ARLO_OK;
 }
 
+// LayerNorm-fold plans (see arlo_runtime::ln_fold).  Per layer l:
+//   QKV:  l = 0 plain on x (the embedding LayerNorm's output); l >= 1 EPI_LNFOLD on y2(l-1) (X) with the
+//         folded weights of LN2(l-1) and statistics S2
+//   out:  EPI_RESID_LN, residual X = y2(l-1) normalised on the fly with LN2(l-1) and S2 (plain x for
+//         l = 0) -> y1 (Y) and its statistics S1
+//   FFN1: EPI_LNFOLD_GELU on y1 with the folded weights of LN1(l) and S1 -> F
+//   FFN2: EPI_RESID_LN, residual y1 normalised with LN1(l) and S1 -> y2(l) (X) and S2
+// The pooler normalises the CLS rows of y2(last) with LN2(last) and S2.
+static int plan_bucket_fold(arlo_runtime* rt, Bucket& bk) {
+  arlo_weights* w = rt->w;
+  const arlo_model_config& c = w->cfg;
+  const int b = bk.b, L = rt->L, M = b * L, H = c.hidden, F = c.ffn;
+  const float eps = c.ln_eps;
+  bk.plans.resize(c.layers);
+  bk.fused_ln = false;
+  const FoldLayer& f0 = w->fold[c.layers > 1 ? 1 : 0];
+  cudaStream_t ts = rt->own_stream;
+  // tile codes timed on layer 0's shapes (the folded epilogues' costs)
+  const int t_qkv = pick_tile(M, 3 * H, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, 3 * H, H, rt->X, c.layers > 1 ? f0.wq : w->lt(0, LW_QKV),
+                        c.layers > 1 ? f0.sq : (const float*)w->lt(0, LB_QKV), nullptr, rt->QKV,
+                        c.layers > 1 ? EPI_LNFOLD : EPI_BIAS, code); });
+  const int t_f1 = pick_tile(M, F, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, F, H, rt->Y, w->fold[0].w1, w->fold[0].s1, nullptr, rt->F, EPI_LNFOLD_GELU, code); });
+  const int t_o = pick_tile(M, H, H, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X, rt->Y, EPI_RESID_LN,
+                        code); });
+  const int t_f2 = pick_tile(M, H, F, ts, [&](TcGemmPlan* p, int code) {
+    return tc_plan_gemm(p, M, H, F, rt->F, w->lt(0, LW_2), (const float*)w->lt(0, LB_2), rt->Y, rt->X, EPI_RESID_LN,
+                        code); });
+  if (cudaStreamSynchronize(ts) != cudaSuccess) return set_error(ARLO_ECUDA, "tile selection failed");
+  bk.tiles[0] = t_qkv; bk.tiles[1] = t_o; bk.tiles[2] = t_f1; bk.tiles[3] = t_f2;
+  auto ln_g = [&](int l, int k) { return (const float*)w->lt(l, k); };
+  for (int l = 0; l < c.layers; ++l) {
+    LayerPlans& p = bk.plans[l];
+    const FoldLayer& f = w->fold[l];
+    bool ok = l == 0 ? tc_plan_gemm(&p.qkv, M, 3 * H, H, rt->X, w->lt(0, LW_QKV), (const float*)w->lt(0, LB_QKV),
+                                    nullptr, rt->QKV, EPI_BIAS, t_qkv)
+                     : tc_plan_gemm(&p.qkv, M, 3 * H, H, rt->X, f.wq, f.sq, nullptr, rt->QKV, EPI_LNFOLD, t_qkv);
+    ok = ok &&
+         tc_plan_gemm(&p.o, M, H, H, rt->O, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X, rt->Y, EPI_RESID_LN, t_o) &&
+         tc_plan_gemm(&p.f1, M, F, H, rt->Y, f.w1, f.s1, nullptr, rt->F, EPI_LNFOLD_GELU, t_f1) &&
+         tc_plan_gemm(&p.f2, M, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->Y, rt->X, EPI_RESID_LN, t_f2);
+    if (!ok) return set_error(ARLO_ECUDA, "LayerNorm-fold plan: tensor-map encoding failed");
+    if (l >= 1) p.qkv.fold = FoldArgs{f.cq, nullptr, rt->S2, 1, nullptr, eps, rt->max_batch * rt->L};
+    p.o.fold = FoldArgs{l >= 1 ? ln_g(l - 1, LN2_G) : nullptr, l >= 1 ? ln_g(l - 1, LN2_B) : nullptr,
+                        l >= 1 ? rt->S2 : nullptr, 1, rt->S1, eps, rt->max_batch * rt->L};
+    p.f1.fold = FoldArgs{f.c1, nullptr, rt->S1, 1, nullptr, eps, rt->max_batch * rt->L};
+    p.f2.fold = FoldArgs{ln_g(l, LN1_G), ln_g(l, LN1_B), rt->S1, 1, rt->S2, eps, rt->max_batch * rt->L};
+  }
+  bk.cls_prune = getenv("ARLO_NO_CLS_PRUNE") == nullptr;
+  if (bk.cls_prune) {
+    // last layer on the b CLS rows: out-projection reads rows i*L of the context and of X (and of
+    // S2); everything after it is compact [b, .]
+    const int l = c.layers - 1;
+    const FoldLayer& f = w->fold[l];
+    const bool ok =
+        attn_plan(&bk.attn_cls, rt->dt, b, L, c.heads, rt->QKV, 1) &&
+        tc_plan_gemm_strided(&bk.cls.o, b, H, H, rt->O, L * H, w->lt(l, LW_O), (const float*)w->lt(l, LB_O), rt->X,
+                             L * H, rt->Y, EPI_RESID_LN, 0) &&
+        tc_plan_gemm(&bk.cls.f1, b, F, H, rt->Y, f.w1, f.s1, nullptr, rt->F, EPI_LNFOLD_GELU, 0) &&
+        tc_plan_gemm(&bk.cls.f2, b, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->Y, rt->X,
+                     EPI_RESID_LN, 0);
+    if (!ok) return set_error(ARLO_ECUDA, "CLS-row LayerNorm-fold plan: tensor-map encoding failed");
+    bk.cls.o.fold = FoldArgs{l >= 1 ? ln_g(l - 1, LN2_G) : nullptr, l >= 1 ? ln_g(l - 1, LN2_B) : nullptr,
+                             l >= 1 ? rt->S2 : nullptr, L, rt->S1, eps, rt->max_batch * rt->L};
+    bk.cls.f1.fold = FoldArgs{f.c1, nullptr, rt->S1, 1, nullptr, eps, rt->max_batch * rt->L};
+    bk.cls.f2.fold = FoldArgs{ln_g(l, LN1_G), ln_g(l, LN1_B), rt->S1, 1, rt->S2, eps, rt->max_batch * rt->L};
+  }
+  return ARLO_OK;
+}
+
 static int plan_bucket(arlo_runtime* rt, Bucket& bk) {
   if (rt->latency) return plan_bucket_latency(rt, bk);
+  if (rt->ln_fold) return plan_bucket_fold(rt, bk);
   const arlo_weights* w = rt->w;
   const arlo_model_config& c = w->cfg;
   const int M = bk.b * rt->L, H = c.hidden, F = c.ffn;
@@ -482,7 +646,8 @@ extern "C" int arlo_runtime_create(int32_t L, int32_t max_batch, const arlo_weig
 }
 
 extern "C" int32_t arlo_runtime_family(const arlo_runtime* rt) {
-  return rt ? (rt->fused ? (int32_t)ARLO_RUNTIME_FUSED : rt->latency ? (int32_t)ARLO_RUNTIME_LATENCY : (int32_t)ARLO_RUNTIME_THROUGHPUT)
+  return rt ? (rt->fused ? (int32_t)ARLO_RUNTIME_FUSED : rt->latency ? (int32_t)ARLO_RUNTIME_SPLITK
+                : rt->ln_fold ? (int32_t)ARLO_RUNTIME_LATENCY : (int32_t)ARLO_RUNTIME_THROUGHPUT)
             : ARLO_EINVAL;
 }
 
@@ -491,7 +656,7 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   clear_error();
   if (!w || !out) return set_error(ARLO_EINVAL, "arlo_runtime_create: null argument");
   if (family != ARLO_RUNTIME_DEFAULT && family != ARLO_RUNTIME_LATENCY && family != ARLO_RUNTIME_THROUGHPUT &&
-      family != ARLO_RUNTIME_FUSED)
+      family != ARLO_RUNTIME_FUSED && family != ARLO_RUNTIME_SPLITK)
     return set_error(ARLO_EINVAL, "arlo_runtime_create_ex: unknown runtime family %d", family);
   const arlo_model_config& c = w->cfg;
   if (L < 16 || L % 16 || L > c.max_pos)
@@ -508,14 +673,17 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   if (!rt) return set_error(ARLO_ENOMEM, "out of host memory");
   rt->L = L;
   rt->max_batch = max_batch;
-  rt->w = w;
+  rt->w = const_cast<arlo_weights*>(w);  // (the LayerNorm-fold cache is built lazily inside it)
   rt->device = w->device;
   rt->dt = c.dtype == ARLO_BF16 ? DT_BF16 : DT_FP32;
   // batch-1 runtimes (the paper's setting) stream weights with split-K GEMMs
   // (DEFAULT = THROUGHPUT: measured on B200, the split-K family does not shorten a batch-1 forward;
   // its 87 dependent kernels cost ~4.5 us each whatever the GEMM kernel)
-  rt->latency = rt->dt == DT_BF16 && family == ARLO_RUNTIME_LATENCY;
+  rt->latency = rt->dt == DT_BF16 && family == ARLO_RUNTIME_SPLITK;
   rt->fused = family == ARLO_RUNTIME_FUSED;
+  // LATENCY family = the LayerNorm fold (ARLO_LN_FOLD=1 applies it to the THROUGHPUT family too, A/B)
+  rt->ln_fold = rt->dt == DT_BF16 && (family == ARLO_RUNTIME_LATENCY || getenv("ARLO_LN_FOLD") != nullptr) &&
+                !rt->latency && !rt->fused && c.hidden % 32 == 0;
   auto fail = [&](int code) { destroy_runtime(rt); return code; };
   cudaError_t e = cudaStreamCreateWithFlags(&rt->own_stream, cudaStreamNonBlocking);
   if (e != cudaSuccess) return fail(cuda_fail(e, "cudaStreamCreate"));
@@ -536,6 +704,9 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   const size_t off_O = off; off = al(off + es * Mmax * H);
   const size_t off_Y = off; off = al(off + es * Mmax * H);
   const size_t off_F = off; off = al(off + es * Mmax * F);
+  const size_t st_bytes = rt->ln_fold ? 4 * Mmax * (H / 32) * 2 : 0;
+  const size_t off_S1 = off; off = al(off + st_bytes);
+  const size_t off_S2 = off; off = al(off + st_bytes);
   e = cudaMalloc(&rt->arena, off);
   if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "arena of %zu bytes: %s", off, cudaGetErrorString(e)));
   e = cudaMemset(rt->arena, 0, off);
@@ -548,6 +719,12 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   rt->pooled = (float*)(a + off_pooled);
   rt->gbar = (unsigned*)(a + off_gbar);
   rt->X = a + off_X; rt->QKV = a + off_QKV; rt->O = a + off_O; rt->Y = a + off_Y; rt->F = a + off_F;
+  if (rt->ln_fold) {
+    rt->S1 = (float*)(a + off_S1);
+    rt->S2 = (float*)(a + off_S2);
+    const int rc = ensure_fold(rt->w, rt->own_stream);
+    if (rc) return fail(rc);
+  }
   rt->h_stage_bytes = off_ids + 4 * Mmax + 4 * (size_t)max_batch * c.num_labels + 64;
   e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
   if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "pinned staging: %s", cudaGetErrorString(e)));
@@ -722,6 +899,23 @@ extern "C" int arlo_op_gemm(int32_t dtype, int32_t M, int32_t N, int32_t K, cons
   } else {
     ARLO_CUDA(launch_gemm_simt(DT_FP32, M, N, K, A, W, bias, residual, out, epi, s), "simt gemm");
   }
+  return ARLO_OK;
+}
+
+extern "C" int arlo_op_gemm_fold(int32_t M, int32_t N, int32_t K, const void* A, const void* W, const float* v0,
+                                 const float* v1, const float* v2, const float* st_in, int32_t st_in_stride,
+                                 float* st_out, int32_t st_ld, float eps, const void* residual, void* out,
+                                 int32_t epi, int32_t force_bn, void* stream) {
+  clear_error();
+  if (M < 1 || N % 64 || K % 64 || N < 64 || K < 64 || !A || !W || !v0 || !out ||
+      (epi != EPI_LNFOLD && epi != EPI_LNFOLD_GELU && epi != EPI_RESID_LN) || (epi == EPI_RESID_LN && !residual) ||
+      (epi != EPI_RESID_LN && (!v1 || !st_in)) || st_in_stride < 1 || ((st_in || st_out) && st_ld < M))
+    return set_error(ARLO_EINVAL, "arlo_op_gemm_fold: bad arguments");
+  TcGemmPlan p;
+  if (!tc_plan_gemm(&p, M, N, K, A, W, v0, residual, out, epi, force_bn) || p.splitk)
+    return set_error(ARLO_EINVAL, "arlo_op_gemm_fold: plan failed (tile %d)", force_bn);
+  p.fold = FoldArgs{v1, v2, st_in, st_in_stride, st_out, eps, st_ld};
+  ARLO_CUDA(tc_launch_gemm(p, (cudaStream_t)stream), "LayerNorm-fold gemm");
   return ARLO_OK;
 }
 

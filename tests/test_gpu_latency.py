@@ -1,6 +1,6 @@
-"""The latency (batch-1) runtime family: split-K weight-streaming GEMMs (needs a B200).
+"""The split-K runtime family: split-K weight-streaming GEMMs for batch 1 (needs a B200).
 
-PAPER.md:L282 §5 runs every runtime at batch 1.  The latency family serves that setting
+PAPER.md:L282 §5 runs every runtime at batch 1.  The split-K family serves that setting
 with the split-K kernel (csrc/gemm_splitk.cu); these tests pin it to the oracle per op and
 end to end, and check its contract: the split factor depends on the weight shape only, so
 a request's logits are bitwise equal on every latency runtime L >= its length, and every
@@ -76,8 +76,8 @@ def test_splitk_tile_widths_and_M_bitwise(arlo_lib, epi):
 
 
 def _latency_runtime(arlo_lib, W, L):
-    rt = arlo_lib.Runtime(W, L, 1, arlo_lib.RUNTIME_LATENCY)
-    assert rt.family == arlo_lib.RUNTIME_LATENCY
+    rt = arlo_lib.Runtime(W, L, 1, arlo_lib.RUNTIME_SPLITK)
+    assert rt.family == arlo_lib.RUNTIME_SPLITK
     assert all(c > arlo_lib.SPLITK_CODE for c in rt.gemm_tiles(1))
     return rt
 

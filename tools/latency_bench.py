@@ -3,8 +3,8 @@
     python tools/latency_bench.py [bert-base|bert-large] [families,...] > gpurun_out/latency.json
 
 Per runtime L: median of 50 graph replays (CUDA events per replay) of a b = 1 forward in
-the latency family (split-K weight streaming), the throughput family (bucket 1 of a
-max_batch = 32 runtime) and, at L <= 128, the fused family (one persistent kernel).  Per GEMM shape at M = 64: the split-K kernel vs the skinny /
+the latency family (LayerNorm fold), the throughput family (bucket 1 of a max_batch = 32
+runtime), the split-K family and, at L <= 128, the fused family (one persistent kernel).  Per GEMM shape at M = 64: the split-K kernel vs the skinny /
 tile kernel the chooser picks, as weight-streaming bandwidth (weight bytes / time) with
 the weights cold (L2 flushed before each launch) and the activations warm.
 """
@@ -71,7 +71,8 @@ def main():
     out = {"config": name, "forward_ms": {}, "gemm_M64": {}}
     for L in ((64, 128, 256, 512) if name == "bert-base" else (128, 256, 512)):
         row = {}
-        fams = [("latency", 1, arlo.RUNTIME_LATENCY), ("throughput", 32, arlo.RUNTIME_THROUGHPUT)]
+        fams = [("latency", 1, arlo.RUNTIME_LATENCY), ("throughput", 32, arlo.RUNTIME_THROUGHPUT),
+                ("splitk", 1, arlo.RUNTIME_SPLITK)]
         if L <= 128:
             fams.append(("fused", 1, arlo.RUNTIME_FUSED))
         if len(sys.argv) > 2:
