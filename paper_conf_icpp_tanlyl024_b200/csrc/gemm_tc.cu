@@ -285,7 +285,9 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   const bool stamp = threadIdx.x == 0 && g_trace != nullptr && sc < 64;  // (sc: chunks stored so far)
   const bool first_tile = sc == 0;
   if (stamp && first_tile) trace_clk(32);
-  uint32_t r[2][CW];
+  // the fold epilogues load one TMEM chunk at a time (their extra operands otherwise spill)
+  constexpr int NB = EPI >= EPI_LNFOLD ? 1 : 2;
+  uint32_t r[NB][CW];
   uint4 rv[2][RV];
   const bool rsm = rbuf != nullptr;  // residual tile in shared memory (TMA-prefetched), output in place
   constexpr int NV = nvec_of(EPI);
@@ -300,7 +302,15 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   for (int k = 0; k < NCMAX; ++k) {
     if (k >= nc) break;
     const int c = cg + k * kEpiGroups;  // chunk index within the tile
-    const int cur = k & 1, nxt = cur ^ 1;
+    const int cur = NB == 2 ? (k & 1) : 0, nxt = NB == 2 ? (cur ^ 1) : 0;
+    if (NB == 1 && k > 0) {
+      ptx::tmem_ld_32x32b_x32(t_row + c * CW, r[0]);
+      if (is_resid(EPI) && row_ok && !rbuf) {
+#pragma unroll
+        for (int j = 0; j < RV; ++j) rv[0][j] = ld_dep_v4(res4 + c * RV + j);
+      }
+      ptx::tmem_wait_ld();
+    }
     if (stamp && first_tile && k < 6) trace_clk(34 + 5 * k);
     // this chunk's 32 rows x 32 columns in the residual buffer (64-byte rows, 64B swizzle)
     uint8_t* rchunk = rsm ? rbuf + c * (BM * CW * 2) + q * (32 * CW * 2) : nullptr;
@@ -309,7 +319,7 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       for (int j = 0; j < RV; ++j)
         rv[cur][j] = *reinterpret_cast<const uint4*>(rchunk + lane * (CW * 2) + ((j ^ ((lane >> 1) & 3)) * 16));
     }
-    if (k + 1 < nc) {
+    if (NB == 2 && k + 1 < nc) {
       ptx::tmem_ld_32x32b_x32(t_row + (c + kEpiGroups) * CW, r[nxt]);
       if (is_resid(EPI) && row_ok && !rsm) {
 #pragma unroll

@@ -1,6 +1,7 @@
 """Per-CTA pipeline timeline of one tcgen05 GEMM launch (globaltimer stamps).
 
-    python tools/gemm_trace.py M N K [BN] [EPI]      BN < 0 = CTA-pair kernel; EPI 0 bias, 1 GELU, 2 residual
+    python tools/gemm_trace.py M N K [BN] [EPI]      BN < 0 = CTA-pair kernel; EPI 0 bias, 1 GELU, 2 residual,
+                                                     3 / 4 / 5 LayerNorm fold (arlo_op_gemm_fold)
 Slots per CTA: 0 start (after setup), 1 end; per tile i: 2+6i producer starts tile,
 3+6i MMA got accumulator, 4+6i first stage landed, 5+6i last MMA issued,
 6+6i epilogue got tile, 7+6i epilogue done (warp 0).
@@ -21,13 +22,26 @@ dev = torch.device("cuda")
 A = torch.randn(M, K, device=dev).to(torch.bfloat16)
 W = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
 b = torch.zeros(N, device=dev)
-R = torch.randn(M, N, device=dev).to(torch.bfloat16) if epi == 2 else None
+R = torch.randn(M, N, device=dev).to(torch.bfloat16) if epi in (2, 5) else None
 out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
+v1, v2 = torch.rand(N, device=dev) + 0.5, torch.rand(N, device=dev)
+st_in = torch.rand((N if epi == 5 else K) // 32, M, 2, device=dev) + 1
+st_out = torch.zeros(N // 32, M, 2, device=dev)
+
+
+def launch():
+    if epi >= 3:  # LayerNorm-fold epilogues (arlo_op_gemm_fold)
+        arlo.op_gemm_fold(A, W, b, out, epi, v1=v1, v2=v2 if epi == 5 else None, st_in=st_in,
+                          st_out=st_out if epi == 5 else None, residual=R, force_bn=bn)
+    else:
+        arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R, force_bn=bn)
+
+
 for _ in range(3):
-    arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R, force_bn=bn)
+    launch()
 buf = torch.zeros(148 * 64, dtype=torch.int64, device=dev)
 arlo.check(arlo.lib.arlo_debug_gemm_trace(buf.data_ptr()))
-arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R, force_bn=bn)
+launch()
 torch.cuda.synchronize()
 arlo.check(arlo.lib.arlo_debug_gemm_trace(None))
 t = buf.cpu().numpy().reshape(148, 64).astype(np.float64)
