@@ -519,12 +519,17 @@ def bert_large_per_L(arlo, torch, dev, stream, device_index, flush, reps=20):
 def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
     """Roofline of the dominant kernel.  The four GEMMs of the L=128, b=32 runtime (the bucket
     that serves the most requests, 43 %; M = 4096) are timed in the tile configuration its
-    CUDA graph actually replays (rt.gemm_tiles(32), chosen by timing at runtime creation),
-    each launch bracketed by CUDA events on the launching stream, `reps` launches averaged.
-    Before each launch (outside the events) L2 is flushed and the activations are rewritten,
-    as in the forward: A (and the residual) were just produced by the previous kernel and sit
-    in L2, the layer's weights come from HBM.  The dominant kernel is the GEMM with the
-    largest time; achieved = 2MNK / its mean launch time."""
+    CUDA graph actually replays (rt.gemm_tiles(32), chosen by timing at runtime creation).
+    Each GEMM is timed the way the forward runs it, inside a CUDA graph, after its inputs were
+    written: graph G1 = `reps` x [L2 flush, A (and residual) rewritten, GEMM], graph G0 = the
+    same without the GEMM, both replayed on the launching stream between CUDA events; the
+    launch time is (t(G1) - t(G0)) / reps.  A is L2-resident (just written, as the previous
+    kernel leaves it), the layer's weights come from HBM, and the GEMM's prologue is not
+    overlapped with its predecessor (no PDL edge from a copy), so this is conservative against
+    the forward.  `single_launch_us` is the same launch timed alone with events on the stream
+    outside a graph: it adds ~8 us of launch overhead that the kernel's own globaltimer span
+    does not show (tools/roofline_ctx.py, profiles/r02_roofline_ctx.txt).  The dominant kernel
+    is the GEMM with the largest time; achieved = 2MNK / its launch time."""
     H, F = 768, 3072
     M = 128 * 32
     codes = rt128.gemm_tiles(32)
@@ -541,23 +546,33 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
         res = torch.randn(m, n, device=dev, generator=g).to(torch.bfloat16) if epi == arlo.EPI_BIAS_RESIDUAL else None
         out = torch.empty(m, n, device=dev, dtype=torch.bfloat16)
         A0, R0 = A.clone(), (res.clone() if res is not None else None)
-        for _ in range(3):
+
+        def gemm():
             arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
-        ev = []
-        for _ in range(reps):
+
+        def prep():
             flush.zero_()
             A.copy_(A0)  # the predecessor's output: L2-resident, the weights are not
             if res is not None:
                 res.copy_(R0)
+
+        for _ in range(3):
+            gemm()
+        ev = []
+        for _ in range(reps):
+            prep()
             a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             a.record(stream)
-            arlo.op_gemm(arlo.BF16, A, Wt, bias, out, epi=epi, residual=res, force_bn=code, stream=stream)
+            gemm()
             e.record(stream)
             ev.append((a, e))
         torch.cuda.synchronize()
-        t_us = 1e3 * float(np.mean([a.elapsed_time(e) for a, e in ev]))
+        t_single = 1e3 * float(np.mean([a.elapsed_time(e) for a, e in ev]))
+        g1 = graph_us(torch, stream, lambda: (prep(), gemm()), reps)
+        g0 = graph_us(torch, stream, prep, reps)
+        t_us = (g1 - g0) / reps
         fl = metrics.gemm_flops(m, n, k)
-        table[name] = {"M": m, "N": n, "K": k, "tile_code": code, "launch_us": t_us,
+        table[name] = {"M": m, "N": n, "K": k, "tile_code": code, "launch_us": t_us, "single_launch_us": t_single,
                        "tflops": fl / (t_us / 1e6) / 1e12, "frac": fl / (t_us / 1e6) / 1e12 / peak}
     dom = max(table, key=lambda k: table[k]["launch_us"])
     d = table[dom]
@@ -574,9 +589,33 @@ def roofline_dominant(arlo, torch, dev, stream, rt128, flush, reps=30):
     roof = {"kernel": f"{kname} ({dom}, M={d['M']} N={d['N']} K={d['K']}, L=128 b=32 graph tile)", "bound": "tensor",
             "achieved": round(d["tflops"], 1), "peak": peak, "unit": "TFLOP/s", "frac": round(d["frac"], 4),
             "traffic": traffic, "peak_source": src + " bf16_tflops (burst)", "launch_us": round(d["launch_us"], 2),
-            "algorithmic_flops_per_launch": metrics.gemm_flops(d["M"], d["N"], d["K"]),
-            "l2": "flushed before each launch, then A / residual rewritten (L2-resident as in the forward), W cold"}
+            "single_launch_us": round(d["single_launch_us"], 2), "algorithmic_flops_per_launch": metrics.gemm_flops(d["M"], d["N"], d["K"]),
+            "l2": "flushed before each launch, then A / residual rewritten (L2-resident as in the forward), W cold",
+            "timing": "in a CUDA graph: (graph[flush, rewrite, GEMM] - graph[flush, rewrite]) / reps, CUDA events"}
     return roof, table
+
+
+def graph_us(torch, stream, body, n):
+    """Device time (us) of one replay of a CUDA graph of n x body(), median of 5, CUDA events on `stream`."""
+    with torch.cuda.stream(stream):
+        for _ in range(2):
+            body()
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=stream):
+            for _ in range(n):
+                body()
+        g.replay()
+        ts = []
+        for _ in range(5):
+            a, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record(stream)
+            g.replay()
+            e.record(stream)
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(e) * 1e3)
+    del g
+    return float(np.median(ts))
 
 
 def per_L_table(runtimes, torch, dev, stream, cfg, restricted=False, b_list=None):
