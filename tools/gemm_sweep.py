@@ -57,7 +57,7 @@ def time_op(fn, reps=20):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--epi", type=int, default=0)
+    ap.add_argument("--epi", type=int, default=0, help="-1: each shape's own BERT epilogue (N = 4K GELU, N <= K residual, else bias)")
     ap.add_argument("--set", default="base")
     ap.add_argument("--no-cublas", action="store_true")
     ap.add_argument("forces", nargs="*", type=int)
@@ -65,19 +65,20 @@ def main():
     forces = a.forces or [0, 256, 192, 128, -256, -192, -128]
     dev = torch.device("cuda")
     for (M, N, K) in SETS[a.set]:
+        epi = a.epi if a.epi >= 0 else (1 if N == 4 * K else 2 if N <= K else 0)
         A = torch.randn(M, K, device=dev).to(torch.bfloat16)
         W = (0.02 * torch.randn(N, K, device=dev)).to(torch.bfloat16)
         b = torch.zeros(N, device=dev)
-        R = torch.randn(M, N, device=dev).to(torch.bfloat16) if a.epi == 2 else None
+        R = torch.randn(M, N, device=dev).to(torch.bfloat16) if epi == 2 else None
         out = torch.empty(M, N, device=dev, dtype=torch.bfloat16)
-        line = f"{M:6d} {N:5d} {K:5d} choice={arlo.gemm_tile_choice(M, N, K):5d}:"
+        line = f"{M:6d} {N:5d} {K:5d} epi={epi} choice={arlo.gemm_tile_choice(M, N, K):5d}:"
         fl = 2.0 * M * N * K
         for f in forces:
             bn = f - 4000 if f > 4000 else f - 1000 if f > 1000 else abs(f or 64)
             if N % bn:
                 line += f"  {f:5d}=   n/a  "
                 continue
-            t = time_op(lambda st: arlo.op_gemm(arlo.BF16, A, W, b, out, epi=a.epi, residual=R, force_bn=f, stream=st))
+            t = time_op(lambda st: arlo.op_gemm(arlo.BF16, A, W, b, out, epi=epi, residual=R, force_bn=f, stream=st))
             line += f"  {f:5d}={fl / t / 1e12:5.0f}TF/{t * 1e6:6.1f}us"
         if not a.no_cublas:
             t = time_op(lambda st: torch.matmul(A, W.t()))

@@ -27,5 +27,11 @@ full attn_l128 attn_tc python tools/profile_ops.py attn 32 128 12 128
 full attn_l512 attn_tc python tools/profile_ops.py attn 64 512 16 512
 full layernorm layernorm python tools/profile_ops.py ln 4096 768
 python tools/ncu_summary.py $out/*.ncu-rep > $out/ncu_summary.txt 2>&1
+# per-launch DRAM traffic of the four L=128 b=32 GEMMs, keyed as bench.py's roofline looks it up
+cp profiles/traffic.json $out/traffic.json 2>/dev/null
+python tools/ncu_summary.py --traffic $out/traffic.json qkv_L128_b32_tile$1_dram_bytes=$out/qkv_L128b32.ncu-rep \
+    out_proj_L128_b32_tile$2_dram_bytes=$out/out_L128b32.ncu-rep ffn1_L128_b32_tile$3_dram_bytes=$out/ffn1_L128b32.ncu-rep \
+    ffn2_L128_b32_tile$4_dram_bytes=$out/ffn2_L128b32.ncu-rep > $out/traffic.log 2>&1
+ncu -i $out/ffn1_L128b32.ncu-rep --page source --csv > $out/ffn1_source.csv 2>/dev/null
 # keep the pulled-back directory small (gpurun merges <= 64 MiB): the reports stay on the box
 mkdir -p /tmp/ncu_reps && mv $out/*.ncu-rep /tmp/ncu_reps/ 2>/dev/null
