@@ -113,18 +113,20 @@ __device__ __forceinline__ float gelu_erf_fast(float z) {
 #endif
 }
 
-// gelu_erf_fast on two values with the sm_100 paired fp32 instructions (FFMA2 / FMUL2):
-// the same A&S 7.1.26 evaluation, half the FMA-pipe issue slots.  Every GEMM
-// epilogue (single CTA, CTA pair, skinny) uses this one function, so a given
-// element is computed bitwise identically whatever tile produced it.  The
-// polynomial is negated (exact) so that the last step is one FFMA2:
-// GELU = max(z, 0) + (-0.5 |z| erfc(a)).
+// GELU (erf form, reading S2) on two values with the sm_100 paired fp32 instructions (FFMA2 /
+// FMUL2).  Every GEMM epilogue (single CTA, CTA pair, skinny, split-K, fused) uses this one
+// function, so a given element is computed bitwise identically whatever tile produced it.
+// Default: Abramowitz & Stegun 7.1.28, erfc(a) = (1 + c1 a + ... + c6 a^6)^-16, |erf error| <=
+// 3e-7 (pinned against scipy in tests/test_gelu_fast.py): ONE MUFU op (rcp) per element.  The
+// 7.1.26 form below (ARLO_GELU2_AS26) takes two (rcp, ex2); the GELU epilogue runs at the
+// 16/clk/SM MUFU rate (gemm_trace: ~2000 of a chunk's cycles are its math), so halving the MUFU
+// count shortens the exposed epilogue of the one- and two-round FFN1 GEMMs.
+// GELU = max(z, 0) + (-0.5 |z| erfc(|z| / sqrt 2)).
 __device__ __forceinline__ float2 f2(float v) { return make_float2(v, v); }
 __device__ __forceinline__ float2 gelu2_erf_fast(float2 z) {
   const float2 az = make_float2(fabsf(z.x), fabsf(z.y));
-#if defined(ARLO_GELU2_AS28)
-  // A&S 7.1.28: erfc(a) = (1 + c1 a + ... + c6 a^6)^-16, |erf error| <= 3e-7; a = |z|/sqrt 2 is
-  // folded into the coefficients (c_k 2^(-k/2)).  One MUFU (rcp) per element instead of two.
+#if !defined(ARLO_GELU2_AS26)
+  // A&S 7.1.28; a = |z| / sqrt 2 is folded into the coefficients (c_k 2^(-k/2))
   float2 p = __ffma2_rn(az, f2(0.0000430638f * 0.125f), f2(0.0002765672f * 0.17677669529663687f));
   p = __ffma2_rn(az, p, f2(0.0001520143f * 0.25f));
   p = __ffma2_rn(az, p, f2(0.0092705272f * 0.35355339059327379f));
@@ -137,7 +139,7 @@ __device__ __forceinline__ float2 gelu2_erf_fast(float2 z) {
   r = __fmul2_rn(r, r);
   r = __fmul2_rn(r, r);  // erfc(a)
   return __ffma2_rn(__fmul2_rn(az, f2(-0.5f)), r, make_float2(fmaxf(z.x, 0.0f), fmaxf(z.y, 0.0f)));
-#endif
+#else  // A&S 7.1.26 (two MUFU ops)
   const float2 d = __ffma2_rn(az, f2(0.3275911f * 0.70710678118654752f), f2(1.0f));
   const float2 t = make_float2(rcp_approx(d.x), rcp_approx(d.y));
   float2 q = __ffma2_rn(t, f2(-0.5f * 1.061405429f), f2(-0.5f * -1.453152027f));
@@ -148,6 +150,7 @@ __device__ __forceinline__ float2 gelu2_erf_fast(float2 z) {
   const float2 e = make_float2(ex2_approx(s.x), ex2_approx(s.y));  // exp(-z^2/2) = exp(-a^2)
   const float2 h = __fmul2_rn(__fmul2_rn(q, t), az);                // -0.5 |z| erfc(a) / exp(-a^2)
   return __ffma2_rn(h, e, make_float2(fmaxf(z.x, 0.0f), fmaxf(z.y, 0.0f)));
+#endif
 }
 
 // Pack two floats into a bf16x2 word (RNE), low half = a.

@@ -11,7 +11,7 @@
 // TensorRT engines for sm_86):
 //  * persistent CTAs (grid = min(tiles, #SMs)), static round-robin tile order
 //    (N fastest), single-CTA 128 x BN tiles or CTA-pair (cta_group::2) 256 x BN tiles;
-//  * warps 0..EW-1 = epilogue (EW = 8, or 12 for GELU at M <= 8192; Roles<EW>):
+//  * warps 0..EW-1 = epilogue (EW = 8; Roles<EW>):
 //    warp w reads TMEM lane quarter w % 4 and the 32-column chunks w/4, w/4 + EW/4, ...;
 //    tcgen05.ld, bias / GELU / residual on paired fp32 instructions, RNE to bf16,
 //    st.shared into a 64B-swizzled staging tile, TMA bulk tensor store.  Two TMEM
@@ -49,7 +49,10 @@ constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 stagi
 #ifndef ARLO_STG_BUFS
 #define ARLO_STG_BUFS 2
 #endif
-constexpr int kStgBufs = ARLO_STG_BUFS;         // staging tiles per epilogue warp (TMA stores in flight)
+constexpr int kStgBufs = ARLO_STG_BUFS;
+#ifndef ARLO_EPI_PAIRS
+#define ARLO_EPI_PAIRS 1  // A/B hook: 0 = one chunk per store step for the bias / GELU epilogues
+#endif         // staging tiles per epilogue warp (TMA stores in flight)
 // Per epilogue warp: kStgBufs output staging tiles, then the bias of the warp's chunks of the
 // current tile (32 fp32 per chunk, <= 4 chunks), staged before the accumulator wait so that the
 // epilogue math reads bias from shared memory, not from L2 (a cold __ldg per chunk cost ~400
@@ -67,11 +70,12 @@ constexpr int kWarpStg = kStgBufs * kStgBytes + kBiasWarpBytes;
 constexpr int kStagingBytes = kEpiWarps * kWarpStg;
 
 // Warp-role layout of the persistent kernels for EW epilogue warps (EW / 4 column groups per
-// TMEM lane quarter), then the TMA producer and the MMA warp.  EW = 8 by default; the
-// GELU epilogue (two MUFU ops per element) runs with EW = 12 where it, not the mainloop,
-// paces the kernel (M <= 8192: FFN1 at M = 4096 918 -> 985 TF, at M = 8192 1093 -> 1168 TF,
-// gpurun_out/ab18; at M = 16384 and K = 1024 the 12-warp variant lost); the
+// TMEM lane quarter), then the TMA producer and the MMA warp.  EW = 8.  Round 1 ran the GELU
+// epilogue (then two MUFU ops per element) with EW = 12 at M <= 8192; with the one-MUFU GELU
+// (A&S 7.1.28) and the two-chunk store step, 8 warps win at every M (FFN1 M = 2048 / 4096 / 8192:
+// 737 / 953 / 1132 vs 710 / 927 / 1100 TF; profiles/r02_epilogue_pairs_ab.txt).  The
 // bias / residual epilogues lose with 12 (fewer smem stages, more residual traffic in flight).
+// ARLO_GELU_EW12_MAX_M keeps the 12-warp instantiation reachable for A/B runs.
 template <int EW>
 struct Roles {
   static_assert(EW % 4 == 0, "epilogue warps cover the four TMEM lane quarters");
@@ -298,6 +302,73 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
   ptx::tmem_ld_32x32b_x32(t_row + cg * CW, r[0]);
   ptx::tmem_wait_ld();
   if (stamp && first_tile) trace_clk(33);
+  // Bias / GELU epilogues: two chunks per step.  Both chunks' math runs back to back (the second
+  // chunk's TMEM load overlaps the first's math), then one proxy fence, one warp sync and two TMA
+  // stores from the two staging tiles: half the fixed per-chunk store cost (fence + sync + issue +
+  // staging wait were ~500 of a ~1000-cycle chunk, tools/gemm_trace.py).  Same per-element
+  // arithmetic (epi_pack4): bitwise the one-chunk loop.  8 epilogue warps only: with 12 (GELU at
+  // M <= 8192, <= 144 registers per thread) the second live chunk spilled and the pair loop lost
+  // (FFN1 M = 4096 948 -> 928 TF; at M = 16384, 8 warps: 1097 -> 1197 TF, gpurun A/B).
+  if constexpr ((EPI == EPI_BIAS || EPI == EPI_BIAS_GELU) && ARLO_EPI_PAIRS && !ARLO_EPI_DIRECT &&
+                kEpiGroups < 3) {
+    static_assert(kStgBufs >= 2, "chunk-pair epilogue needs two staging tiles per warp");
+    auto chunk_math = [&](const uint32_t* rr, int kk, uint32_t* pk) {
+      const float4* bias4 = ARLO_BIAS_SMEM ? reinterpret_cast<const float4*>(sbias) + kk * (CW / 4)
+                                           : reinterpret_cast<const float4*>(bias + n0 + (cg + kk * kEpiGroups) * CW);
+#pragma unroll
+      for (int j = 0; j < CW / 4; ++j) {
+        const float4 b4 = ARLO_BIAS_SMEM ? bias4[j] : __ldg(bias4 + j);
+        epi_pack4<EPI>(&rr[4 * j], b4, 0u, 0u, pk[2 * j], pk[2 * j + 1]);
+      }
+    };
+    auto stage = [&](const uint32_t* pk, uint8_t* buf) {
+#pragma unroll
+      for (int j = 0; j < CW / 8; ++j) {
+        const int sw = j ^ ((lane >> 1) & 3);  // TMA 64B swizzle of a 64-byte row
+        *reinterpret_cast<uint4*>(buf + lane * (CW * 2) + sw * 16) =
+            make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+      }
+    };
+#pragma unroll 1
+    for (int k = 0; k < nc; k += 2) {
+      const bool two = k + 1 < nc, more = k + 2 < nc;
+      const int c0 = cg + k * kEpiGroups, c1 = c0 + kEpiGroups;
+      if (stamp && first_tile && k < 12) trace_clk(34 + 5 * (k / 2));
+      if (two) ptx::tmem_ld_32x32b_x32(t_row + c1 * CW, r[1]);  // overlaps chunk k's math
+      uint32_t pk[CW / 2];
+      chunk_math(r[0], k, pk);
+      if (stamp && first_tile && k < 12) trace_clk(35 + 5 * (k / 2));
+      if (sc > 0) {  // the previous step's TMA stores have finished reading both staging tiles
+        if (lane == 0) ptx::bulk_wait_read<0>();
+        __syncwarp();
+      }
+      if (stamp && first_tile && k < 12) trace_clk(36 + 5 * (k / 2));
+      stage(pk, stg);
+      if (two) ptx::tmem_wait_ld();
+      if (!more) {  // every TMEM load of this warp has completed: hand the accumulator back
+        ptx::tc_fence_before();
+        __syncwarp();
+        if (lane == 0) release();
+      }
+      if (two) {
+        chunk_math(r[1], k + 1, pk);
+        stage(pk, stg + kStgBytes);
+      }
+      if (more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
+      ptx::fence_proxy_async_smem();
+      __syncwarp();
+      if (lane == 0) {
+        ptx::tma_store_2d(tmC, stg, n0 + c0 * CW, row0);
+        if (two) ptx::tma_store_2d(tmC, stg + kStgBytes, n0 + c1 * CW, row0);
+        ptx::bulk_commit();
+      }
+      sc += two ? 2 : 1;
+      if (stamp && first_tile && k < 12) trace_clk(37 + 5 * (k / 2));
+      if (more) ptx::tmem_wait_ld();
+      if (stamp && first_tile && k < 12) trace_clk(38 + 5 * (k / 2));
+    }
+    return;
+  }
 #pragma unroll
   for (int k = 0; k < NCMAX; ++k) {
     if (k >= nc) break;
@@ -1515,7 +1586,7 @@ bool tc_plan_gemm_strided(TcGemmPlan* p, int M, int N, int K, const void* A, int
   const int slots = pair ? num_sms() / 2 : num_sms();
   p->grid = (tiles < slots ? tiles : slots) * (pair ? 2 : 1);
 #ifndef ARLO_GELU_EW12_MAX_M
-#define ARLO_GELU_EW12_MAX_M 8192  // A/B hook: 0 keeps 8 epilogue warps everywhere
+#define ARLO_GELU_EW12_MAX_M 0  // A/B hook: 8192 = 12 epilogue warps for GELU at M <= 8192 (round 1)
 #endif
   p->ew = ((epi == EPI_BIAS_GELU || epi == EPI_LNFOLD_GELU) && M <= ARLO_GELU_EW12_MAX_M) ? 12 : kEpiWarps;
   p->fold = FoldArgs{};
