@@ -52,6 +52,9 @@ constexpr int kStgBytes = 32 * 64;             // one 32-row x 32-col bf16 stagi
 constexpr int kStgBufs = ARLO_STG_BUFS;
 #ifndef ARLO_EPI_PAIRS
 #define ARLO_EPI_PAIRS 1  // A/B hook: 0 = one chunk per store step for the bias / GELU epilogues
+#endif
+#ifndef ARLO_EPI_PAIRS_RESID
+#define ARLO_EPI_PAIRS_RESID 0  // A/B hook: 1 = two-chunk store step for the residual epilogue too
 #endif         // staging tiles per epilogue warp (TMA stores in flight)
 // Per epilogue warp: kStgBufs output staging tiles, then the bias of the warp's chunks of the
 // current tile (32 fp32 per chunk, <= 4 chunks), staged before the accumulator wait so that the
@@ -368,6 +371,64 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
       if (stamp && first_tile && k < 12) trace_clk(38 + 5 * (k / 2));
     }
     return;
+  }
+  // Residual epilogue, residual tile TMA-prefetched into shared memory (the default): the same
+  // two-chunk step, each chunk written in place over its residual and TMA-stored from there.
+  if constexpr (EPI == EPI_BIAS_RESID && ARLO_EPI_PAIRS_RESID && !ARLO_EPI_DIRECT && kEpiGroups < 3) {
+    if (rsm) {
+      auto chunk = [&](const uint32_t* rr, int kk, uint8_t* rch) {
+        const float4* bias4 = ARLO_BIAS_SMEM ? reinterpret_cast<const float4*>(sbias) + kk * (CW / 4)
+                                             : reinterpret_cast<const float4*>(bias + n0 + (cg + kk * kEpiGroups) * CW);
+        uint32_t pk[CW / 2];
+#pragma unroll
+        for (int j = 0; j < CW / 8; ++j) {  // 8 columns: one 16-byte residual vector
+          const int sw = j ^ ((lane >> 1) & 3);
+          const uint4 u = *reinterpret_cast<const uint4*>(rch + lane * (CW * 2) + sw * 16);
+          const float4 b0 = ARLO_BIAS_SMEM ? bias4[2 * j] : __ldg(bias4 + 2 * j);
+          const float4 b1 = ARLO_BIAS_SMEM ? bias4[2 * j + 1] : __ldg(bias4 + 2 * j + 1);
+          epi_pack4<EPI>(&rr[8 * j], b0, u.x, u.y, pk[4 * j], pk[4 * j + 1]);
+          epi_pack4<EPI>(&rr[8 * j + 4], b1, u.z, u.w, pk[4 * j + 2], pk[4 * j + 3]);
+        }
+#pragma unroll
+        for (int j = 0; j < CW / 8; ++j) {
+          const int sw = j ^ ((lane >> 1) & 3);
+          *reinterpret_cast<uint4*>(rch + lane * (CW * 2) + sw * 16) =
+              make_uint4(pk[4 * j], pk[4 * j + 1], pk[4 * j + 2], pk[4 * j + 3]);
+        }
+      };
+#pragma unroll 1
+      for (int k = 0; k < nc; k += 2) {
+        const bool two = k + 1 < nc, more = k + 2 < nc;
+        const int c0 = cg + k * kEpiGroups, c1 = c0 + kEpiGroups;
+        uint8_t* rch0 = rbuf + c0 * (BM * CW * 2) + q * (32 * CW * 2);
+        uint8_t* rch1 = rbuf + c1 * (BM * CW * 2) + q * (32 * CW * 2);
+        if (stamp && first_tile && k < 12) trace_clk(34 + 5 * (k / 2));
+        if (two) ptx::tmem_ld_32x32b_x32(t_row + c1 * CW, r[1]);  // overlaps chunk k's math
+        chunk(r[0], k, rch0);
+        if (stamp && first_tile && k < 12) trace_clk(35 + 5 * (k / 2));
+        if (two) ptx::tmem_wait_ld();
+        if (!more) {  // every TMEM load of this warp has completed: hand the accumulator back
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) release();
+        }
+        if (stamp && first_tile && k < 12) trace_clk(36 + 5 * (k / 2));
+        if (two) chunk(r[1], k + 1, rch1);
+        if (more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
+        ptx::fence_proxy_async_smem();
+        __syncwarp();
+        if (lane == 0) {
+          ptx::tma_store_2d(tmC, rch0, n0 + c0 * CW, row0);
+          if (two) ptx::tma_store_2d(tmC, rch1, n0 + c1 * CW, row0);
+          ptx::bulk_commit();
+        }
+        sc += two ? 2 : 1;
+        if (stamp && first_tile && k < 12) trace_clk(37 + 5 * (k / 2));
+        if (more) ptx::tmem_wait_ld();
+        if (stamp && first_tile && k < 12) trace_clk(38 + 5 * (k / 2));
+      }
+      return;
+    }
   }
 #pragma unroll
   for (int k = 0; k < NCMAX; ++k) {

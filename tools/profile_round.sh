@@ -33,5 +33,17 @@ python tools/ncu_summary.py --traffic $out/traffic.json qkv_L128_b32_tile$1_dram
     out_proj_L128_b32_tile$2_dram_bytes=$out/out_L128b32.ncu-rep ffn1_L128_b32_tile$3_dram_bytes=$out/ffn1_L128b32.ncu-rep \
     ffn2_L128_b32_tile$4_dram_bytes=$out/ffn2_L128b32.ncu-rep > $out/traffic.log 2>&1
 ncu -i $out/ffn1_L128b32.ncu-rep --page source --csv > $out/ffn1_source.csv 2>/dev/null
+# the build-time tile choice of a shape can differ between runs when two codes time within noise:
+# capture the traffic of every candidate tile of the four GEMMs (metrics only, one launch each)
+for g in "qkv 2304 768 0" "out_proj 768 768 2" "ffn1 3072 768 1" "ffn2 768 3072 2"; do
+  set -- $g
+  for code in -256 -192 -128 256 192 128 96; do
+    [ $(( $2 % (code < 0 ? -code : code) )) -eq 0 ] || continue
+    timeout 300 ncu --metrics dram__bytes_read.sum,dram__bytes_write.sum,gpu__time_duration.sum --clock-control none \
+        -k regex:gemm -s 2 -c 1 -o $out/t_$1_$code python tools/profile_ops.py gemm 4096 $2 $3 $4 $code > /dev/null 2>&1 &&
+      python tools/ncu_summary.py --traffic $out/traffic.json $1_L128_b32_tile${code}_dram_bytes=$out/t_$1_$code.ncu-rep \
+        >> $out/traffic.log 2>&1
+  done
+done
 # keep the pulled-back directory small (gpurun merges <= 64 MiB): the reports stay on the box
 mkdir -p /tmp/ncu_reps && mv $out/*.ncu-rep /tmp/ncu_reps/ 2>/dev/null
