@@ -54,7 +54,7 @@ constexpr int kStgBufs = ARLO_STG_BUFS;
 #define ARLO_EPI_PAIRS 1  // A/B hook: 0 = one chunk per store step for the bias / GELU epilogues
 #endif
 #ifndef ARLO_EPI_PAIRS_RESID
-#define ARLO_EPI_PAIRS_RESID 0  // A/B hook: 1 = two-chunk store step for the residual epilogue too
+#define ARLO_EPI_PAIRS_RESID 1  // A/B hook: 0 = one chunk per store step for the residual epilogue
 #endif         // staging tiles per epilogue warp (TMA stores in flight)
 // Per epilogue warp: kStgBufs output staging tiles, then the bias of the warp's chunks of the
 // current tile (32 fp32 per chunk, <= 4 chunks), staged before the accumulator wait so that the
