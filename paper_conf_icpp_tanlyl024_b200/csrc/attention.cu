@@ -668,7 +668,7 @@ cudaError_t attn_launch(const AttnPlan& p, const int32_t* lengths, void* o, cuda
     // A/B only: P aliased over S (128 TMEM columns), three CTAs per SM.  Correct (tests green)
     // but not faster: at b = 32, 12 heads the 384 CTAs run in one wave (span 8.5 vs 9.5 us in
     // isolation), yet each CTA serialises S(c+1) behind PV(c) and three CTAs share the MUFU /
-    // TMEM-read budget: 10.6 vs 10.1 us graph-replayed (gpurun_out/ab22)
+    // TMEM-read budget: 10.6 vs 10.1 us graph-replayed (round-1 A/B, raw log not kept)
     if (p.L <= 128) return attn_launch_cfg<1, 1, 1>(p, lengths, o, s);
 #else
 #if !defined(ARLO_ATTN_NO_PACK)

@@ -18,7 +18,7 @@ namespace arlo {
 namespace {
 
 #ifndef ARLO_LN_ROWS
-#define ARLO_LN_ROWS 16  // rows (warps) per CTA: 16 -> 4.08 us at M=4096 vs 4.40 (8), 4.10 (32); gpurun_out/ab23
+#define ARLO_LN_ROWS 16  // rows (warps) per CTA: 16 -> 4.08 us at M=4096 vs 4.40 (8), 4.10 (32) (round-1 A/B)
 #endif
 constexpr int kRowsPerBlock = ARLO_LN_ROWS;  // one warp per row
 #ifndef ARLO_LN_SMEM
