@@ -106,7 +106,10 @@ int arlo_op_ln_gemm(int32_t M, int32_t N, int32_t K, const void* y, const float*
  *   epi ARLO_EPI_RESID_LN (5): out = bf16((acc + v0_n) + LN(r)) with LN(r) = ((r - mean) * rstd) *
  *     v1_n + v2_n from the residual rows r and their statistics st_in (N / 32 granules; st_in = NULL:
  *     plain residual r); st_out (optional) receives the statistics of the bf16 output rows.
- * Device pointers; M >= 1, N and K multiples of 64; force_bn as for arlo_op_gemm (no split-K).
+ * Device pointers; M >= 1, N and K multiples of 64; force_bn as for arlo_op_gemm.  Split-K codes
+ * (2000 + BN, BN in {32, 64, 128}: splitk_factor(N, K) partial sums in a fixed order) are accepted
+ * for epi 5 only (the LATENCY runtimes' FFN2); there each granule's statistics are the column-order
+ * sums of its 8 four-column quads, added by an xor tree (the same at every M and tile width).
  * Errors: EINVAL, ECUDA.
  */
 enum { ARLO_EPI_LNFOLD = 3, ARLO_EPI_LNFOLD_GELU = 4, ARLO_EPI_RESID_LN = 5 };

@@ -56,8 +56,11 @@ template <int BN, int EPI>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                    bf16* __restrict__ out, int M, int N, int kc, int a_rows, int stages, int a_stage,
-                   const float* __restrict__ bias, const bf16* __restrict__ resid, int ldr) {
+                   const float* __restrict__ bias, const bf16* __restrict__ resid, int ldr, const FoldArgs fa) {
   using R = SkRed<BN>;
+  // EPI_RESID_LN: (mean, rstd) of the residual rows of this 128-row block, from their granule
+  // statistics (fa.st_in); rstd < 0 marks a plain residual (no statistics: layer 0's input)
+  __shared__ float2 rs[EPI == EPI_RESID_LN ? BM : 1];
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
@@ -133,6 +136,13 @@ gemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
     }
     ptx::mma_commit_w(tfull);
   } else {
+    if constexpr (EPI == EPI_RESID_LN) {  // the residual rows' statistics, overlapping the main loop
+      pdl_wait();
+      const int grow = m0 + warp * 32 + lane;
+      rs[warp * 32 + lane] = fa.st_in != nullptr && grow < M
+                                 ? fold_row_stats(fa.st_in, (size_t)grow * fa.st_in_stride, fa.st_ld, N / 32, N, fa.eps)
+                                 : make_float2(0.f, -1.f);
+    }
     // partial -> own shared memory: thread = row (TMEM lane), BN fp32 columns
     ptx::mbar_wait(tfull, 0);
     ptx::tc_fence_after();
@@ -172,15 +182,43 @@ gemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
     const int grow = m0 + row, col = n0 + q * 4;
     const float4 b4 = __ldg(reinterpret_cast<const float4*>(bias + col));
     uint32_t ua = 0, ub = 0;
-    if (EPI == EPI_BIAS_RESID) {
+    if (EPI == EPI_BIAS_RESID || EPI == EPI_RESID_LN) {
       const uint2 u = ld_dep_v2(resid + (size_t)grow * ldr + col);
       ua = u.x;
       ub = u.y;
     }
-    const uint32_t r4[4] = {__float_as_uint(acc.x), __float_as_uint(acc.y), __float_as_uint(acc.z),
-                            __float_as_uint(acc.w)};
     uint32_t p0, p1;
-    epi_pack4<EPI>(r4, b4, ua, ub, p0, p1);
+    if constexpr (EPI == EPI_RESID_LN) {
+      // y = (acc + b) + LN(r) (epilogue.cuh), then the (sum y, sum y^2) of the 32-column granule of
+      // the bf16 outputs: each quad's sums in column order, then an xor tree over the granule's 8
+      // quads, which are 8 consecutive lanes (Q and kThreads are multiples of 8, so a granule is
+      // either wholly inside this iteration or wholly outside it).  A function of N and K only, so
+      // every runtime of the family produces each statistic alike.
+      const float4 g4 = fa.v1 ? __ldg(reinterpret_cast<const float4*>(fa.v1 + col)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float4 e4 = fa.v2 ? __ldg(reinterpret_cast<const float4*>(fa.v2 + col)) : make_float4(0.f, 0.f, 0.f, 0.f);
+      const float2 rowst = rs[row];
+      p0 = epi_fold_pair<EPI>(make_float2(acc.x, acc.y), make_float2(b4.x, b4.y), make_float2(g4.x, g4.y),
+                              make_float2(e4.x, e4.y), ua, rowst);
+      p1 = epi_fold_pair<EPI>(make_float2(acc.z, acc.w), make_float2(b4.z, b4.w), make_float2(g4.z, g4.w),
+                              make_float2(e4.z, e4.w), ub, rowst);
+      const float2 y0 = unpack_bf16x2(p0), y1 = unpack_bf16x2(p1);
+      float s1 = y0.x, s2 = y0.x * y0.x;
+      s1 += y0.y; s2 = fmaf(y0.y, y0.y, s2);
+      s1 += y1.x; s2 = fmaf(y1.x, y1.x, s2);
+      s1 += y1.y; s2 = fmaf(y1.y, y1.y, s2);
+      const unsigned gmask = 0xffu << (lane & 24);
+#pragma unroll
+      for (int o = 1; o < 8; o <<= 1) {
+        s1 += __shfl_xor_sync(gmask, s1, o);
+        s2 += __shfl_xor_sync(gmask, s2, o);
+      }
+      if ((lane & 7) == 0 && fa.st_out != nullptr)
+        reinterpret_cast<float2*>(fa.st_out)[(size_t)(col / 32) * fa.st_ld + grow] = make_float2(s1, s2);
+    } else {
+      const uint32_t r4[4] = {__float_as_uint(acc.x), __float_as_uint(acc.y), __float_as_uint(acc.z),
+                              __float_as_uint(acc.w)};
+      epi_pack4<EPI>(r4, b4, ua, ub, p0, p1);
+    }
     *reinterpret_cast<uint2*>(out + (size_t)grow * N + col) = make_uint2(p0, p1);
   }
   ptx::cluster_sync();  // no CTA leaves (releasing its shared memory) while a peer still reads it
@@ -195,7 +233,7 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
   auto kern = gemm_splitk_kernel<BN, EPI>;
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [&] {
-    return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemOptIn); });
+    return cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemOptIn - 2048); });
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3(p.splits, p.N / BN, (p.M + BM - 1) / BM);
@@ -212,7 +250,7 @@ cudaError_t launch_cfg(const TcGemmPlan& p, cudaStream_t s) {
   cfg.attrs = attr;
   cfg.numAttrs = pdl_enabled() ? 2 : 1;
   return cudaLaunchKernelEx(&cfg, kern, p.tmA, p.tmB, (bf16*)p.out, p.M, p.N, p.kc, p.a_rows, p.stages, p.a_stage,
-                            p.bias, (const bf16*)p.resid, p.ldr);
+                            p.bias, (const bf16*)p.resid, p.ldr, p.fold);
 }
 
 template <int BN>
@@ -221,6 +259,7 @@ cudaError_t launch_bn(const TcGemmPlan& p, cudaStream_t s) {
     case EPI_BIAS: return launch_cfg<BN, EPI_BIAS>(p, s);
     case EPI_BIAS_GELU: return launch_cfg<BN, EPI_BIAS_GELU>(p, s);
     case EPI_BIAS_RESID: return launch_cfg<BN, EPI_BIAS_RESID>(p, s);
+    case EPI_RESID_LN: return launch_cfg<BN, EPI_RESID_LN>(p, s);
   }
   return cudaErrorInvalidValue;
 }
@@ -263,7 +302,8 @@ bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int 
   const int red = BM * (bn + 4) * 4;
   const long ctas = (long)S * (N / bn) * ((M + BM - 1) / BM);
   // two CTAs per SM when the grid exceeds one wave, else the whole opt-in budget
-  int budget = ctas > num_sms() ? kSmemOptIn / 2 - 1024 : kSmemOptIn;
+  // (less 2 KB for the kernel's static shared memory: the EPI_RESID_LN row statistics)
+  int budget = ctas > num_sms() ? kSmemOptIn / 2 - 2048 : kSmemOptIn - 2048;
   if (const char* e = getenv("ARLO_SPLITK_SMEM")) budget = atoi(e);  // A/B: per-CTA smem budget (bytes)
   const int fixed = 1024 + red + 8 * 64;
   int stages = (budget - fixed) / (a_stage + b_stage);

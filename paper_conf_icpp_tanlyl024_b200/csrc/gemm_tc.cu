@@ -213,25 +213,7 @@ __device__ __forceinline__ void stage_colv(float* sv, const float* __restrict__ 
 }
 
 
-// Epilogue arithmetic of one 32-column chunk of a row for the LayerNorm-fold modes (paired fp32):
-//  EPI_LNFOLD(_GELU): x = acc * rstd + (nrm * s + c), nrm = -rstd * mean (rowst = (nrm, rstd)); GELU;
-//  EPI_RESID_LN: x = (acc + b) + LN(r), LN(r) = ((r - mean) * rstd) * gamma + beta
-//    (rowst = (mean, rstd) of the residual row; mean 0 / rstd 1 / gamma 1 / beta 0 = plain residual
-//    is not used: a plain residual passes rowst.y < 0).
-template <int EPI>
-__device__ __forceinline__ uint32_t epi_fold_pair(float2 a, float2 v0, float2 v1, float2 v2, uint32_t ru, float2 rowst) {
-  float2 x;
-  if constexpr (EPI == EPI_LNFOLD || EPI == EPI_LNFOLD_GELU) {  // v0 = s, v1 = c
-    x = __ffma2_rn(a, f2(rowst.y), __ffma2_rn(f2(rowst.x), v0, v1));
-    if (EPI == EPI_LNFOLD_GELU) x = gelu2_erf_fast(x);
-  } else {  // v0 = bias, v1 = gamma, v2 = beta
-    float2 rr = unpack_bf16x2(ru);
-    if (rowst.y >= 0.f) rr = __ffma2_rn(__fmul2_rn(__fadd2_rn(rr, f2(-rowst.x)), f2(rowst.y)), v1, v2);
-    x = __fadd2_rn(__fadd2_rn(a, v0), rr);
-  }
-  return pack_bf16x2(x.x, x.y);
-}
-
+// epi_fold_pair (the per-pair arithmetic of the LayerNorm-fold modes) is in epilogue.cuh.
 template <int EPI>
 __device__ __forceinline__ void epi_fold_chunk(const uint32_t* acc, const float* sv, const uint32_t* ru, float2 rowst,
                                                uint32_t* pk) {

@@ -377,16 +377,22 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
 // the candidates and wins ties.  Every tile code computes each output element with the same K
 // chain, so the choice changes time only, never a bit of the result (tile-width bitwise tests).
 // ARLO_NO_AUTOTUNE=1 keeps the analytic chooser.
+// `only` (optional): time these codes instead, the first one the incumbent (the split-K tile widths
+// of the fold family's FFN2, which share one arithmetic whatever the width).
 template <typename PlanFn>
-static int pick_tile(int M, int N, int K, cudaStream_t s, PlanFn plan) {
-  const int base = tc_choose_bn(M, N, K);
+static int pick_tile(int M, int N, int K, cudaStream_t s, PlanFn plan, const std::vector<int>* only = nullptr) {
+  const int base = only ? (*only)[0] : tc_choose_bn(M, N, K);
   if (getenv("ARLO_NO_AUTOTUNE") != nullptr) return base;
   std::vector<int> cands = {base};
-  for (int code : {-256, -192, -128, 256, 192, 128, 96, 64})
-    if (code != base && N % (code < 0 ? -code : code) == 0) cands.push_back(code);
-  if (M <= 1024)
-    for (int bn : {16, 32, 64})
-      if (kSkinnyCode + bn != base && N % bn == 0) cands.push_back(kSkinnyCode + bn);
+  if (only) {
+    cands = *only;
+  } else {
+    for (int code : {-256, -192, -128, 256, 192, 128, 96, 64})
+      if (code != base && N % (code < 0 ? -code : code) == 0) cands.push_back(code);
+    if (M <= 1024)
+      for (int bn : {16, 32, 64})
+        if (kSkinnyCode + bn != base && N % bn == 0) cands.push_back(kSkinnyCode + bn);
+  }
   cudaEvent_t e0, e1;
   if (cudaEventCreate(&e0) != cudaSuccess) return base;
   if (cudaEventCreate(&e1) != cudaSuccess) { cudaEventDestroy(e0); return base; }
@@ -485,9 +491,18 @@ static int plan_bucket_fold(arlo_runtime* rt, Bucket& bk) {
   const int t_o = pick_tile(M, H, H, ts, [&](TcGemmPlan* p, int code) {
     return tc_plan_gemm(p, M, H, H, rt->O, w->lt(0, LW_O), (const float*)w->lt(0, LB_O), rt->X, rt->Y, EPI_RESID_LN,
                         code); });
+  // FFN2 (K = 4H: the longest K chain, 4H/16 MMAs per output tile) runs split-K: S = f(N, K)
+  // CTAs per column tile, partials reduced in a fixed order; its arithmetic is the same at every M,
+  // so it holds for every runtime and bucket of the family, the CLS rows included.
+  // ARLO_FOLD_FFN2_TILE=1 keeps the tile kernels (A/B).
+  std::vector<int> sk_codes;
+  if (getenv("ARLO_FOLD_FFN2_TILE") == nullptr)
+    for (int bn : {64, 32, 128})
+      if (H % bn == 0) sk_codes.push_back(kSplitKCode + bn);
+  const bool f2_splitk = !sk_codes.empty();
   const int t_f2 = pick_tile(M, H, F, ts, [&](TcGemmPlan* p, int code) {
     return tc_plan_gemm(p, M, H, F, rt->F, w->lt(0, LW_2), (const float*)w->lt(0, LB_2), rt->Y, rt->X, EPI_RESID_LN,
-                        code); });
+                        code); }, f2_splitk ? &sk_codes : nullptr);
   if (cudaStreamSynchronize(ts) != cudaSuccess) return set_error(ARLO_ECUDA, "tile selection failed");
   bk.tiles[0] = t_qkv; bk.tiles[1] = t_o; bk.tiles[2] = t_f1; bk.tiles[3] = t_f2;
   auto ln_g = [&](int l, int k) { return (const float*)w->lt(l, k); };
@@ -520,7 +535,7 @@ static int plan_bucket_fold(arlo_runtime* rt, Bucket& bk) {
                              L * H, rt->Y, EPI_RESID_LN, 0) &&
         tc_plan_gemm(&bk.cls.f1, b, F, H, rt->Y, f.w1, f.s1, nullptr, rt->F, EPI_LNFOLD_GELU, 0) &&
         tc_plan_gemm(&bk.cls.f2, b, H, F, rt->F, w->lt(l, LW_2), (const float*)w->lt(l, LB_2), rt->Y, rt->X,
-                     EPI_RESID_LN, 0);
+                     EPI_RESID_LN, f2_splitk ? kSplitKCode + (H % 64 == 0 ? 64 : 32) : 0);
     if (!ok) return set_error(ARLO_ECUDA, "CLS-row LayerNorm-fold plan: tensor-map encoding failed");
     bk.cls.o.fold = FoldArgs{l >= 1 ? ln_g(l - 1, LN2_G) : nullptr, l >= 1 ? ln_g(l - 1, LN2_B) : nullptr,
                              l >= 1 ? rt->S2 : nullptr, L, rt->S1, eps, rt->max_batch * rt->L};
@@ -912,7 +927,7 @@ extern "C" int arlo_op_gemm_fold(int32_t M, int32_t N, int32_t K, const void* A,
       (epi != EPI_RESID_LN && (!v1 || !st_in)) || st_in_stride < 1 || ((st_in || st_out) && st_ld < M))
     return set_error(ARLO_EINVAL, "arlo_op_gemm_fold: bad arguments");
   TcGemmPlan p;
-  if (!tc_plan_gemm(&p, M, N, K, A, W, v0, residual, out, epi, force_bn) || p.splitk)
+  if (!tc_plan_gemm(&p, M, N, K, A, W, v0, residual, out, epi, force_bn) || (p.splitk && epi != EPI_RESID_LN))
     return set_error(ARLO_EINVAL, "arlo_op_gemm_fold: plan failed (tile %d)", force_bn);
   p.fold = FoldArgs{v1, v2, st_in, st_in_stride, st_out, eps, st_ld};
   ARLO_CUDA(tc_launch_gemm(p, (cudaStream_t)stream), "LayerNorm-fold gemm");

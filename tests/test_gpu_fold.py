@@ -202,3 +202,40 @@ def test_runtime_fold_against_unfolded(arlo_lib):
             assert np.argmax(a[i]) == np.argmax(b[i])
     folded.close()
     plain.close()
+
+
+@pytest.mark.parametrize("M,N,K", [(64, 768, 3072), (300, 768, 3072), (1, 1024, 4096)])
+def test_splitk_resid_ln_epilogue(arlo_lib, M, N, K):
+    """Split-K EPI_RESID_LN (the LATENCY runtimes' FFN2): oracle parity of the rows and of the output
+    statistics (also with a plain residual), and every split-K tile width and M gives bitwise the same
+    rows and statistics (its arithmetic is a function of N and K only: the family's cross-L contract)."""
+    eps = 1e-12
+    A, W, b = rnd((M, K), 31, 1.1, 0.05), rnd((N, K), 32, 0.02), rnd((N,), 33, 0.02)
+    R = rnd((M, N), 34, 1.5, 0.3)
+    g, be = rnd((N,), 35, 0.1, 1.0), rnd((N,), 36, 0.1)
+    st_r = granule_stats(R).astype(np.float32)
+    ref = orc.linear(A, W, b) + ln_from_stats(R.astype(np.float64), st_r.astype(np.float64), g, be, eps)
+    runs = []  # (m, rows, statistics); the first is code 2064 at m = M
+    for code in (2064, 2032, 2128):
+        if N % (code - 2000):
+            continue
+        for m in sorted({M, min(M, 64), min(M, 7)}, reverse=True):
+            o = torch.empty((m, N), device="cuda", dtype=torch.bfloat16)
+            so = torch.full((N // 32, m, 2), float("nan"), device="cuda")
+            arlo_lib.op_gemm_fold(bf(A[:m]), bf(W), f32(b), o, arlo_lib.EPI_RESID_LN, v1=f32(g), v2=f32(be),
+                                  st_in=f32(gm(st_r[:m])), st_out=so, eps=eps, residual=bf(R[:m]), force_bn=code)
+            runs.append((m, o, so))
+    torch.cuda.synchronize()
+    _, ref_o, ref_s = runs[0]
+    y = ref_o.float().cpu().numpy()
+    np.testing.assert_allclose(y, ref, rtol=1e-2, atol=2e-2)
+    np.testing.assert_allclose(ref_s.cpu().numpy(), gm(granule_stats(y)), rtol=2e-6, atol=1e-4)
+    for m, o, so in runs[1:]:
+        assert torch.equal(o, ref_o[:m])
+        assert torch.equal(so, ref_s[:, :m])
+    # st_in = NULL: plain residual
+    o2 = torch.empty((M, N), device="cuda", dtype=torch.bfloat16)
+    arlo_lib.op_gemm_fold(bf(A), bf(W), f32(b), o2, arlo_lib.EPI_RESID_LN, v1=f32(g), v2=f32(be), residual=bf(R),
+                          force_bn=2064)
+    torch.cuda.synchronize()
+    np.testing.assert_allclose(o2.float().cpu().numpy(), orc.linear(A, W, b) + R, rtol=1e-2, atol=2e-2)

@@ -24,6 +24,7 @@ SETS = {
               (128, 2304, 768), (128, 768, 3072), (512, 2304, 768), (512, 768, 3072),
               (128, 3072, 1024), (128, 1024, 4096)],
 }
+SETS["ffn2_small"] = [(m, 768, 3072) for m in (64, 128, 256, 384, 512)] + [(m, 1024, 4096) for m in (128, 256, 512)]
 SETS["mid"] = [(m, n, k) for m in (1024, 2048, 8192) for (n, k) in ((2304, 768), (3072, 768), (768, 3072), (768, 768))]
 SETS["all"] = SETS["base"] + SETS["large"] + SETS["small"] + SETS["mid"]
 
@@ -74,7 +75,7 @@ def main():
         line = f"{M:6d} {N:5d} {K:5d} epi={epi} choice={arlo.gemm_tile_choice(M, N, K):5d}:"
         fl = 2.0 * M * N * K
         for f in forces:
-            bn = f - 4000 if f > 4000 else f - 1000 if f > 1000 else abs(f or 64)
+            bn = f - 4000 if f > 4000 else f - 2000 if f > 2000 else f - 1000 if f > 1000 else abs(f or 64)
             if N % bn:
                 line += f"  {f:5d}=   n/a  "
                 continue
