@@ -49,7 +49,7 @@ struct SkRed {
   static constexpr int LD = BN + 4;  // fp32 row stride of the partial (spreads rows over banks)
   static constexpr int BYTES = BM * LD * 4;
   static constexpr int B_BYTES = BN * BK * 2;
-  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN;
+  static constexpr int TMEM_COLS = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
 };
 
 template <int BN, int EPI>
@@ -65,8 +65,11 @@ gemm_splitk_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constan
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sA = smem;
   uint8_t* sB = sA + stages * a_stage;
-  float* red = reinterpret_cast<float*>(sB + stages * R::B_BYTES);  // [BM][LD] fp32 partial
-  uint64_t* full = reinterpret_cast<uint64_t*>(red + BM * R::LD);
+  // [BM][LD] fp32 partial, over the operand ring: it is written only after the last MMA has
+  // completed (tfull), when no stage is read or written any more
+  float* red = reinterpret_cast<float*>(smem);
+  const int ring = stages * (a_stage + R::B_BYTES);
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + (ring > R::BYTES ? ring : R::BYTES));
   uint64_t* empty = full + stages;
   uint64_t* tfull = empty + stages;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tfull + 1);
@@ -284,7 +287,7 @@ int splitk_factor(int N, int K) {
 int splitk_bn(int M, int N, int S) {
   const long mblocks = (M + BM - 1) / BM;
   const long cap = 2L * num_sms();
-  for (int bn : {32, 64, 128})
+  for (int bn : {32, 64, 128, 192})
     if (N % bn == 0 && (long)(N / bn) * S * mblocks <= cap) return bn;
   return N % 128 == 0 ? 128 : N % 64 == 0 ? 64 : 32;
 }
@@ -294,7 +297,7 @@ bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int 
   if (M <= 0 || N % 64 || K % 64 || K <= 0 || lda < K || lda % 8 || ldr < N || ldr % 8) return false;
   const int S = splitk_factor(N, K);
   if (bn == 0) bn = splitk_bn(M, N, S);
-  if ((bn != 32 && bn != 64 && bn != 128) || N % bn) return false;
+  if ((bn != 32 && bn != 64 && bn != 128 && bn != 192) || N % bn) return false;
   const int kc = K / S, kblocks = kc / BK;
   const int a_rows = M < BM ? ((M + 7) & ~7) : BM;
   const int a_stage = ((a_rows * BK * 2) + 1023) & ~1023;
@@ -305,7 +308,7 @@ bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int 
   // (less 2 KB for the kernel's static shared memory: the EPI_RESID_LN row statistics)
   int budget = ctas > num_sms() ? kSmemOptIn / 2 - 2048 : kSmemOptIn - 2048;
   if (const char* e = getenv("ARLO_SPLITK_SMEM")) budget = atoi(e);  // A/B: per-CTA smem budget (bytes)
-  const int fixed = 1024 + red + 8 * 64;
+  const int fixed = 1024 + 8 * 64;  // (the partial `red` lives over the operand ring)
   int stages = (budget - fixed) / (a_stage + b_stage);
   if (stages > kMaxStages) stages = kMaxStages;
   if (stages < 2) stages = 2;  // (a budget too small for two stages is exceeded)
@@ -313,7 +316,7 @@ bool tc_plan_gemm_splitk(TcGemmPlan* p, int M, int N, int K, const void* A, int 
   p->M = M; p->N = N; p->K = K; p->BN = bn; p->epi = epi; p->grid = (int)ctas; p->ew = 4;
   p->pair = false; p->skinny = false; p->ln = false; p->splitk = true; p->fold = FoldArgs{}; p->lnp = LnPrologue{};
   p->splits = S; p->kc = kc; p->stages = stages; p->a_stage = a_stage; p->a_rows = a_rows;
-  p->smem = fixed + stages * (a_stage + b_stage);
+  p->smem = fixed + (stages * (a_stage + b_stage) > red ? stages * (a_stage + b_stage) : red);
   p->bias = bias; p->resid = resid; p->ldr = ldr; p->out = out;
   if (!encode_tmap_bf16_2d(&p->tmA, A, (uint64_t)K, (uint64_t)M, BK, a_rows, 128, (uint64_t)lda)) return false;
   if (!encode_tmap_bf16_2d(&p->tmB, W, (uint64_t)K, (uint64_t)N, BK, bn, 128)) return false;
@@ -325,6 +328,7 @@ cudaError_t splitk_launch(const TcGemmPlan& p, cudaStream_t s) {
     case 32: return launch_bn<32>(p, s);
     case 64: return launch_bn<64>(p, s);
     case 128: return launch_bn<128>(p, s);
+    case 192: return launch_bn<192>(p, s);
   }
   return cudaErrorInvalidValue;
 }

@@ -497,7 +497,7 @@ static int plan_bucket_fold(arlo_runtime* rt, Bucket& bk) {
   // ARLO_FOLD_FFN2_TILE=1 keeps the tile kernels (A/B).
   std::vector<int> sk_codes;
   if (getenv("ARLO_FOLD_FFN2_TILE") == nullptr)
-    for (int bn : {64, 32, 128})
+    for (int bn : {64, 32, 128, 192})  // (BN = 192: M = 512 in 16 clusters, within one wave of 6-CTA clusters)
       if (H % bn == 0) sk_codes.push_back(kSplitKCode + bn);
   const bool f2_splitk = !sk_codes.empty();
   const int t_f2 = pick_tile(M, H, F, ts, [&](TcGemmPlan* p, int code) {

@@ -216,7 +216,7 @@ def test_splitk_resid_ln_epilogue(arlo_lib, M, N, K):
     st_r = granule_stats(R).astype(np.float32)
     ref = orc.linear(A, W, b) + ln_from_stats(R.astype(np.float64), st_r.astype(np.float64), g, be, eps)
     runs = []  # (m, rows, statistics); the first is code 2064 at m = M
-    for code in (2064, 2032, 2128):
+    for code in (2064, 2032, 2128, 2192):
         if N % (code - 2000):
             continue
         for m in sorted({M, min(M, 64), min(M, 7)}, reverse=True):
