@@ -15,7 +15,8 @@
 //    K range of A through a TMA ring (W requested before the PDL wait: weights never depend
 //    on the previous kernel), and accumulates its partial sum in TMEM (M=128 tcgen05.mma,
 //    K=16 steps);
-//  * each CTA copies its fp32 partial to its own shared memory; after a cluster barrier the
+//  * each CTA copies its fp32 partial to its own shared memory (over its operand ring, idle by
+//    then); after a cluster barrier the
 //    rows are reduced over distributed shared memory in the FIXED order
 //    ((p_0 + p_1) + p_2) + ... + p_{S-1}, each row quad by exactly one CTA, then the shared
 //    epilogue (bias, GELU or residual, RNE to bf16; epilogue.cuh) and a direct store.
@@ -283,7 +284,10 @@ int splitk_factor(int N, int K) {
   return best;
 }
 
-// Tile width: the narrowest of 32 / 64 / 128 that keeps the grid within two CTAs per SM.
+// Tile width: the narrowest of 32 / 64 / 128 / 192 that keeps the grid within two CTAs per SM.
+// (The LATENCY family times the widths instead: at most 22 six-CTA clusters are resident at once
+// on B200 (ncu launch__cluster_max_active), so the width that keeps a GEMM in one wave of clusters
+// can be wider than this rule's.)
 int splitk_bn(int M, int N, int S) {
   const long mblocks = (M + BM - 1) / BM;
   const long cap = 2L * num_sms();
