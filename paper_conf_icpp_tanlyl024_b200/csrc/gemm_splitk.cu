@@ -19,7 +19,8 @@
 //    then); after a cluster barrier the
 //    rows are reduced over distributed shared memory in the FIXED order
 //    ((p_0 + p_1) + p_2) + ... + p_{S-1}, each row quad by exactly one CTA, then the shared
-//    epilogue (bias, GELU or residual, RNE to bf16; epilogue.cuh) and a direct store.
+//    epilogue (bias, GELU, residual, or the LATENCY family's residual + on-the-fly LayerNorm
+//    with the output's granule statistics; RNE to bf16; epilogue.cuh) and a direct store.
 //
 // S = splitk_factor(N, K) depends on the weight shape only, never on M, so every runtime of
 // the latency family produces each output element with the same sequence of fp32 additions:
