@@ -53,6 +53,9 @@ constexpr int kStgBufs = ARLO_STG_BUFS;
 #ifndef ARLO_EPI_PAIRS
 #define ARLO_EPI_PAIRS 1  // A/B hook: 0 = one chunk per store step for the bias / GELU epilogues
 #endif
+#ifndef ARLO_EPI_EARLY_LD
+#define ARLO_EPI_EARLY_LD 0  // A/B hook: 1 = the next step's first TMEM load before the second chunk's math
+#endif
 #ifndef ARLO_EPI_PAIRS_RESID
 #define ARLO_EPI_PAIRS_RESID 1  // A/B hook: 0 = one chunk per store step for the residual epilogue
 #endif         // staging tiles per epilogue warp (TMA stores in flight)
@@ -335,11 +338,12 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
         __syncwarp();
         if (lane == 0) release();
       }
+      if (ARLO_EPI_EARLY_LD && more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
       if (two) {
         chunk_math(r[1], k + 1, pk);
         stage(pk, stg + kStgBytes);
       }
-      if (more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
+      if (!ARLO_EPI_EARLY_LD && more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
       ptx::fence_proxy_async_smem();
       __syncwarp();
       if (lane == 0) {
@@ -395,8 +399,9 @@ __device__ __forceinline__ void epilogue_tile(uint32_t t_acc, int q, int cg, int
           if (lane == 0) release();
         }
         if (stamp && first_tile && k < 12) trace_clk(36 + 5 * (k / 2));
+        if (ARLO_EPI_EARLY_LD && more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
         if (two) chunk(r[1], k + 1, rch1);
-        if (more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
+        if (!ARLO_EPI_EARLY_LD && more) ptx::tmem_ld_32x32b_x32(t_row + (c1 + kEpiGroups) * CW, r[0]);
         ptx::fence_proxy_async_smem();
         __syncwarp();
         if (lane == 0) {
