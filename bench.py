@@ -403,6 +403,7 @@ def main():
         extras["bert_large"] = bl
         result["bert_large_frac_of_burst"] = {f"L{L}_b{b}": rnd(bl["per_L"][str(L)][str(b)]["frac_of_peak"], 3)
                                               for L in (256, 512) for b in (32, 64)}
+        result["bert_large_b1_latency_family_ms"] = {L: rnd(v) for L, v in bl["latency_family_b1_ms"].items()}
         if args.full:
             extras["trace_replay"] = trace_replay(arlo, torch, runtimes, cfg, stream, result, pl)
             extras["cluster_replay"] = cluster_replay(arlo, torch, W, runtimes, cfg, stream)
@@ -510,8 +511,16 @@ def bert_large_per_L(arlo, torch, dev, stream, device_index, flush, reps=20):
                            "sm_mhz": clk.get("sm_mhz"), "clock_reasons": clk.get("reasons")}
         out[str(L)] = row
         rt.close()
+    # the paper's batch-1 runtimes for BERT-large too, LATENCY family
+    lat_rts = {}
+    for L in (128, 256, 512):
+        lat_rts[L] = arlo.Runtime(W, L, 1, arlo.RUNTIME_LATENCY)
+        lat_rts[L].set_stream(stream)
+    lat_b1 = per_L_table(lat_rts, torch, dev, stream, cfg, b_list=(1,))
+    for rt in lat_rts.values():
+        rt.close()
     W.close()
-    return {"per_L": out, "peak_tflops": peak, "peak_sustained_tflops": peak_sus, "peak_source": src, "reps": reps,
+    return {"per_L": out, "latency_family_b1_ms": {L: lat_b1[L]["1"]["median"] for L in lat_b1}, "peak_tflops": peak, "peak_sustained_tflops": peak_sus, "peak_source": src, "reps": reps,
             "note": "static FLOPs = layers*(24bLH^2+4bL^2H)+b(2H^2+2HC); median of per-forward CUDA-event times, "
                     "L2 flushed before each forward"}
 
