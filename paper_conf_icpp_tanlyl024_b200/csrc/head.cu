@@ -37,10 +37,59 @@ __device__ __forceinline__ void unpack16(const uint4& u, float* f) {
 // The warp's W_p row is loaded into registers BEFORE the PDL wait (weights never depend
 // on the previous kernel); the CLS rows are then staged with every 16-byte load of a thread
 // issued before any shared-memory store (one L2 round trip, not one per element).
+// Classifier logit (sequence row, label c) by one warp: lane-strided 16-byte loads of the W_c row
+// and of the pooled row, fixed fma order, then warp_sum.  Shared by the classifier kernel and the
+// pooler's last-CTA classifier, so both give a sequence's logits bitwise alike.
+template <typename T, int MAXV>
+__device__ __forceinline__ float classifier_dot(const uint4 (&wv)[MAXV], const float* p, int nvec, int lane) {
+  constexpr int VN = 16 / sizeof(T);
+  float s = 0.f;
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i) {
+    const int v = lane + 32 * i;
+    if (v < nvec) {
+      float w[VN];
+      unpack16<T>(wv[i], w);
+#pragma unroll
+      for (int e = 0; e < VN; e += 4) {
+        const uint4 qu = ld_dep_v4(p + v * VN + e);
+        const float4 q = make_float4(__uint_as_float(qu.x), __uint_as_float(qu.y), __uint_as_float(qu.z),
+                                     __uint_as_float(qu.w));
+        s = fmaf(w[e], q.x, s);
+        s = fmaf(w[e + 1], q.y, s);
+        s = fmaf(w[e + 2], q.z, s);
+        s = fmaf(w[e + 3], q.w, s);
+      }
+    }
+  }
+  return warp_sum(s);
+}
+
+template <typename T, int MAXV>
+__device__ __forceinline__ void load_wrow(uint4 (&wv)[MAXV], const T* __restrict__ w, int row, int H, int lane) {
+  constexpr int VN = 16 / sizeof(T);
+  const uint4* wr = reinterpret_cast<const uint4*>(w + (size_t)row * H);
+#pragma unroll
+  for (int i = 0; i < MAXV; ++i)
+    if (lane + 32 * i < H / VN) wv[i] = __ldg(wr + lane + 32 * i);
+}
+
+// HeadCls (runtimes): the classifier runs in the pooler's grid.  Every CTA of a sequence group
+// (blockIdx.y) counts itself in cnt[blockIdx.y] after its pooled features are written (release);
+// the last one (acquire) computes the group's logits with classifier_dot and resets the counter
+// for the next replay.  One dependent launch less per forward.
+struct HeadCls {
+  const void* w_c;
+  const float* b_c;
+  float* logits;
+  int C;
+  unsigned* cnt;  // [ceil(B / 8)] zero-initialised, or nullptr: separate classifier kernel
+};
+
 template <typename T, int MAXV>
 __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const T* __restrict__ x,
                                                      const T* __restrict__ w_p, const float* __restrict__ b_p,
-                                                     float* __restrict__ pooled, const HeadLn ln) {
+                                                     float* __restrict__ pooled, const HeadLn ln, const HeadCls hc) {
   // [kRows][nvec] raw 16-byte vectors of T: lane-consecutive vectors are bank-conflict free
   // (fp32 staging with 8 floats per lane put lanes 4 apart on the same banks: 8-way STS,
   // 2x LDS.128 wavefronts; the pooler was shared-memory bound at 22 us for b = 32)
@@ -100,7 +149,7 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
     }
   }
   __syncthreads();
-  if (j >= H) return;
+  if (j < H) {
   float acc[kRows];
 #pragma unroll
   for (int r = 0; r < kRows; ++r) acc[r] = 0.f;
@@ -124,6 +173,25 @@ __global__ void __launch_bounds__(256) pooler_kernel(int B, int L, int H, const 
     const float v = warp_sum(acc[r]);
     if (lane == 0 && r < nb) pooled[(size_t)(b0 + r) * H + j] = tanhf(v + b_p[j]);
   }
+  }
+  if (hc.cnt == nullptr) return;
+  __shared__ int s_last;
+  __syncthreads();  // this CTA's pooled features are written
+  if (threadIdx.x == 0) {
+    __threadfence();
+    s_last = atomicAdd(hc.cnt + blockIdx.y, 1u) == gridDim.x - 1;
+  }
+  __syncthreads();
+  if (!s_last) return;
+  __threadfence();
+  for (int t = warp; t < nb * hc.C; t += kFeat) {
+    const int r = t / hc.C, c = t - r * hc.C;
+    uint4 wv[MAXV];
+    load_wrow<T, MAXV>(wv, (const T*)hc.w_c, c, H, lane);
+    const float s = classifier_dot<T, MAXV>(wv, pooled + (size_t)(b0 + r) * H, nvec, lane);
+    if (lane == 0) hc.logits[(size_t)(b0 + r) * hc.C + c] = s + hc.b_c[c];
+  }
+  if (threadIdx.x == 0) hc.cnt[blockIdx.y] = 0;  // (every CTA of the group has counted itself)
 }
 
 // One warp per (sequence, label): 16-byte loads of the W_c row (before the PDL wait) and of
@@ -139,32 +207,9 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
   const int nvec = H / VN;
   for (int c = warp; c < C; c += 2) {
     uint4 wv[MAXV];
-    const uint4* wr = reinterpret_cast<const uint4*>(w_c + (size_t)c * H);
-#pragma unroll
-    for (int i = 0; i < MAXV; ++i)
-      if (lane + 32 * i < nvec) wv[i] = __ldg(wr + lane + 32 * i);
+    load_wrow<T, MAXV>(wv, w_c, c, H, lane);
     if (c == warp) pdl_wait();
-    const float* p = pooled + (size_t)b * H;
-    float s = 0.f;
-#pragma unroll
-    for (int i = 0; i < MAXV; ++i) {
-      const int v = lane + 32 * i;
-      if (v < nvec) {
-        float w[VN];
-        unpack16<T>(wv[i], w);
-#pragma unroll
-        for (int e = 0; e < VN; e += 4) {
-          const uint4 qu = ld_dep_v4(p + v * VN + e);
-          const float4 q = make_float4(__uint_as_float(qu.x), __uint_as_float(qu.y), __uint_as_float(qu.z),
-                                       __uint_as_float(qu.w));
-          s = fmaf(w[e], q.x, s);
-          s = fmaf(w[e + 1], q.y, s);
-          s = fmaf(w[e + 2], q.z, s);
-          s = fmaf(w[e + 3], q.w, s);
-        }
-      }
-    }
-    s = warp_sum(s);
+    const float s = classifier_dot<T, MAXV>(wv, pooled + (size_t)b * H, nvec, lane);
     if (lane == 0) logits[(size_t)b * C + c] = s + b_c[c];
   }
   if (warp >= C) pdl_wait();
@@ -172,7 +217,7 @@ __global__ void __launch_bounds__(64) classifier_kernel(int H, int C, const floa
 
 template <typename T, int MAXV>
 cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
-                     const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
+                     const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln, unsigned* cnt) {
   const size_t smem = (size_t)kRows * H * sizeof(T);
   static std::atomic<uint64_t> attr_done{0};
   cudaError_t e = once_per_device(attr_done, [] {
@@ -185,35 +230,36 @@ cudaError_t launch_t(int B, int L, int H, int C, const void* x, const void* w_p,
   if (e != cudaSuccess) return e;
   dim3 grid((H + kFeat - 1) / kFeat, (B + kRows - 1) / kRows);
   e = launch_k(pooler_kernel<T, MAXV>, grid, dim3(256), smem, s, B, L, H, (const T*)x, (const T*)w_p,
-                           b_p, pooled, ln);
-  if (e != cudaSuccess) return e;
+                           b_p, pooled, ln, HeadCls{w_c, b_c, logits, C, cnt});
+  if (e != cudaSuccess || cnt != nullptr) return e;
   return launch_k(classifier_kernel<T, MAXV>, dim3(B), dim3(64), 0, s, H, C, (const float*)pooled, (const T*)w_c,
                   b_c, logits);
 }
 
 template <typename T>
 cudaError_t launch_dt(int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p, const void* w_c,
-                      const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
+                      const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln, unsigned* cnt) {
   const int maxv = (H * (int)sizeof(T) + 511) / 512;
   switch (maxv) {
-    case 1: return launch_t<T, 1>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    case 2: return launch_t<T, 2>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    case 3: return launch_t<T, 3>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    case 4: return launch_t<T, 4>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    case 5: case 6: return launch_t<T, 6>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    case 7: case 8: return launch_t<T, 8>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
-    default: return launch_t<T, 16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln);
+    case 1: return launch_t<T, 1>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    case 2: return launch_t<T, 2>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    case 3: return launch_t<T, 3>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    case 4: return launch_t<T, 4>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    case 5: case 6: return launch_t<T, 6>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    case 7: case 8: return launch_t<T, 8>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
+    default: return launch_t<T, 16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt);
   }
 }
 
 }  // namespace
 
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p, const float* b_p,
-                        const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln) {
+                        const void* w_c, const float* b_c, float* pooled, float* logits, cudaStream_t s, HeadLn ln,
+                        unsigned* cnt) {
   if (B <= 0) return cudaSuccess;
   if (H > 2048 || H % 8) return cudaErrorInvalidValue;
-  return dt == DT_BF16 ? launch_dt<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln)
-                       : launch_dt<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, HeadLn{});
+  return dt == DT_BF16 ? launch_dt<bf16>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, ln, cnt)
+                       : launch_dt<float>(B, L, H, C, x, w_p, b_p, w_c, b_c, pooled, logits, s, HeadLn{}, cnt);
 }
 
 }  // namespace arlo

@@ -153,7 +153,9 @@ struct HeadLn {
 };
 cudaError_t launch_head(DType dt, int B, int L, int H, int C, const void* x, const void* w_p,
                         const float* b_p, const void* w_c, const float* b_c, float* pooled,
-                        float* logits, cudaStream_t s, HeadLn ln = HeadLn{});
+                        float* logits, cudaStream_t s, HeadLn ln = HeadLn{}, unsigned* cnt = nullptr);
+// (cnt: [ceil(B / 8)] zero-initialised counters -> the classifier runs in the pooler's last CTA of
+//  each 8-sequence group instead of a second kernel; the runtimes pass their arena's counters)
 
 // ---- fused persistent forward (encoder_fused.cu): the whole batch-1 forward as one kernel ----
 struct FusedPlanImpl;

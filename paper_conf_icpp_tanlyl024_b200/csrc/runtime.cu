@@ -261,6 +261,7 @@ struct arlo_runtime {
   float* logits = nullptr;     // [max_batch * C]
   float* pooled = nullptr;     // [max_batch * H] fp32 pooler output
   unsigned* gbar = nullptr;    // grid barrier of the LayerNorm-prologue GEMMs (zero-initialised)
+  unsigned* head_cnt = nullptr;  // pooler -> classifier arrival counters, one per 8 sequences (zero-initialised)
   void *X = nullptr, *QKV = nullptr, *O = nullptr, *Y = nullptr, *F = nullptr;
   // pinned host staging
   void* h_stage = nullptr;
@@ -309,7 +310,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
     const int l = c.layers - 1;
     HeadLn hl{rt->S2, (const float*)w->lt(l, LN2_G), (const float*)w->lt(l, LN2_B), c.ln_eps, rt->max_batch * L};
     ARLO_CUDA(launch_head(dt, b, bk.cls_prune ? 1 : L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1),
-                          w->hd(2), (const float*)w->hd(3), rt->pooled, rt->logits, s, hl),
+                          w->hd(2), (const float*)w->hd(3), rt->pooled, rt->logits, s, hl, rt->head_cnt),
               "head launch");
     return ARLO_OK;
   }
@@ -366,7 +367,7 @@ static int enqueue_forward(arlo_runtime* rt, Bucket& bk, cudaStream_t s) {
   }
   // the pooler reads position 0 of sequence i at row i*L of X, or row i after a CLS-only last layer
   ARLO_CUDA(launch_head(dt, b, bk.cls_prune ? 1 : L, H, c.num_labels, rt->X, w->hd(0), (const float*)w->hd(1), w->hd(2),
-                        (const float*)w->hd(3), rt->pooled, rt->logits, s),
+                        (const float*)w->hd(3), rt->pooled, rt->logits, s, HeadLn{}, rt->head_cnt),
             "head launch");
   return ARLO_OK;
 }
@@ -714,6 +715,7 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   const size_t off_logits = off; off = al(off + 4 * (size_t)max_batch * c.num_labels);
   const size_t off_pooled = off; off = al(off + 4 * (size_t)max_batch * H);
   const size_t off_gbar = off; off = al(off + 64);
+  const size_t off_hcnt = off; off = al(off + 4 * (size_t)((max_batch + 7) / 8));
   const size_t off_X = off; off = al(off + es * Mmax * H);
   const size_t off_QKV = off; off = al(off + es * Mmax * 3 * H);
   const size_t off_O = off; off = al(off + es * Mmax * H);
@@ -733,6 +735,9 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   rt->logits = (float*)(a + off_logits);
   rt->pooled = (float*)(a + off_pooled);
   rt->gbar = (unsigned*)(a + off_gbar);
+  // classifier in the pooler's last CTA (ARLO_HEAD_IN_POOLER=1): bitwise the same logits, one launch
+  // less, but measured no faster (the last CTA's serial classifier costs what the hop saved)
+  rt->head_cnt = getenv("ARLO_HEAD_IN_POOLER") ? (unsigned*)(a + off_hcnt) : nullptr;
   rt->X = a + off_X; rt->QKV = a + off_QKV; rt->O = a + off_O; rt->Y = a + off_Y; rt->F = a + off_F;
   if (rt->ln_fold) {
     rt->S1 = (float*)(a + off_S1);

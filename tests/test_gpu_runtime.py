@@ -178,7 +178,8 @@ def test_enqueue_matches_infer(arlo_lib):
     rt.enqueue(12, torch.from_numpy(ids).cuda(), torch.from_numpy(lengths).cuda(), out)
     s.synchronize()
     np.testing.assert_array_equal(out.cpu().numpy(), a[:12])
-    assert rt.kernel_count(12) in (3 + 5 * cfg.layers, 3 + 7 * cfg.layers)  # fused / unfused LayerNorm
+    # embedding + 5 or 7 per layer (LayerNorm fold / kernels) + pooler + classifier
+    assert rt.kernel_count(12) in (3 + 5 * cfg.layers, 3 + 7 * cfg.layers)
     rt.close()
 
 
@@ -218,3 +219,39 @@ def test_autotuned_tiles_are_bitwise_the_analytic_choice(arlo_lib, monkeypatch):
     monkeypatch.setenv("ARLO_NO_AUTOTUNE", "1")
     out_plain = run(arlo_lib, W, L, mb, ids, lengths)
     assert np.array_equal(out_tuned, out_plain)
+
+
+@pytest.mark.parametrize("dtype", [0, 1])
+def test_head_classifier_in_pooler_is_bitwise(arlo_lib, monkeypatch, dtype):
+    """ARLO_HEAD_IN_POOLER=1: the classifier runs in the pooler's last CTA of each 8-sequence group
+    (one launch less per forward); its logits are bitwise those of the separate classifier kernel
+    (the default), for groups of 8 and a ragged last group, over repeated replays (the arrival
+    counters reset themselves)."""
+    monkeypatch.setenv("ARLO_HEAD_IN_POOLER", "1")
+    cfg = wl.BERT_BASE
+    w, W = weights(arlo_lib, cfg, dtype)
+    lengths = wl.sample_lengths(21, seed=61, lo=0, hi=128)
+    ids = wl.sample_token_ids(cfg, lengths, 128, seed=62)
+    n, L, mb = len(lengths), 128, 24
+    ids_full = np.zeros((mb, L), np.int32)
+    ids_full[:n] = ids
+    len_full = np.zeros(mb, np.int32)
+    len_full[:n] = lengths
+    rt = arlo_lib.Runtime(W, L, mb)
+    fused = []
+    for _ in range(3):  # same runtime: the counters must have reset after each forward
+        out = np.full((mb, 2), np.nan, np.float32)
+        rt.infer(ids_full, len_full, out)
+        fused.append(out[:n].copy())
+    k_fused = rt.kernel_count(n)
+    rt.close()
+    monkeypatch.delenv("ARLO_HEAD_IN_POOLER")
+    rt2 = arlo_lib.Runtime(W, L, mb)
+    two = np.full((mb, 2), np.nan, np.float32)
+    rt2.infer(ids_full, len_full, two)
+    assert rt2.kernel_count(n) == k_fused + 1
+    rt2.close()
+    for f in fused:
+        np.testing.assert_array_equal(f, two[:n])
+    ref = orc.forward_batch(cfg, w, ids, lengths)
+    assert np.max(np.abs(two[:n] - ref)) <= (2e-2 if dtype == 0 else 1e-4)
