@@ -42,11 +42,15 @@ def derive_runtime_set(curve: dict, tol: float = 0.05, max_len: int = 512):
 
 
 def capacities(per_L_ms: dict, slo_ms: float, max_batch: int):
-    """M_i: largest profiled batch whose forward latency fits the SLO (>= 1)."""
+    """M_i per runtime for Algorithm 1's congestion P = N / M, the same reading
+    as the cluster replays (reading S18, slo_capacity): the requests one instance finishes inside one
+    SLO window with every batch meeting the SLO.  per_L_ms[L] = {batch: profiled latency ms}; batches
+    missing from the profile are interpolated linearly (reading S15)."""
     caps = {}
     for L, row in per_L_ms.items():
-        ok = [b for b, ms in row.items() if ms <= slo_ms]
-        caps[L] = max(ok) if ok else 1
+        bs = sorted(row)
+        lat = np.interp(np.arange(1, max_batch + 1), bs, [row[b] for b in bs])
+        caps[L] = slo_capacity(lat, slo_ms)
     return caps
 
 
