@@ -175,7 +175,7 @@ int arlo_enqueue(arlo_runtime* rt, int32_t n, const int32_t* token_ids, const in
                  float* logits);
 
 /* Batch bucket (captured graph size) that serves n requests: the smallest of
- * 1, 2, 4, 8, 12, 16, ..., 32 (every 4), 40, 48, ... (every 8), max_batch that is >= n.
+ * 1, 2, 4, 6, 8, ..., 32 (every 2), 40, 48, ... (every 8), max_batch that is >= n.
  * EINVAL unless 1 <= n <= max_batch. */
 int32_t arlo_runtime_bucket(const arlo_runtime* rt, int32_t n);
 

@@ -749,14 +749,16 @@ extern "C" int arlo_runtime_create_ex(int32_t L, int32_t max_batch, const arlo_w
   e = cudaMallocHost(&rt->h_stage, rt->h_stage_bytes);
   if (e != cudaSuccess) return fail(set_error(ARLO_ENOMEM, "pinned staging: %s", cudaGetErrorString(e)));
 
-  // batch buckets 1, 2, 4, 8, then every multiple of 4 up to 32 and of 8 beyond, and max_batch: a
-  // partly filled batch pads to at most 3 empty slots below 32 (7 above).  The padded slots are
-  // computed for nothing (the batch dimension's padding waste); multiples of 8
-  // left up to 7 (e.g. 17 requests in a 24 bucket).  ARLO_BUCKET_STEP8=1: the round-1 set.
+  // batch buckets 1, 2, 4, then every multiple of `step` (2) up to 32 and of 8 beyond, and max_batch:
+  // a partly filled batch pads to at most step - 1 empty slots below 32 (7 above).  The padded slots
+  // are computed for nothing (the batch dimension's padding waste); round 1's
+  // multiples of 8 left up to 7 (e.g. 17 requests in a 24 bucket).  ARLO_BUCKET_STEP=4 / 8: coarser.
   std::vector<int> bs;
-  const int fine = getenv("ARLO_BUCKET_STEP8") ? 8 : 4;
-  for (int b = 1; b < max_batch && b < 8; b *= 2) bs.push_back(b);
-  for (int b = 8; b < max_batch; b += (b < 32 ? fine : 8)) bs.push_back(b);
+  int step = 2;
+  if (const char* e = getenv("ARLO_BUCKET_STEP")) step = atoi(e) >= 1 ? atoi(e) : 2;
+  if (getenv("ARLO_BUCKET_STEP8")) step = 8;
+  for (int b = 1; b < max_batch && b <= 4; b *= 2) bs.push_back(b);
+  for (int b = step < 4 ? 4 + step : 8; b < max_batch; b += (b < 32 ? step : 8)) bs.push_back(b);
   bs.push_back(max_batch);
   rt->buckets.resize(bs.size());
   for (size_t i = 0; i < bs.size(); ++i) {
